@@ -1,0 +1,190 @@
+/*
+ * cudanp.h -- C ABI of the B200-native CUDA-NP hot path (libcudanp.so).
+ *
+ * Paper: Y. Yang, H. Zhou, "CUDA-NP: Realizing Nested Thread-Level
+ * Parallelism in GPGPU Applications", PPoPP'14.  "P:n" = line n of the
+ * paper text; "Rn" = reading n in DESIGN.md.
+ *
+ * The problem: N independent outer work items
+ * (the original GPU threads, "masters"), each running sequential code plus a
+ * parallel inner loop of runtime trip count L with an optional
+ * reduction or scan.  Each call runs hand-written sm_100a
+ * master/slave kernels: a team of S threads (S counts the master, P:180;
+ * S in {1,2,4,8,16,32}) shares each item's loop, with
+ *   dist: CUDANP_DIST_CYCLIC or CUDANP_DIST_BLOCK (R5), and
+ *   map : CUDANP_MAP_INTRA_WARP (team = S lanes of one warp) or
+ *         CUDANP_MAP_INTER_WARP (team = one lane in each of S warps)
+ *         (P:189-191), CUDANP_MAP_AUTO choosing per the rules of P:340-342.
+ * S = 1 means no nesting: the tuned one-thread-per-item kernel.
+ *
+ * Conventions for every call:
+ *  - Data pointers are DEVICE pointers owned by the caller; the library never
+ *    allocates, frees or retains them.  Matrices and item arrays are
+ *    row-major fp32/int32.  Outputs must not overlap inputs.
+ *  - `stream` is a cudaStream_t passed as void* (NULL = legacy default
+ *    stream).  Calls validate their arguments synchronously, enqueue work on
+ *    `stream` and return without synchronizing.  No C++ exception crosses
+ *    the ABI.  The functions keep no state and are thread-safe.
+ *  - Return value: a cudanp_status.  CUDANP_ERR_INVALID is returned before
+ *    any launch (no partial work).  CUDANP_ERR_CUDA reports a launch error
+ *    (text in cudanp_last_error()); faults during asynchronous execution
+ *    surface at the caller's next synchronization.
+ *  - N = 0 or L = 0 is valid: reduce writes init (or the identity) for each
+ *    item, scan writes nothing, TMV/MV write 0 when the inner count is 0.
+ *  - Misaligned pointers or leading dimensions that are not multiples of 4
+ *    are not errors; they take the scalar (non-128-bit) path.
+ */
+#ifndef CUDANP_H_
+#define CUDANP_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+  CUDANP_OK = 0,
+  CUDANP_ERR_INVALID = 1,     /* bad argument; nothing launched            */
+  CUDANP_ERR_UNSUPPORTED = 2, /* valid but not built (e.g. intra-warp S=3) */
+  CUDANP_ERR_CUDA = 3,        /* CUDA runtime error at launch              */
+  CUDANP_ERR_NCCL = 4         /* reserved for collective errors            */
+} cudanp_status;
+
+typedef enum { CUDANP_DIST_CYCLIC = 0, CUDANP_DIST_BLOCK = 1 } cudanp_dist;
+typedef enum { CUDANP_MAP_AUTO = 0, CUDANP_MAP_INTRA_WARP = 1, CUDANP_MAP_INTER_WARP = 2 } cudanp_map;
+typedef enum { CUDANP_F32 = 0, CUDANP_I32 = 1 } cudanp_dtype;
+typedef enum { CUDANP_SUM = 0, CUDANP_MAX = 1 } cudanp_op;
+
+/* ------------------------------------------------------------------------
+ * The four hot-path calls (north star).
+ * ---------------------------------------------------------------------- */
+
+/* TMV, Fig 2: y[j] = sum_{i<n_inner} A[i*lda + j] * x[i], for
+ * j < n_outer.  Master = column j (one output per master); the inner loop
+ * runs over the h = n_inner rows.  A: n_inner x lda fp32 (lda >= n_outer),
+ * x: n_inner fp32, y: n_outer fp32.  fp32 FMA accumulation; the S partial
+ * sums are combined by the team reduction. */
+int cudanp_tmv(const float* A, int64_t lda, const float* x, float* y,
+               int64_t n_outer, int64_t n_inner, int S, int dist, int map, void* stream);
+
+/* MV (Table 1 "MV"): y[i] = sum_{j<n_inner} A[i*lda + j] * x[j],
+ * for i < n_outer.  Master = row i; inner loop over the w = n_inner columns.
+ * A: n_outer x lda fp32 (lda >= n_inner), x: n_inner, y: n_outer. */
+int cudanp_mv(const float* A, int64_t lda, const float* x, float* y,
+              int64_t n_outer, int64_t n_inner, int S, int dist, int map, void* stream);
+
+/* Batched loop-reduce (reduction clause; Fig 6d):
+ * out[n] = init[n] (op) fold_{i<L} in[n*L + i] for n < N = n_outer,
+ * L = n_inner.  Item-major [N][L] layout.  dtype CUDANP_F32 or CUDANP_I32;
+ * op CUDANP_SUM (int32 wraps modulo 2^32, R13) or CUDANP_MAX (identity -inf /
+ * INT32_MIN, R14).  init may be NULL (identity).  The master loads init[n]
+ * and stores out[n]. */
+int cudanp_batched_loop_reduce(const void* in, const void* init, void* out,
+                               int64_t n_outer, int64_t n_inner, int dtype, int op,
+                               int S, int dist, int map, void* stream);
+
+/* Batched inclusive scan (scan clause; inclusive per R1):
+ * out[n*L + k] = init[n] + sum_{i<=k} in[n*L + i].  init may be NULL (0);
+ * when given, the master loads it and broadcasts it to its slaves with
+ * read_from_master.  Every team member stores its own elements. */
+int cudanp_batched_loop_scan(const void* in, const void* init, void* out,
+                             int64_t n_outer, int64_t n_inner, int dtype,
+                             int S, int dist, int map, void* stream);
+
+/* ------------------------------------------------------------------------
+ * Comparison kernels.  Same operands as the NP
+ * call; `impl` selects:
+ *   CUDANP_IMPL_S1_LITERAL: Fig 2 verbatim -- one thread per item, scalar
+ *       serial loop, no vector loads;
+ *   CUDANP_IMPL_DP_THREAD : CUDA dynamic parallelism (CDP2): every master
+ *       launches a child grid for its loop; the child stores the result;
+ *   CUDANP_IMPL_DP_BLOCK  : DP with one child launch per thread block (the
+ *       paper's manual optimisation).
+ * DP variants need enough device-runtime launch slots: see
+ * cudanp_dp_set_pending_launch_limit.  A DP launch that the device runtime
+ * refuses sets a device error flag; cudanp_dp_error_count() reads it.
+ * ---------------------------------------------------------------------- */
+typedef enum {
+  CUDANP_IMPL_S1_LITERAL = 1,
+  CUDANP_IMPL_DP_THREAD = 2,
+  CUDANP_IMPL_DP_BLOCK = 3
+} cudanp_impl;
+
+int cudanp_tmv_variant(int impl, const float* A, int64_t lda, const float* x, float* y,
+                       int64_t n_outer, int64_t n_inner, void* stream);
+int cudanp_mv_variant(int impl, const float* A, int64_t lda, const float* x, float* y,
+                      int64_t n_outer, int64_t n_inner, void* stream);
+int cudanp_batched_loop_reduce_variant(int impl, const void* in, const void* init, void* out,
+                                       int64_t n_outer, int64_t n_inner, int dtype, int op,
+                                       void* stream);
+int cudanp_batched_loop_scan_variant(int impl, const void* in, const void* init, void* out,
+                                     int64_t n_outer, int64_t n_inner, int dtype, void* stream);
+/* cudaDeviceSetLimit(cudaLimitDevRuntimePendingLaunchCount, n) on the
+ * current device. */
+int cudanp_dp_set_pending_launch_limit(size_t n);
+/* Number of device-side child launches that failed since the last reset
+ * (synchronizes the device); reset = 1 clears the counter. */
+int cudanp_dp_error_count(int reset, int64_t* count_out);
+
+/* ------------------------------------------------------------------------
+ * Launch shape actually used (the paper's resource analysis, Table 1 P:96,
+ * and autotune space P:384): for an NP call with these arguments,
+ * report the kernel's block size, grid size, registers per thread, static
+ * shared memory bytes and the resolved map.  `op_kind`: 0 tmv, 1 mv,
+ * 2 reduce, 3 scan.  Any out pointer may be NULL.
+ * ---------------------------------------------------------------------- */
+int cudanp_launch_info(int op_kind, int64_t n_outer, int64_t n_inner, int dtype, int op,
+                       int S, int dist, int map, int vec4,
+                       int* block_threads, int64_t* grid_ctas, int* regs_per_thread,
+                       int* smem_bytes, int* resolved_map);
+
+/* ------------------------------------------------------------------------
+ * Multi-GPU helper (one process per GPU; outer items are independent,
+ * P:13): the contiguous range [floor(g*N/G), floor((g+1)*N/G)) that
+ * rank g of G owns.
+ * ---------------------------------------------------------------------- */
+int cudanp_shard_range(int64_t n_outer, int nranks, int rank, int64_t* begin, int64_t* end);
+
+/* ------------------------------------------------------------------------
+ * Test and benchmark support (not part of the method).
+ * ---------------------------------------------------------------------- */
+
+/* Device-side counter-based input generator:
+ * out[r*ld + c] = value(kind, splitmix64(splitmix64(seed ^ (stream_id<<56))
+ * ^ ((row0 + r) * w_global + col0 + c))) for r < rows, c < cols.
+ * kind: 0 f32_unit, 1 f32_signed, 2 f32_int4, 3 i32_small (parameter B),
+ * 4 i32_full, 5 ones (fp32), 6 ones (int32).  B must be a power of two. */
+int cudanp_generate(void* out, int64_t rows, int64_t cols, int64_t ld, int64_t row0,
+                    int64_t col0, int64_t w_global, int stream_id, int kind, int64_t B,
+                    uint64_t seed, void* stream);
+
+/* Runs the kernels' own iteration-distribution code on the device and copies
+ * owner[u*V + k] = slave that executes element u*V+k of a loop of n_inner
+ * elements back to the HOST array owner_host (n_inner int32).  V in {1,4}.
+ * Synchronous. */
+int cudanp_debug_owner_map(int64_t n_inner, int S, int dist, int V, int32_t* owner_host);
+
+/* Runs the kernels' own team formation for one CTA of `map` with team size S
+ * on the device and copies master/slave ids of each linear thread id to the
+ * HOST arrays (nthreads = 32*S for inter-warp, 32 for intra-warp).
+ * Synchronous.  Returns the thread count through *nthreads. */
+int cudanp_debug_team_ids(int S, int map, int32_t* master_host, int32_t* slave_host,
+                          int* nthreads);
+
+/* Runs read_from_master on the device: for each team of a warp (intra) or
+ * CTA (inter), every member returns the value its master held; values[t] =
+ * 1000*t + 7 before, out_host[t] after.  Synchronous. */
+int cudanp_debug_broadcast(int S, int map, int32_t* out_host, int* nthreads);
+
+const char* cudanp_status_string(int status);
+/* Detail text for the last non-OK return on this host thread. */
+const char* cudanp_last_error(void);
+/* Library version as major*10000 + minor*100 + patch. */
+int cudanp_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* CUDANP_H_ */

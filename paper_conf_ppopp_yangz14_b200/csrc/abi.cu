@@ -1,0 +1,440 @@
+// abi.cu -- the extern "C" boundary of libcudanp.so (include/cudanp.h):
+// argument validation before any launch, choice of map / vector path,
+// dispatch to the kernels, status codes and error text.  Also the device-side
+// input generator and the debug exports that run the kernels' own team and
+// distribution code.
+#include <cstdarg>
+#include <cstdlib>
+
+#include "common.cuh"
+#include "np_team.cuh"
+
+namespace cudanp {
+
+// ---- kernels' host entry points (np_reduce.cu, np_scan.cu, np_matvec.cu, np_dp.cu)
+int reduce_np(const void*, const void*, void*, int64_t, int64_t, int, int, int, int, int, bool,
+              cudaStream_t, LaunchInfo*);
+int reduce_literal(const void*, const void*, void*, int64_t, int64_t, int, int, cudaStream_t);
+int scan_np(const void*, const void*, void*, int64_t, int64_t, int, int, int, int, bool,
+            cudaStream_t, LaunchInfo*);
+int scan_literal(const void*, const void*, void*, int64_t, int64_t, int, cudaStream_t);
+int tmv_np(const float*, int64_t, const float*, float*, int64_t, int64_t, int, int, int, bool,
+           cudaStream_t, LaunchInfo*);
+int mv_np(const float*, int64_t, const float*, float*, int64_t, int64_t, int, int, int, bool,
+          cudaStream_t, LaunchInfo*);
+int tmv_literal(const float*, int64_t, const float*, float*, int64_t, int64_t, cudaStream_t);
+int mv_literal(const float*, int64_t, const float*, float*, int64_t, int64_t, cudaStream_t);
+int dp_tmv(bool, const float*, int64_t, const float*, float*, int64_t, int64_t, cudaStream_t);
+int dp_mv(bool, const float*, int64_t, const float*, float*, int64_t, int64_t, cudaStream_t);
+int dp_reduce(bool, const void*, const void*, void*, int64_t, int64_t, int, int, cudaStream_t);
+int dp_scan(bool, const void*, const void*, void*, int64_t, int64_t, int, cudaStream_t);
+int dp_error_count(int, int64_t*);
+
+static thread_local char g_err[512] = "";
+
+void set_error(const char* fmt, ...) {
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(g_err, sizeof(g_err), fmt, ap);
+  va_end(ap);
+}
+void clear_error() { g_err[0] = 0; }
+
+int sm_count() {
+  static int cache[64] = {0};
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess) { cudaGetLastError(); return 148; }
+  if (dev < 0 || dev >= 64) dev = 0;
+  if (!cache[dev]) {
+    int n = 0;
+    if (cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || n < 1) {
+      cudaGetLastError();
+      n = 148;
+    }
+    cache[dev] = n;
+  }
+  return cache[dev];
+}
+
+// ---------------------------------------------------------------- validation
+static bool size_ok(int64_t a, int64_t b) {  // a*b*4 bytes addressable
+  if (a < 0 || b < 0) return false;
+  if (a == 0 || b == 0) return true;
+  return a <= (INT64_MAX / 8) / b;
+}
+
+static int check_common(int S, int dist, int map, int64_t n_outer, int64_t n_inner) {
+  if (!valid_S(S)) return fail_invalid("S must be one of 1,2,4,8,16,32");
+  if (dist != CUDANP_DIST_CYCLIC && dist != CUDANP_DIST_BLOCK) return fail_invalid("dist");
+  if (map != CUDANP_MAP_AUTO && map != CUDANP_MAP_INTRA_WARP && map != CUDANP_MAP_INTER_WARP)
+    return fail_invalid("map");
+  if (n_outer < 0 || n_inner < 0) return fail_invalid("negative size");
+  if (!size_ok(n_outer, n_inner)) return fail_invalid("size overflows int64 byte offsets");
+  return CUDANP_OK;
+}
+
+static int check_dtype_op(int dtype, int op) {
+  if (dtype != CUDANP_F32 && dtype != CUDANP_I32) return fail_invalid("dtype");
+  if (op != CUDANP_SUM && op != CUDANP_MAX) return fail_invalid("op");
+  return CUDANP_OK;
+}
+
+// MAP_AUTO per P:340-342 / P:486: keep the access pattern coalesced.  TMV's
+// masters (columns) are adjacent in memory -> inter-warp; MV rows and
+// item-major reduce/scan rows are contiguous per master -> intra-warp.
+static int resolve_map(int map, bool is_tmv) {
+  if (map != CUDANP_MAP_AUTO) return map;
+  return is_tmv ? MAP_INTER : MAP_INTRA;
+}
+
+static int check_tmv_args(const float* A, int64_t lda, const float* x, float* y, int64_t w,
+                          int64_t h, int S, int dist, int map) {
+  int rc = check_common(S, dist, map, w, h);
+  if (rc) return rc;
+  if (w > 0 && h > 0 && lda < w) return fail_invalid("lda < n_outer (TMV row length)");
+  if (!size_ok(h, lda)) return fail_invalid("h*lda overflows");
+  if (w > 0 && !y) return fail_invalid("y is NULL");
+  if (w > 0 && h > 0 && (!A || !x)) return fail_invalid("A or x is NULL");
+  return CUDANP_OK;
+}
+
+static int check_mv_args(const float* A, int64_t lda, const float* x, float* y, int64_t h,
+                         int64_t w, int S, int dist, int map) {
+  int rc = check_common(S, dist, map, h, w);
+  if (rc) return rc;
+  if (h > 0 && w > 0 && lda < w) return fail_invalid("lda < n_inner (MV row length)");
+  if (!size_ok(h, lda)) return fail_invalid("h*lda overflows");
+  if (h > 0 && !y) return fail_invalid("y is NULL");
+  if (h > 0 && w > 0 && (!A || !x)) return fail_invalid("A or x is NULL");
+  return CUDANP_OK;
+}
+
+static bool tmv_vec(const float* A, int64_t lda, const float* y, int64_t w) {
+  return (w % 4 == 0) && (lda % 4 == 0) && aligned16(A) && aligned16(y);
+}
+static bool mv_vec(const float* A, int64_t lda, const float* x, int64_t w) {
+  return (w % 4 == 0) && (lda % 4 == 0) && aligned16(A) && aligned16(x);
+}
+
+// ---------------------------------------------------------------- generator
+// Counter-based generator, written independently of the
+// oracle's copy; tests check the two agree bit for bit.
+__host__ __device__ __forceinline__ uint64_t mix64(uint64_t z) {
+  z += 0x9E3779B97F4A7C15ull;
+  z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+  z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+  return z ^ (z >> 31);
+}
+
+__global__ void generate_kernel(void* out, int64_t rows, int64_t cols, int64_t ld, int64_t row0,
+                                int64_t col0, int64_t wg, uint64_t key, int kind, int64_t B) {
+  const int64_t total = rows * cols;
+  for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < total;
+       e += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t r = e / cols, c = e - r * cols;
+    const uint64_t idx = (uint64_t)(row0 + r) * (uint64_t)wg + (uint64_t)(col0 + c);
+    const uint64_t h = mix64(key ^ idx);
+    const int64_t o = r * ld + c;
+    switch (kind) {
+      case 0: ((float*)out)[o] = (float)(h >> 40 | 1ull) * 0x1p-24f; break;
+      case 1: ((float*)out)[o] = (float)((int64_t)(h >> 40 | 1ull) * 2 - (1ll << 24)) * 0x1p-24f; break;
+      case 2: ((float*)out)[o] = (float)(h >> 62); break;
+      case 3: ((int32_t*)out)[o] = (int32_t)((int64_t)((h >> 32) & (uint64_t)(2 * B - 1)) - B); break;
+      case 4: ((int32_t*)out)[o] = (int32_t)(uint32_t)(h >> 32); break;
+      case 5: ((float*)out)[o] = 1.0f; break;
+      case 6: ((int32_t*)out)[o] = 1; break;
+      default: break;
+    }
+  }
+}
+
+// ---------------------------------------------------------------- debug kernels
+// Each uses the very Range / IntraTeam / InterTeam code the kernels use.
+template <int S, int DIST>
+__global__ void owner_kernel(int64_t L, int V, int32_t* owner) {
+  const int s = threadIdx.x;
+  const int64_t nunits = (L + V - 1) / V;
+  const Range<S, DIST> r(nunits, L, V, s);
+  for (int64_t u = r.begin; u < r.end; u += r.step)
+    for (int k = 0; k < V; ++k)
+      if (u * V + k < L) owner[u * V + k] = s;
+}
+
+template <int S>
+__global__ void team_intra_kernel(int32_t* master, int32_t* slave) {
+  const IntraTeam<S> t;
+  const int tid = threadIdx.x;
+  master[tid] = (tid >> 5) * IntraTeam<S>::kTeamsPerWarp + t.team;
+  slave[tid] = t.slave;
+}
+template <int S>
+__global__ void team_inter_kernel(int32_t* master, int32_t* slave) {
+  const InterTeam<S> t;
+  const int tid = threadIdx.y * 32 + threadIdx.x;
+  master[tid] = t.master;
+  slave[tid] = t.slave;
+}
+template <int S>
+__global__ void bcast_intra_kernel(int32_t* out) {
+  const IntraTeam<S> t;
+  const int tid = threadIdx.x;
+  out[tid] = t.read_from_master((int32_t)(1000 * tid + 7));
+}
+template <int S>
+__global__ void bcast_inter_kernel(int32_t* out) {
+  __shared__ int32_t slot[32];
+  const InterTeam<S> t;
+  const int tid = threadIdx.y * 32 + threadIdx.x;
+  out[tid] = t.read_from_master((int32_t)(1000 * tid + 7), slot);
+}
+
+}  // namespace cudanp
+
+using namespace cudanp;
+
+static cudaStream_t as_stream(void* s) { return (cudaStream_t)s; }
+
+extern "C" {
+
+int cudanp_version(void) { return 100; }
+
+const char* cudanp_status_string(int status) {
+  switch (status) {
+    case CUDANP_OK: return "CUDANP_OK";
+    case CUDANP_ERR_INVALID: return "CUDANP_ERR_INVALID";
+    case CUDANP_ERR_UNSUPPORTED: return "CUDANP_ERR_UNSUPPORTED";
+    case CUDANP_ERR_CUDA: return "CUDANP_ERR_CUDA";
+    case CUDANP_ERR_NCCL: return "CUDANP_ERR_NCCL";
+    default: return "CUDANP_UNKNOWN_STATUS";
+  }
+}
+
+const char* cudanp_last_error(void) { return g_err; }
+
+int cudanp_tmv(const float* A, int64_t lda, const float* x, float* y, int64_t n_outer,
+               int64_t n_inner, int S, int dist, int map, void* stream) {
+  int rc = check_tmv_args(A, lda, x, y, n_outer, n_inner, S, dist, map);
+  if (rc) return rc;
+  return tmv_np(A, lda, x, y, n_outer, n_inner, S, dist, resolve_map(map, true),
+                tmv_vec(A, lda, y, n_outer), as_stream(stream), nullptr);
+}
+
+int cudanp_mv(const float* A, int64_t lda, const float* x, float* y, int64_t n_outer,
+              int64_t n_inner, int S, int dist, int map, void* stream) {
+  int rc = check_mv_args(A, lda, x, y, n_outer, n_inner, S, dist, map);
+  if (rc) return rc;
+  return mv_np(A, lda, x, y, n_outer, n_inner, S, dist, resolve_map(map, false),
+               mv_vec(A, lda, x, n_inner), as_stream(stream), nullptr);
+}
+
+// out_per_item: reduce writes one value per item even when L = 0; scan
+// writes N*L values, so out may be NULL when L = 0.
+static int check_batched(const void* in, void* out, int64_t N, int64_t L, int S, int dist, int map,
+                         int dtype, int op, bool out_per_item) {
+  int rc = check_common(S, dist, map, N, L);
+  if (rc) return rc;
+  rc = check_dtype_op(dtype, op);
+  if (rc) return rc;
+  if (N > 0 && (out_per_item || L > 0) && !out) return fail_invalid("out is NULL");
+  if (N > 0 && L > 0 && !in) return fail_invalid("in is NULL");
+  return CUDANP_OK;
+}
+
+int cudanp_batched_loop_reduce(const void* in, const void* init, void* out, int64_t n_outer,
+                               int64_t n_inner, int dtype, int op, int S, int dist, int map,
+                               void* stream) {
+  int rc = check_batched(in, out, n_outer, n_inner, S, dist, map, dtype, op, true);
+  if (rc) return rc;
+  const bool vec = (n_inner % 4 == 0) && aligned16(in);
+  return reduce_np(in, init, out, n_outer, n_inner, dtype, op, S, dist, resolve_map(map, false),
+                   vec, as_stream(stream), nullptr);
+}
+
+int cudanp_batched_loop_scan(const void* in, const void* init, void* out, int64_t n_outer,
+                             int64_t n_inner, int dtype, int S, int dist, int map, void* stream) {
+  int rc = check_batched(in, out, n_outer, n_inner, S, dist, map, dtype, CUDANP_SUM, false);
+  if (rc) return rc;
+  const bool vec = (n_inner % 4 == 0) && aligned16(in) && aligned16(out);
+  return scan_np(in, init, out, n_outer, n_inner, dtype, S, dist, resolve_map(map, false), vec,
+                 as_stream(stream), nullptr);
+}
+
+// ---------------------------------------------------------------- variants
+static int check_impl(int impl) {
+  if (impl != CUDANP_IMPL_S1_LITERAL && impl != CUDANP_IMPL_DP_THREAD && impl != CUDANP_IMPL_DP_BLOCK)
+    return fail_invalid("impl");
+  return CUDANP_OK;
+}
+
+int cudanp_tmv_variant(int impl, const float* A, int64_t lda, const float* x, float* y,
+                       int64_t n_outer, int64_t n_inner, void* stream) {
+  int rc = check_impl(impl);
+  if (!rc) rc = check_tmv_args(A, lda, x, y, n_outer, n_inner, 1, 0, 0);
+  if (rc) return rc;
+  if (impl == CUDANP_IMPL_S1_LITERAL) return tmv_literal(A, lda, x, y, n_outer, n_inner, as_stream(stream));
+  return dp_tmv(impl == CUDANP_IMPL_DP_BLOCK, A, lda, x, y, n_outer, n_inner, as_stream(stream));
+}
+
+int cudanp_mv_variant(int impl, const float* A, int64_t lda, const float* x, float* y,
+                      int64_t n_outer, int64_t n_inner, void* stream) {
+  int rc = check_impl(impl);
+  if (!rc) rc = check_mv_args(A, lda, x, y, n_outer, n_inner, 1, 0, 0);
+  if (rc) return rc;
+  if (impl == CUDANP_IMPL_S1_LITERAL) return mv_literal(A, lda, x, y, n_outer, n_inner, as_stream(stream));
+  return dp_mv(impl == CUDANP_IMPL_DP_BLOCK, A, lda, x, y, n_outer, n_inner, as_stream(stream));
+}
+
+int cudanp_batched_loop_reduce_variant(int impl, const void* in, const void* init, void* out,
+                                       int64_t n_outer, int64_t n_inner, int dtype, int op,
+                                       void* stream) {
+  int rc = check_impl(impl);
+  if (!rc) rc = check_batched(in, out, n_outer, n_inner, 1, 0, 0, dtype, op, true);
+  if (rc) return rc;
+  if (impl == CUDANP_IMPL_S1_LITERAL)
+    return reduce_literal(in, init, out, n_outer, n_inner, dtype, op, as_stream(stream));
+  return dp_reduce(impl == CUDANP_IMPL_DP_BLOCK, in, init, out, n_outer, n_inner, dtype, op,
+                   as_stream(stream));
+}
+
+int cudanp_batched_loop_scan_variant(int impl, const void* in, const void* init, void* out,
+                                     int64_t n_outer, int64_t n_inner, int dtype, void* stream) {
+  int rc = check_impl(impl);
+  if (!rc) rc = check_batched(in, out, n_outer, n_inner, 1, 0, 0, dtype, CUDANP_SUM, false);
+  if (rc) return rc;
+  if (impl == CUDANP_IMPL_S1_LITERAL)
+    return scan_literal(in, init, out, n_outer, n_inner, dtype, as_stream(stream));
+  return dp_scan(impl == CUDANP_IMPL_DP_BLOCK, in, init, out, n_outer, n_inner, dtype,
+                 as_stream(stream));
+}
+
+int cudanp_dp_set_pending_launch_limit(size_t n) {
+  if (cudaDeviceSetLimit(cudaLimitDevRuntimePendingLaunchCount, n) != cudaSuccess)
+    return check_launch("cudaDeviceSetLimit(DevRuntimePendingLaunchCount)");
+  return CUDANP_OK;
+}
+
+int cudanp_dp_error_count(int reset, int64_t* count_out) { return dp_error_count(reset, count_out); }
+
+// ---------------------------------------------------------------- launch info
+int cudanp_launch_info(int op_kind, int64_t n_outer, int64_t n_inner, int dtype, int op, int S,
+                       int dist, int map, int vec4, int* block_threads, int64_t* grid_ctas,
+                       int* regs_per_thread, int* smem_bytes, int* resolved_map) {
+  int rc = check_common(S, dist, map, n_outer, n_inner);
+  if (rc) return rc;
+  LaunchInfo info;
+  const bool v = vec4 != 0;
+  const int m = resolve_map(map, op_kind == 0);
+  switch (op_kind) {
+    case 0: rc = tmv_np(nullptr, 0, nullptr, nullptr, n_outer, n_inner, S, dist, m, v, 0, &info); break;
+    case 1: rc = mv_np(nullptr, 0, nullptr, nullptr, n_outer, n_inner, S, dist, m, v, 0, &info); break;
+    case 2:
+      rc = check_dtype_op(dtype, op);
+      if (!rc) rc = reduce_np(nullptr, nullptr, nullptr, n_outer, n_inner, dtype, op, S, dist, m, v, 0, &info);
+      break;
+    case 3:
+      rc = check_dtype_op(dtype, CUDANP_SUM);
+      if (!rc) rc = scan_np(nullptr, nullptr, nullptr, n_outer, n_inner, dtype, S, dist, m, v, 0, &info);
+      break;
+    default: return fail_invalid("op_kind");
+  }
+  if (rc) return rc;
+  if (block_threads) *block_threads = info.block_threads;
+  if (grid_ctas) *grid_ctas = info.grid;
+  if (regs_per_thread) *regs_per_thread = info.regs;
+  if (smem_bytes) *smem_bytes = info.smem;
+  if (resolved_map) *resolved_map = info.map;
+  return CUDANP_OK;
+}
+
+// ---------------------------------------------------------------- sharding
+int cudanp_shard_range(int64_t n_outer, int nranks, int rank, int64_t* begin, int64_t* end) {
+  if (n_outer < 0 || nranks < 1 || rank < 0 || rank >= nranks || !begin || !end)
+    return fail_invalid("shard_range arguments");
+  *begin = (int64_t)(((__int128)rank * n_outer) / nranks);
+  *end = (int64_t)(((__int128)(rank + 1) * n_outer) / nranks);
+  return CUDANP_OK;
+}
+
+// ---------------------------------------------------------------- test support
+int cudanp_generate(void* out, int64_t rows, int64_t cols, int64_t ld, int64_t row0, int64_t col0,
+                    int64_t w_global, int stream_id, int kind, int64_t B, uint64_t seed,
+                    void* stream) {
+  if (rows < 0 || cols < 0 || ld < cols || row0 < 0 || col0 < 0 || w_global < 0)
+    return fail_invalid("generate sizes");
+  if (kind < 0 || kind > 6) return fail_invalid("generate kind");
+  if (kind == 3 && (B < 1 || (B & (B - 1)))) return fail_invalid("generate B must be a power of two");
+  if (rows * cols == 0) return CUDANP_OK;
+  if (!out) return fail_invalid("generate out is NULL");
+  const uint64_t key = mix64(seed ^ ((uint64_t)stream_id << 56));
+  const int64_t total = rows * cols;
+  int64_t grid = (total + 255) / 256;
+  const int64_t cap = (int64_t)sm_count() * 16;
+  if (grid > cap) grid = cap;
+  generate_kernel<<<(unsigned)grid, 256, 0, as_stream(stream)>>>(out, rows, cols, ld, row0, col0,
+                                                                 w_global, key, kind, B);
+  return check_launch("generate launch");
+}
+
+}  // extern "C"
+
+extern "C" {
+
+static int copy_back(void* dst, const void* src, size_t bytes, const char* what) {
+  if (cudaDeviceSynchronize() != cudaSuccess) return check_launch(what);
+  if (cudaMemcpy(dst, src, bytes, cudaMemcpyDeviceToHost) != cudaSuccess) return check_launch(what);
+  return CUDANP_OK;
+}
+
+int cudanp_debug_owner_map(int64_t n_inner, int S, int dist, int V, int32_t* owner_host) {
+  if (!valid_S(S) || (dist != 0 && dist != 1) || (V != 1 && V != 4) || n_inner < 0 ||
+      n_inner > (1 << 26) || (n_inner > 0 && !owner_host))
+    return fail_invalid("debug_owner_map arguments");
+  if (n_inner == 0) return CUDANP_OK;
+  int32_t* d = nullptr;
+  if (cudaMalloc(&d, n_inner * sizeof(int32_t)) != cudaSuccess) return check_launch("cudaMalloc");
+  cudaMemset(d, 0xff, n_inner * sizeof(int32_t));
+  CUDANP_DISPATCH_S(S, {
+    if (dist == DIST_CYCLIC) owner_kernel<kS, DIST_CYCLIC><<<1, kS>>>(n_inner, V, d);
+    else owner_kernel<kS, DIST_BLOCK><<<1, kS>>>(n_inner, V, d);
+  });
+  int rc = copy_back(owner_host, d, n_inner * sizeof(int32_t), "debug_owner_map");
+  cudaFree(d);
+  return rc;
+}
+
+int cudanp_debug_team_ids(int S, int map, int32_t* master_host, int32_t* slave_host, int* nthreads) {
+  if (!valid_S(S) || (map != CUDANP_MAP_INTRA_WARP && map != CUDANP_MAP_INTER_WARP) ||
+      !master_host || !slave_host || !nthreads)
+    return fail_invalid("debug_team_ids arguments");
+  const int n = map == CUDANP_MAP_INTRA_WARP ? 64 : 32 * S;
+  int32_t* d = nullptr;
+  if (cudaMalloc(&d, 2 * n * sizeof(int32_t)) != cudaSuccess) return check_launch("cudaMalloc");
+  CUDANP_DISPATCH_S(S, {
+    if (map == CUDANP_MAP_INTRA_WARP) team_intra_kernel<kS><<<1, 64>>>(d, d + n);
+    else team_inter_kernel<kS><<<1, dim3(32, kS)>>>(d, d + n);
+  });
+  int rc = copy_back(master_host, d, n * sizeof(int32_t), "debug_team_ids");
+  if (!rc) rc = copy_back(slave_host, d + n, n * sizeof(int32_t), "debug_team_ids");
+  cudaFree(d);
+  *nthreads = n;
+  return rc;
+}
+
+int cudanp_debug_broadcast(int S, int map, int32_t* out_host, int* nthreads) {
+  if (!valid_S(S) || (map != CUDANP_MAP_INTRA_WARP && map != CUDANP_MAP_INTER_WARP) || !out_host ||
+      !nthreads)
+    return fail_invalid("debug_broadcast arguments");
+  const int n = map == CUDANP_MAP_INTRA_WARP ? 64 : 32 * S;
+  int32_t* d = nullptr;
+  if (cudaMalloc(&d, n * sizeof(int32_t)) != cudaSuccess) return check_launch("cudaMalloc");
+  CUDANP_DISPATCH_S(S, {
+    if (map == CUDANP_MAP_INTRA_WARP) bcast_intra_kernel<kS><<<1, 64>>>(d);
+    else bcast_inter_kernel<kS><<<1, dim3(32, kS)>>>(d);
+  });
+  int rc = copy_back(out_host, d, n * sizeof(int32_t), "debug_broadcast");
+  cudaFree(d);
+  *nthreads = n;
+  return rc;
+}
+
+}  // extern "C"

@@ -1,0 +1,89 @@
+// common.cuh -- host-side helpers shared by the libcudanp translation units:
+// status/error text, argument checks, launch-shape computation.
+#pragma once
+#include <cstdint>
+#include <cstdio>
+#include <cstring>
+#include <cuda_runtime.h>
+
+#include "../../include/cudanp.h"
+
+namespace cudanp {
+
+// Thread-local detail for cudanp_last_error().
+void set_error(const char* fmt, ...);
+void clear_error();
+
+inline int fail_invalid(const char* what) {
+  set_error("invalid argument: %s", what);
+  return CUDANP_ERR_INVALID;
+}
+
+inline int check_launch(const char* what) {
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) {
+    set_error("%s: %s", what, cudaGetErrorString(e));
+    return CUDANP_ERR_CUDA;
+  }
+  return CUDANP_OK;
+}
+
+inline bool valid_S(int S) {
+  return S == 1 || S == 2 || S == 4 || S == 8 || S == 16 || S == 32;
+}
+
+inline bool aligned16(const void* p) { return ((uintptr_t)p & 15u) == 0; }
+
+// SM count of the current device (cached per device ordinal).
+int sm_count();
+
+// Grid for a persistent grid-stride kernel: enough CTAs to cover `work_ctas`
+// units of CTA work, capped at (resident CTAs per SM) x (SM count), so the
+// grid is a whole number of waves.
+template <class K>
+inline int64_t persistent_grid(K kernel, int block_threads, size_t dyn_smem, int64_t work_ctas) {
+  int per_sm = 0;
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kernel, block_threads, dyn_smem) !=
+          cudaSuccess ||
+      per_sm < 1) {
+    cudaGetLastError();
+    per_sm = 1;
+  }
+  int64_t cap = (int64_t)per_sm * sm_count();
+  if (work_ctas < 1) work_ctas = 1;
+  return work_ctas < cap ? work_ctas : cap;
+}
+
+template <class K>
+inline void kernel_attrs(K kernel, int* regs, int* smem) {
+  cudaFuncAttributes a;
+  if (cudaFuncGetAttributes(&a, kernel) == cudaSuccess) {
+    if (regs) *regs = a.numRegs;
+    if (smem) *smem = (int)a.sharedSizeBytes;
+  } else {
+    cudaGetLastError();
+  }
+}
+
+// Launch-shape record filled by the dispatchers when info-only is requested.
+struct LaunchInfo {
+  int block_threads = 0;
+  int64_t grid = 0;
+  int regs = 0;
+  int smem = 0;
+  int map = 0;
+};
+
+}  // namespace cudanp
+
+// Dispatch a runtime team size to a compile-time constant `kS`.
+#define CUDANP_DISPATCH_S(S, ...)                        \
+  switch (S) {                                           \
+    case 1: { constexpr int kS = 1; __VA_ARGS__; } break;   \
+    case 2: { constexpr int kS = 2; __VA_ARGS__; } break;   \
+    case 4: { constexpr int kS = 4; __VA_ARGS__; } break;   \
+    case 8: { constexpr int kS = 8; __VA_ARGS__; } break;   \
+    case 16: { constexpr int kS = 16; __VA_ARGS__; } break; \
+    case 32: { constexpr int kS = 32; __VA_ARGS__; } break; \
+    default: return fail_invalid("S must be one of 1,2,4,8,16,32"); \
+  }

@@ -1,0 +1,247 @@
+// np_reduce.cu -- batched loop-reduce: out[n] = init[n] (op) fold_i in[n*L+i].
+//
+// One outer item = one original thread whose parallel loop (trip count L)
+// carries a reduction clause (Fig 6d).  CUDA-NP
+// gives the item a team of S threads; each runs its share of the loop
+// (cyclic P:166 / block R5), the team combines the partials (shfl for
+// intra-warp, shared memory for inter-warp) and the master alone
+// finishes the item.
+//
+// B200 design: the loop body is an HBM stream, so each
+// lane issues 128-bit read-only loads (LDG.E.128.CONSTANT) when rows are
+// 16-byte aligned, keeps K items in flight (memory-level parallelism), and the
+// grid is persistent: a whole number of waves of resident CTAs that stride
+// over items.
+#include "common.cuh"
+#include "np_team.cuh"
+
+namespace cudanp {
+
+constexpr int kReduceBlock = 256;  // intra-warp CTA: 8 warps
+constexpr int kReduceK = 4;        // warp tiles in flight per warp (intra)
+
+template <class T, class Op>
+__device__ __forceinline__ T fold4(V4<T> v) {
+  return Op::apply(Op::apply(v.x, v.y), Op::apply(v.z, v.w));
+}
+template <class T, class Op>
+__device__ __forceinline__ V4<T> op4(V4<T> a, V4<T> b) {
+  return {Op::apply(a.x, b.x), Op::apply(a.y, b.y), Op::apply(a.z, b.z), Op::apply(a.w, b.w)};
+}
+
+// ---------------------------------------------------------------- intra-warp
+// Team = S lanes; a warp holds TPW = 32/S teams = TPW items ("warp tile").
+// Each warp processes K consecutive warp tiles per step of a grid-stride
+// loop, so a lane has K independent rows in flight.
+template <class T, class Op, int S, int DIST, bool VEC>
+__global__ void __launch_bounds__(kReduceBlock)
+reduce_intra_kernel(const T* __restrict__ in, const T* __restrict__ init, T* __restrict__ out,
+                    int64_t N, int64_t L) {
+  constexpr int TPW = 32 / S;
+  constexpr int K = kReduceK;
+  const IntraTeam<S> team;
+  const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  const int64_t nunits = VEC ? (L >> 2) : L;
+  // Iteration share of this slave: uniform index math, recomputed by every
+  // slave instead of broadcast.
+  const Range<S, DIST> r(nunits, L, VEC ? 4 : 1, team.slave);
+  const int64_t ntiles = (N + TPW - 1) / TPW;
+
+  for (int64_t t0 = warp * K; t0 < ntiles; t0 += nwarps * K) {
+    int64_t item[K];
+    const T* row[K];
+#pragma unroll
+    for (int k = 0; k < K; ++k) {
+      item[k] = (t0 + k) * TPW + team.team;
+      row[k] = in + (item[k] < N ? item[k] : 0) * L;
+    }
+    T part[K];
+    if constexpr (VEC) {
+      V4<T> acc[K];
+#pragma unroll
+      for (int k = 0; k < K; ++k) {
+        const T id = Op::template identity<T>();
+        acc[k] = {id, id, id, id};
+      }
+      // Parallel loop section: every team member active.
+#pragma unroll 2
+      for (int64_t u = r.begin; u < r.end; u += r.step) {
+        V4<T> v[K];
+#pragma unroll
+        for (int k = 0; k < K; ++k)
+          if (item[k] < N) v[k] = ldg4(row[k] + 4 * u);
+#pragma unroll
+        for (int k = 0; k < K; ++k)
+          if (item[k] < N) acc[k] = op4<T, Op>(acc[k], v[k]);
+      }
+#pragma unroll
+      for (int k = 0; k < K; ++k) part[k] = fold4<T, Op>(acc[k]);
+    } else {
+#pragma unroll
+      for (int k = 0; k < K; ++k) part[k] = Op::template identity<T>();
+#pragma unroll 4
+      for (int64_t u = r.begin; u < r.end; u += r.step) {
+        T v[K];
+#pragma unroll
+        for (int k = 0; k < K; ++k)
+          if (item[k] < N) v[k] = ldg1(row[k] + u);
+#pragma unroll
+        for (int k = 0; k < K; ++k)
+          if (item[k] < N) part[k] = Op::apply(part[k], v[k]);
+      }
+    }
+    // Live-out reduction over the team (shfl), then the master-only
+    // epilogue: combine with init[n] and store.
+#pragma unroll
+    for (int k = 0; k < K; ++k) {
+      const T res = team.template reduce<Op>(part[k]);
+      if (team.is_master() && item[k] < N)
+        out[item[k]] = init ? Op::apply(init[item[k]], res) : res;
+    }
+  }
+}
+
+// ---------------------------------------------------------------- inter-warp
+// blockDim = (32, S): master = threadIdx.x (32 items per CTA step), slave =
+// threadIdx.y.  Partials meet in shared memory; the master warp
+// (slave 0) folds them in slave order and stores.
+template <class T, class Op, int S, int DIST, bool VEC>
+__global__ void __launch_bounds__(32 * S)
+reduce_inter_kernel(const T* __restrict__ in, const T* __restrict__ init, T* __restrict__ out,
+                    int64_t N, int64_t L) {
+  __shared__ T red[S][33];
+  const InterTeam<S> team;
+  const int64_t nunits = VEC ? (L >> 2) : L;
+  const Range<S, DIST> r(nunits, L, VEC ? 4 : 1, team.slave);
+  const int64_t ngroups = (N + 31) / 32;
+
+  for (int64_t g = blockIdx.x; g < ngroups; g += gridDim.x) {
+    const int64_t item = g * 32 + team.master;
+    const bool ok = item < N;
+    const T* row = in + (ok ? item : 0) * L;
+    T part;
+    if constexpr (VEC) {
+      const T id = Op::template identity<T>();
+      V4<T> acc = {id, id, id, id};
+      if (ok) {
+#pragma unroll 4
+        for (int64_t u = r.begin; u < r.end; u += r.step) acc = op4<T, Op>(acc, ldg4(row + 4 * u));
+      }
+      part = fold4<T, Op>(acc);
+    } else {
+      part = Op::template identity<T>();
+      if (ok) {
+#pragma unroll 4
+        for (int64_t u = r.begin; u < r.end; u += r.step) part = Op::apply(part, ldg1(row + u));
+      }
+    }
+    if (S == 1) {
+      if (ok) out[item] = init ? Op::apply(init[item], part) : part;
+      continue;
+    }
+    red[team.slave][team.master] = part;
+    __syncthreads();
+    if (team.is_master()) {
+      T res = red[0][team.master];
+#pragma unroll
+      for (int s = 1; s < S; ++s) res = Op::apply(res, red[s][team.master]);
+      if (ok) out[item] = init ? Op::apply(init[item], res) : res;
+    }
+    __syncthreads();
+  }
+}
+
+// ---------------------------------------------------------------- S=1 literal
+// Fig 2's shape applied to the reduce: one thread per item, a scalar serial
+// loop, no vector loads, no persistent grid (the paper's baseline kernel).
+template <class T, class Op>
+__global__ void __launch_bounds__(256)
+reduce_literal_kernel(const T* __restrict__ in, const T* __restrict__ init, T* __restrict__ out,
+                      int64_t N, int64_t L) {
+  const int64_t n = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (n >= N) return;
+  T acc = Op::template identity<T>();
+  for (int64_t i = 0; i < L; ++i) acc = Op::apply(acc, in[n * L + i]);
+  out[n] = init ? Op::apply(init[n], acc) : acc;
+}
+
+// ---------------------------------------------------------------- dispatch
+template <class T, class Op, int S, int DIST, bool VEC>
+static int launch_reduce_map(const T* in, const T* init, T* out, int64_t N, int64_t L, int map,
+                             cudaStream_t st, LaunchInfo* info) {
+  if (map == MAP_INTRA) {
+    auto kern = reduce_intra_kernel<T, Op, S, DIST, VEC>;
+    constexpr int TPW = 32 / S;
+    const int64_t ntiles = (N + TPW - 1) / TPW;
+    const int64_t per_cta = (kReduceBlock / 32) * kReduceK;
+    const int64_t grid = persistent_grid(kern, kReduceBlock, 0, (ntiles + per_cta - 1) / per_cta);
+    if (info) {
+      info->block_threads = kReduceBlock; info->grid = grid; info->map = MAP_INTRA;
+      kernel_attrs(kern, &info->regs, &info->smem);
+      return CUDANP_OK;
+    }
+    if (N == 0) return CUDANP_OK;
+    kern<<<(unsigned)grid, kReduceBlock, 0, st>>>(in, init, out, N, L);
+  } else {
+    auto kern = reduce_inter_kernel<T, Op, S, DIST, VEC>;
+    const int64_t grid = persistent_grid(kern, 32 * S, 0, (N + 31) / 32);
+    if (info) {
+      info->block_threads = 32 * S; info->grid = grid; info->map = MAP_INTER;
+      kernel_attrs(kern, &info->regs, &info->smem);
+      return CUDANP_OK;
+    }
+    if (N == 0) return CUDANP_OK;
+    kern<<<(unsigned)grid, dim3(32, S), 0, st>>>(in, init, out, N, L);
+  }
+  return check_launch("batched_loop_reduce launch");
+}
+
+template <class T, class Op>
+static int dispatch_reduce_t(const void* in, const void* init, void* out, int64_t N, int64_t L,
+                             int S, int dist, int map, bool vec, cudaStream_t st, LaunchInfo* info) {
+  const T* i = (const T*)in;
+  const T* ini = (const T*)init;
+  T* o = (T*)out;
+  CUDANP_DISPATCH_S(S, {
+    if (dist == DIST_CYCLIC) {
+      return vec ? launch_reduce_map<T, Op, kS, DIST_CYCLIC, true>(i, ini, o, N, L, map, st, info)
+                 : launch_reduce_map<T, Op, kS, DIST_CYCLIC, false>(i, ini, o, N, L, map, st, info);
+    } else {
+      return vec ? launch_reduce_map<T, Op, kS, DIST_BLOCK, true>(i, ini, o, N, L, map, st, info)
+                 : launch_reduce_map<T, Op, kS, DIST_BLOCK, false>(i, ini, o, N, L, map, st, info);
+    }
+  });
+  return CUDANP_OK;
+}
+
+int reduce_np(const void* in, const void* init, void* out, int64_t N, int64_t L, int dtype, int op,
+              int S, int dist, int map, bool vec, cudaStream_t st, LaunchInfo* info) {
+  if (dtype == CUDANP_F32)
+    return op == CUDANP_SUM
+               ? dispatch_reduce_t<float, OpSum>(in, init, out, N, L, S, dist, map, vec, st, info)
+               : dispatch_reduce_t<float, OpMax>(in, init, out, N, L, S, dist, map, vec, st, info);
+  return op == CUDANP_SUM
+             ? dispatch_reduce_t<int32_t, OpSum>(in, init, out, N, L, S, dist, map, vec, st, info)
+             : dispatch_reduce_t<int32_t, OpMax>(in, init, out, N, L, S, dist, map, vec, st, info);
+}
+
+int reduce_literal(const void* in, const void* init, void* out, int64_t N, int64_t L, int dtype,
+                   int op, cudaStream_t st) {
+  if (N == 0) return CUDANP_OK;
+  const unsigned grid = (unsigned)((N + 255) / 256);
+  if (dtype == CUDANP_F32) {
+    if (op == CUDANP_SUM)
+      reduce_literal_kernel<float, OpSum><<<grid, 256, 0, st>>>((const float*)in, (const float*)init, (float*)out, N, L);
+    else
+      reduce_literal_kernel<float, OpMax><<<grid, 256, 0, st>>>((const float*)in, (const float*)init, (float*)out, N, L);
+  } else {
+    if (op == CUDANP_SUM)
+      reduce_literal_kernel<int32_t, OpSum><<<grid, 256, 0, st>>>((const int32_t*)in, (const int32_t*)init, (int32_t*)out, N, L);
+    else
+      reduce_literal_kernel<int32_t, OpMax><<<grid, 256, 0, st>>>((const int32_t*)in, (const int32_t*)init, (int32_t*)out, N, L);
+  }
+  return check_launch("batched_loop_reduce literal launch");
+}
+
+}  // namespace cudanp

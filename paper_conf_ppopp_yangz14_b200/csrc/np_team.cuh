@@ -1,0 +1,192 @@
+// np_team.cuh -- CUDA-NP master/slave team primitives for sm_100a.
+//
+// The paper (Yang & Zhou, PPoPP'14; "P:n" = line n of PAPER.md) turns every
+// original thread into a *master* that owns S-1 *slaves* (S = slave_size
+// counts the master).  Masters alone run sequential code
+// (`if (slave_id==0)`, Fig 3b); at a parallel loop the whole team
+// shares the iterations; live-ins reach the slaves through
+// `read_from_master`; live-outs are combined by a reduction or
+// a scan.  Two thread remaps:
+//   intra-warp: the team is S consecutive lanes of one warp (shfl);
+//   inter-warp: master = threadIdx.x, slave = threadIdx.y, so the team spans
+//               S warps and talks through shared memory.
+//
+// This header holds those primitives written for sm_100a: `__shfl_*_sync`
+// with a width argument (the Kepler `__shfl(var, lane, width)` of P:55),
+// shared-memory exchange plus barriers for inter-warp teams, and the
+// iteration distributions (cyclic = the paper's, block = the north star's).
+// Nothing here depends on the oracle.
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace cudanp {
+
+constexpr unsigned kFull = 0xffffffffu;
+
+enum Map : int { MAP_AUTO = 0, MAP_INTRA = 1, MAP_INTER = 2 };
+enum Dist : int { DIST_CYCLIC = 0, DIST_BLOCK = 1 };
+
+// ---------------------------------------------------------------- operators
+struct OpSum {
+  __device__ __forceinline__ static float apply(float a, float b) { return a + b; }
+  // int32 sum wraps modulo 2^32 (R13): add in uint32.
+  __device__ __forceinline__ static int32_t apply(int32_t a, int32_t b) {
+    return (int32_t)((uint32_t)a + (uint32_t)b);
+  }
+  template <class T> __device__ __forceinline__ static T identity() { return T(0); }
+};
+
+struct OpMax {
+  __device__ __forceinline__ static float apply(float a, float b) { return fmaxf(a, b); }
+  __device__ __forceinline__ static int32_t apply(int32_t a, int32_t b) { return a > b ? a : b; }
+  template <class T> __device__ __forceinline__ static T identity();
+};
+template <> __device__ __forceinline__ float OpMax::identity<float>() { return -__int_as_float(0x7f800000); }
+template <> __device__ __forceinline__ int32_t OpMax::identity<int32_t>() { return INT32_MIN; }
+
+// ---------------------------------------------------------------- vectors
+template <class T> struct V4 { T x, y, z, w; };
+
+// Streaming 128-bit load through the read-only path (LDG.E.128.CONSTANT).
+template <class T>
+__device__ __forceinline__ V4<T> ldg4(const T* p) {
+  V4<T> r;
+  uint32_t a, b, c, d;
+  asm volatile("ld.global.nc.v4.b32 {%0,%1,%2,%3}, [%4];"
+               : "=r"(a), "=r"(b), "=r"(c), "=r"(d) : "l"(p));
+  r.x = __builtin_bit_cast(T, a); r.y = __builtin_bit_cast(T, b);
+  r.z = __builtin_bit_cast(T, c); r.w = __builtin_bit_cast(T, d);
+  return r;
+}
+// Same with L1::no_allocate: data a warp touches once (TMV/MV matrix rows).
+template <class T>
+__device__ __forceinline__ V4<T> ldg4_stream(const T* p) {
+  V4<T> r;
+  uint32_t a, b, c, d;
+  asm volatile("ld.global.nc.L1::no_allocate.v4.b32 {%0,%1,%2,%3}, [%4];"
+               : "=r"(a), "=r"(b), "=r"(c), "=r"(d) : "l"(p));
+  r.x = __builtin_bit_cast(T, a); r.y = __builtin_bit_cast(T, b);
+  r.z = __builtin_bit_cast(T, c); r.w = __builtin_bit_cast(T, d);
+  return r;
+}
+template <class T>
+__device__ __forceinline__ T ldg1(const T* p) { return __ldg(p); }
+
+template <class T>
+__device__ __forceinline__ void stg4(T* p, V4<T> v) {
+  asm volatile("st.global.v4.b32 [%0], {%1,%2,%3,%4};" ::"l"(p),
+               "r"(__builtin_bit_cast(uint32_t, v.x)), "r"(__builtin_bit_cast(uint32_t, v.y)),
+               "r"(__builtin_bit_cast(uint32_t, v.z)), "r"(__builtin_bit_cast(uint32_t, v.w))
+               : "memory");
+}
+
+// ---------------------------------------------------------------- distribution
+// Iterations of a parallel loop of `n` units (a unit = V consecutive
+// elements) owned by slave `s` of a team of S.
+//  cyclic (P:166 `for(i=slave_id;i<N;i+=slave_size)`): s, s+S, ...
+//  block  (north star; R5): chunk c = ceil(L/S) rounded up to a
+//         multiple of V elements, i.e. cu = c/V units; [s*cu, min(n,(s+1)cu)).
+// The bound check stays, so n may be any runtime value >= 0.
+template <int S, int DIST>
+struct Range {
+  int64_t begin, end, step;
+  __device__ __forceinline__ Range(int64_t n_units, int64_t n_elems, int V, int s) {
+    if (DIST == DIST_CYCLIC) {
+      begin = s; end = n_units; step = S;
+    } else {
+      int64_t c = (n_elems + S - 1) / S;
+      int64_t cu = (c + V - 1) / V;
+      begin = (int64_t)s * cu;
+      end = begin + cu < n_units ? begin + cu : n_units;
+      step = 1;
+    }
+  }
+};
+
+// ---------------------------------------------------------------- intra-warp team
+// Team = S consecutive lanes (S a power of two <= 32).  slave =
+// lane % S; the master is the team's lane 0; a warp holds 32/S teams
+// (S=4 -> 8 masters + 24 slaves per warp).
+template <int S>
+struct IntraTeam {
+  static_assert(S >= 1 && S <= 32 && (S & (S - 1)) == 0, "intra-warp S must be 2^k <= 32");
+  static constexpr int kTeamsPerWarp = 32 / S;
+  int lane, slave, team;  // team index within the warp
+
+  __device__ __forceinline__ IntraTeam() {
+    lane = threadIdx.x & 31;
+    slave = lane & (S - 1);
+    team = lane / S;
+  }
+  __device__ __forceinline__ bool is_master() const { return slave == 0; }
+
+  // read_from_master: `__shfl(var, 0, slave_size)`.
+  template <class T>
+  __device__ __forceinline__ T read_from_master(T v) const {
+    if (S == 1) return v;
+    return __shfl_sync(kFull, v, 0, S);
+  }
+  // Value held by the team's last slave (scan carry).
+  template <class T>
+  __device__ __forceinline__ T from_last(T v) const {
+    if (S == 1) return v;
+    return __shfl_sync(kFull, v, S - 1, S);
+  }
+  // Reduction of the team's values (shfl for intra-warp NP):
+  // butterfly over log2(S) steps; every team lane ends with the result.
+  template <class Op, class T>
+  __device__ __forceinline__ T reduce(T v) const {
+#pragma unroll
+    for (int o = S / 2; o > 0; o >>= 1) v = Op::apply(v, __shfl_xor_sync(kFull, v, o, S));
+    return v;
+  }
+  // Inclusive scan over the team ("similar approach to the CUDA SDK"):
+  // Hillis-Steele with shfl_up inside each width-S segment.
+  template <class T>
+  __device__ __forceinline__ T inclusive_scan(T v) const {
+#pragma unroll
+    for (int o = 1; o < S; o <<= 1) {
+      T t = __shfl_up_sync(kFull, v, o, S);
+      if (slave >= o) v = OpSum::apply(v, t);
+    }
+    return v;
+  }
+  // Exclusive value = inclusive value of the previous slave (0 for slave 0).
+  template <class T>
+  __device__ __forceinline__ T exclusive_from_inclusive(T incl) const {
+    if (S == 1) return T(0);
+    T t = __shfl_up_sync(kFull, incl, 1, S);
+    return slave == 0 ? T(0) : t;
+  }
+};
+
+// ---------------------------------------------------------------- inter-warp team
+// blockDim = (32, S): master = threadIdx.x (one per lane), slave =
+// threadIdx.y (one per warp).  A master's slaves sit in S
+// different warps, so every exchange goes through shared memory plus a
+// CTA barrier.  All CTA threads must call the collective
+// members (they contain __syncthreads).
+template <int S>
+struct InterTeam {
+  static_assert(S >= 1 && S <= 32, "inter-warp S <= 32 (CTA = 32 x S <= 1024 threads)");
+  int master, slave;
+  __device__ __forceinline__ InterTeam() {
+    master = threadIdx.x;
+    slave = threadIdx.y;
+  }
+  __device__ __forceinline__ bool is_master() const { return slave == 0; }
+
+  // read_from_master through a per-master smem slot.
+  template <class T>
+  __device__ __forceinline__ T read_from_master(T v, T* slot /*[32]*/) const {
+    if (S == 1) return v;
+    if (slave == 0) slot[master] = v;
+    __syncthreads();
+    T r = slot[master];
+    __syncthreads();
+    return r;
+  }
+};
+
+}  // namespace cudanp

@@ -1,0 +1,293 @@
+"""Thin Python binding of libcudanp.so (include/cudanp.h).
+
+Argument marshalling only: every step of the hot path runs in the library's
+sm_100a kernels.  torch supplies device memory and the current CUDA stream.
+There is no CPU fallback: if the shared library is missing this module raises
+on first use, and a non-OK status from the library raises CudanpError.
+
+Function names follow the C ABI (``cudanp_tmv``, ``cudanp_mv``,
+``cudanp_batched_loop_reduce``, ``cudanp_batched_loop_scan`` and the
+``*_variant`` comparison calls).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import threading
+
+import numpy as np
+
+_PKG = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_PKG, "libcudanp.so")
+
+OK, ERR_INVALID, ERR_UNSUPPORTED, ERR_CUDA, ERR_NCCL = 0, 1, 2, 3, 4
+CYCLIC, BLOCK = 0, 1
+AUTO, INTRA_WARP, INTER_WARP = 0, 1, 2
+F32, I32 = 0, 1
+SUM, MAX = 0, 1
+S1_LITERAL, DP_THREAD, DP_BLOCK = 1, 2, 3
+SLAVE_SIZES = (1, 2, 4, 8, 16, 32)
+KIND = {"f32_unit": 0, "f32_signed": 1, "f32_int4": 2, "i32_small": 3, "i32_full": 4,
+        "ones_f32": 5, "ones_i32": 6}
+SEED = 20140215
+
+_i64, _u64, _int, _vp, _sz = ctypes.c_int64, ctypes.c_uint64, ctypes.c_int, ctypes.c_void_p, ctypes.c_size_t
+_P32 = ctypes.POINTER(ctypes.c_int32)
+_SIGS = {
+    "cudanp_tmv": [_vp, _i64, _vp, _vp, _i64, _i64, _int, _int, _int, _vp],
+    "cudanp_mv": [_vp, _i64, _vp, _vp, _i64, _i64, _int, _int, _int, _vp],
+    "cudanp_batched_loop_reduce": [_vp, _vp, _vp, _i64, _i64, _int, _int, _int, _int, _int, _vp],
+    "cudanp_batched_loop_scan": [_vp, _vp, _vp, _i64, _i64, _int, _int, _int, _int, _vp],
+    "cudanp_tmv_variant": [_int, _vp, _i64, _vp, _vp, _i64, _i64, _vp],
+    "cudanp_mv_variant": [_int, _vp, _i64, _vp, _vp, _i64, _i64, _vp],
+    "cudanp_batched_loop_reduce_variant": [_int, _vp, _vp, _vp, _i64, _i64, _int, _int, _vp],
+    "cudanp_batched_loop_scan_variant": [_int, _vp, _vp, _vp, _i64, _i64, _int, _vp],
+    "cudanp_dp_set_pending_launch_limit": [_sz],
+    "cudanp_dp_error_count": [_int, ctypes.POINTER(_i64)],
+    "cudanp_launch_info": [_int, _i64, _i64, _int, _int, _int, _int, _int, _int,
+                           ctypes.POINTER(_int), ctypes.POINTER(_i64), ctypes.POINTER(_int),
+                           ctypes.POINTER(_int), ctypes.POINTER(_int)],
+    "cudanp_shard_range": [_i64, _int, _int, ctypes.POINTER(_i64), ctypes.POINTER(_i64)],
+    "cudanp_generate": [_vp, _i64, _i64, _i64, _i64, _i64, _i64, _int, _int, _i64, _u64, _vp],
+    "cudanp_debug_owner_map": [_i64, _int, _int, _int, _P32],
+    "cudanp_debug_team_ids": [_int, _int, _P32, _P32, ctypes.POINTER(_int)],
+    "cudanp_debug_broadcast": [_int, _int, _P32, ctypes.POINTER(_int)],
+    "cudanp_status_string": [_int],
+    "cudanp_last_error": [],
+    "cudanp_version": [],
+}
+EXPORTS = tuple(_SIGS)
+
+_lock = threading.Lock()
+_lib = None
+
+
+class CudanpError(RuntimeError):
+    def __init__(self, status: int, where: str, detail: str):
+        super().__init__(f"{where}: status {status} ({_status_name(status)}): {detail}")
+        self.status = status
+
+
+def _status_name(s: int) -> str:
+    return {0: "OK", 1: "ERR_INVALID", 2: "ERR_UNSUPPORTED", 3: "ERR_CUDA", 4: "ERR_NCCL"}.get(s, "?")
+
+
+def load(path: str = LIB_PATH) -> ctypes.CDLL:
+    """Load libcudanp.so.  Raises if it has not been built (no fallback)."""
+    global _lib
+    with _lock:
+        if _lib is None:
+            if not os.path.exists(path):
+                raise ImportError(f"{path} not found: build it with "
+                                  "`python -m paper_conf_ppopp_yangz14_b200.build`")
+            L = ctypes.CDLL(path)
+            for name, args in _SIGS.items():
+                f = getattr(L, name)
+                f.argtypes = args
+                f.restype = ctypes.c_char_p if name in ("cudanp_status_string", "cudanp_last_error") else _int
+            _lib = L
+    return _lib
+
+
+def _check(rc: int, where: str) -> None:
+    if rc != OK:
+        raise CudanpError(rc, where, load().cudanp_last_error().decode())
+
+
+def _stream(stream) -> int | None:
+    import torch
+    if stream is None:
+        return torch.cuda.current_stream().cuda_stream or None
+    if isinstance(stream, int):
+        return stream or None
+    return stream.cuda_stream or None
+
+
+def _ptr(t) -> int | None:
+    if t is None:
+        return None
+    if not t.is_cuda:
+        raise ValueError("tensor must be on a CUDA device (the library takes device pointers)")
+    return t.data_ptr() or None
+
+
+def _dtype_code(t) -> int:
+    import torch
+    if t.dtype == torch.float32:
+        return F32
+    if t.dtype == torch.int32:
+        return I32
+    raise TypeError(f"unsupported dtype {t.dtype}: float32 or int32")
+
+
+# ---------------------------------------------------------------- hot-path calls
+def cudanp_tmv(A, x, y=None, *, S=32, dist=CYCLIC, map=AUTO, n_outer=None, stream=None):
+    """y[j] = sum_i A[i, j] * x[i] (Fig 2).  A: (h, lda) fp32 row-major."""
+    import torch
+    h, lda = A.shape
+    w = lda if n_outer is None else n_outer
+    if y is None:
+        y = torch.empty(w, dtype=torch.float32, device=A.device)
+    _check(load().cudanp_tmv(_ptr(A), lda, _ptr(x), _ptr(y), w, h, S, dist, map, _stream(stream)),
+           "cudanp_tmv")
+    return y
+
+
+def cudanp_mv(A, x, y=None, *, S=32, dist=CYCLIC, map=AUTO, n_inner=None, stream=None):
+    """y[i] = sum_j A[i, j] * x[j].  A: (h, lda) fp32 row-major."""
+    import torch
+    h, lda = A.shape
+    w = lda if n_inner is None else n_inner
+    if y is None:
+        y = torch.empty(h, dtype=torch.float32, device=A.device)
+    _check(load().cudanp_mv(_ptr(A), lda, _ptr(x), _ptr(y), h, w, S, dist, map, _stream(stream)),
+           "cudanp_mv")
+    return y
+
+
+def cudanp_batched_loop_reduce(x, init=None, out=None, *, op=SUM, S=8, dist=CYCLIC, map=AUTO,
+                               stream=None):
+    """out[n] = init[n] (op) fold_i x[n, i].  x: (N, L) fp32/int32."""
+    import torch
+    N, L = x.shape
+    if out is None:
+        out = torch.empty(N, dtype=x.dtype, device=x.device)
+    _check(load().cudanp_batched_loop_reduce(_ptr(x), _ptr(init), _ptr(out), N, L, _dtype_code(x),
+                                             op, S, dist, map, _stream(stream)),
+           "cudanp_batched_loop_reduce")
+    return out
+
+
+def cudanp_batched_loop_scan(x, init=None, out=None, *, S=8, dist=CYCLIC, map=AUTO, stream=None):
+    """Inclusive scan out[n, k] = init[n] + sum_{i<=k} x[n, i]."""
+    import torch
+    N, L = x.shape
+    if out is None:
+        out = torch.empty_like(x)
+    _check(load().cudanp_batched_loop_scan(_ptr(x), _ptr(init), _ptr(out), N, L, _dtype_code(x),
+                                           S, dist, map, _stream(stream)),
+           "cudanp_batched_loop_scan")
+    return out
+
+
+# ---------------------------------------------------------------- comparison kernels
+def cudanp_tmv_variant(impl, A, x, y=None, *, n_outer=None, stream=None):
+    import torch
+    h, lda = A.shape
+    w = lda if n_outer is None else n_outer
+    if y is None:
+        y = torch.empty(w, dtype=torch.float32, device=A.device)
+    _check(load().cudanp_tmv_variant(impl, _ptr(A), lda, _ptr(x), _ptr(y), w, h, _stream(stream)),
+           "cudanp_tmv_variant")
+    return y
+
+
+def cudanp_mv_variant(impl, A, x, y=None, *, n_inner=None, stream=None):
+    import torch
+    h, lda = A.shape
+    w = lda if n_inner is None else n_inner
+    if y is None:
+        y = torch.empty(h, dtype=torch.float32, device=A.device)
+    _check(load().cudanp_mv_variant(impl, _ptr(A), lda, _ptr(x), _ptr(y), h, w, _stream(stream)),
+           "cudanp_mv_variant")
+    return y
+
+
+def cudanp_batched_loop_reduce_variant(impl, x, init=None, out=None, *, op=SUM, stream=None):
+    import torch
+    N, L = x.shape
+    if out is None:
+        out = torch.empty(N, dtype=x.dtype, device=x.device)
+    _check(load().cudanp_batched_loop_reduce_variant(impl, _ptr(x), _ptr(init), _ptr(out), N, L,
+                                                     _dtype_code(x), op, _stream(stream)),
+           "cudanp_batched_loop_reduce_variant")
+    return out
+
+
+def cudanp_batched_loop_scan_variant(impl, x, init=None, out=None, *, stream=None):
+    N, L = x.shape
+    if out is None:
+        import torch
+        out = torch.empty_like(x)
+    _check(load().cudanp_batched_loop_scan_variant(impl, _ptr(x), _ptr(init), _ptr(out), N, L,
+                                                   _dtype_code(x), _stream(stream)),
+           "cudanp_batched_loop_scan_variant")
+    return out
+
+
+def cudanp_dp_set_pending_launch_limit(n: int) -> None:
+    _check(load().cudanp_dp_set_pending_launch_limit(n), "cudanp_dp_set_pending_launch_limit")
+
+
+def cudanp_dp_error_count(reset: bool = True) -> int:
+    c = _i64(0)
+    _check(load().cudanp_dp_error_count(int(reset), ctypes.byref(c)), "cudanp_dp_error_count")
+    return c.value
+
+
+# ---------------------------------------------------------------- support
+def cudanp_launch_info(op_kind: str, n_outer: int, n_inner: int, *, dtype=F32, op=SUM, S=8,
+                       dist=CYCLIC, map=AUTO, vec4=True) -> dict:
+    kinds = {"tmv": 0, "mv": 1, "reduce": 2, "scan": 3}
+    b, g, r, s, m = _int(), _i64(), _int(), _int(), _int()
+    _check(load().cudanp_launch_info(kinds[op_kind], n_outer, n_inner, dtype, op, S, dist, map,
+                                     int(vec4), ctypes.byref(b), ctypes.byref(g), ctypes.byref(r),
+                                     ctypes.byref(s), ctypes.byref(m)), "cudanp_launch_info")
+    return {"block_threads": b.value, "grid_ctas": g.value, "regs_per_thread": r.value,
+            "smem_bytes": s.value, "map": {1: "intra_warp", 2: "inter_warp"}.get(m.value, "?")}
+
+
+def cudanp_shard_range(n_outer: int, nranks: int, rank: int) -> tuple[int, int]:
+    b, e = _i64(), _i64()
+    _check(load().cudanp_shard_range(n_outer, nranks, rank, ctypes.byref(b), ctypes.byref(e)),
+           "cudanp_shard_range")
+    return b.value, e.value
+
+
+def cudanp_generate(out, kind: str, *, stream_id=1, row0=0, col0=0, w_global=None, B=1 << 20,
+                    seed=SEED, stream=None):
+    """Fill a 1-D or 2-D CUDA tensor with the counter-based generator (test/bench support)."""
+    if out.dim() == 1:
+        rows, cols, ld = 1, out.shape[0], out.shape[0]
+    else:
+        rows, cols = out.shape
+        ld = out.stride(0)
+    wg = cols if w_global is None else w_global
+    if out.dim() == 1 and w_global is None:
+        wg = 0  # 1-D: idx = col0 + c
+    _check(load().cudanp_generate(_ptr(out), rows, cols, ld, row0, col0, wg, stream_id, KIND[kind],
+                                  B, seed, _stream(stream)), "cudanp_generate")
+    return out
+
+
+def cudanp_debug_owner_map(n_inner: int, S: int, dist: int, V: int = 1) -> np.ndarray:
+    out = np.empty(max(n_inner, 0), np.int32)
+    _check(load().cudanp_debug_owner_map(n_inner, S, dist, V, out.ctypes.data_as(_P32)),
+           "cudanp_debug_owner_map")
+    return out
+
+
+def cudanp_debug_team_ids(S: int, map_: int):
+    n_max = 1024
+    m = np.empty(n_max, np.int32)
+    s = np.empty(n_max, np.int32)
+    n = _int()
+    _check(load().cudanp_debug_team_ids(S, map_, m.ctypes.data_as(_P32), s.ctypes.data_as(_P32),
+                                        ctypes.byref(n)), "cudanp_debug_team_ids")
+    return m[: n.value].copy(), s[: n.value].copy()
+
+
+def cudanp_debug_broadcast(S: int, map_: int) -> np.ndarray:
+    out = np.empty(1024, np.int32)
+    n = _int()
+    _check(load().cudanp_debug_broadcast(S, map_, out.ctypes.data_as(_P32), ctypes.byref(n)),
+           "cudanp_debug_broadcast")
+    return out[: n.value].copy()
+
+
+def cudanp_status_string(status: int) -> str:
+    return load().cudanp_status_string(status).decode()
+
+
+def cudanp_version() -> int:
+    return load().cudanp_version()

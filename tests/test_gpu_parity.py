@@ -1,0 +1,421 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle,
+element by element, on the same seeded inputs.
+
+Bar (BASELINE.json north_star):
+  * int32 reduce / scan, every max, and fp32 on exactly-representable data
+    (pin P3): bit-exact;
+  * fp32 sums on positive data: max relative error <= tol(L) =
+    1e-5 * max(1, sqrt(L/4096)) (reading R17), against the fp64 oracle.
+Sizes span several tiles/waves and ragged tails; the full-size checks run in
+the same launch configuration bench.py times, on sampled outputs the oracle
+computes one by one.
+"""
+import itertools
+import math
+
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+if not torch.cuda.is_available():
+    pytest.skip("needs a CUDA device", allow_module_level=True)
+
+import oracle as O
+import synth
+from paper_conf_ppopp_yangz14_b200 import build as B
+from paper_conf_ppopp_yangz14_b200 import cudanp as C
+
+pytestmark = pytest.mark.gpu
+
+SS = C.SLAVE_SIZES
+DISTS = (C.CYCLIC, C.BLOCK)
+MAPS = (C.INTRA_WARP, C.INTER_WARP)
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _lib():
+    B.build()
+    C.load()
+
+
+def dev(a):
+    return torch.from_numpy(np.ascontiguousarray(a)).cuda()
+
+
+def host(t):
+    torch.cuda.synchronize()
+    return t.cpu().numpy()
+
+
+def tol(L):
+    return 1e-5 * max(1.0, math.sqrt(max(L, 1) / 4096.0))
+
+
+def assert_rel(got, ref, L, what):
+    got = np.asarray(got, np.float64)
+    ref = np.asarray(ref, np.float64)
+    assert got.shape == ref.shape, what
+    if ref.size == 0:
+        return
+    denom = np.maximum(np.abs(ref), 1e-30)
+    err = np.max(np.abs(got - ref) / denom)
+    assert err <= tol(L), f"{what}: max rel err {err:.3e} > {tol(L):.3e}"
+
+
+def assert_exact(got, ref, what):
+    got = np.asarray(got)
+    ref = np.asarray(ref)
+    assert got.shape == ref.shape, what
+    if not np.array_equal(got.view(np.uint32) if got.dtype == np.float32 else got,
+                          ref.view(np.uint32) if ref.dtype == np.float32 else ref):
+        bad = np.argwhere(got != ref)
+        raise AssertionError(f"{what}: {len(bad)} mismatches, first at {bad[:3].tolist()}: "
+                             f"got {got[tuple(bad[0])]} want {ref[tuple(bad[0])]}")
+
+
+# ------------------------------------------------------------------ infrastructure pins
+def test_device_generator_matches_oracle_generator():
+    # pin P8: three independent implementations of the generator agree
+    for kind, n in [("f32_unit", 4099), ("f32_signed", 1000), ("f32_int4", 777)]:
+        t = torch.empty(n, dtype=torch.float32, device="cuda")
+        C.cudanp_generate(t, kind, stream_id=2, col0=(1 << 32) - 5)
+        assert_exact(host(t), O.gen_f32(2, kind, (1 << 32) - 5, n), kind)
+    for kind, B_ in [("i32_small", 1 << 20), ("i32_small", 1 << 15), ("i32_full", 1)]:
+        t = torch.empty(5000, dtype=torch.int32, device="cuda")
+        C.cudanp_generate(t, kind, stream_id=1, B=B_)
+        assert_exact(host(t), O.gen_i32(1, kind, 0, 5000, B_), kind)
+    # 2-D column shard of a wider matrix, with a padded leading dimension
+    buf = torch.full((7, 12), -1.0, device="cuda")
+    C.cudanp_generate(buf[:, :9], "f32_unit", row0=3, col0=20, w_global=50)
+    want = synth.matrix(7, 9, "f32_unit", row0=3, col0=20, w_global=50)
+    got = host(buf)
+    assert_exact(got[:, :9], want, "2-D shard")
+    assert (got[:, 9:] == -1).all()
+
+
+def test_owner_map_is_the_papers_distribution():
+    # the kernels' own Range code, run on the device, against the oracle's
+    # restatement of P:166 / P:294 (cyclic) and reading R5 (block)
+    for L in [0, 1, 3, 12, 31, 32, 33, 150, 1000, 4096]:
+        for S in SS:
+            for dist in DISTS:
+                for V in (1, 4):
+                    got = C.cudanp_debug_owner_map(L, S, dist, V)
+                    assert_exact(got, O.owner_map(L, S, dist, V), f"L={L} S={S} dist={dist} V={V}")
+    # loop count 12, slave_size 8 -> 4 slaves take 2 iterations, 4 take 1
+    assert np.bincount(C.cudanp_debug_owner_map(12, 8, C.CYCLIC, 1)).tolist() == [2, 2, 2, 2, 1, 1, 1, 1]
+
+
+def test_team_ids_match_paper_remap():
+    for S in SS:
+        m, s = C.cudanp_debug_team_ids(S, C.INTRA_WARP)
+        om, os_ = O.team_ids(S, O.INTRA_WARP, len(m))
+        assert_exact(m, om, f"intra master S={S}")
+        assert_exact(s, os_, f"intra slave S={S}")
+        m, s = C.cudanp_debug_team_ids(S, C.INTER_WARP)
+        assert len(m) == 32 * S  # CTA = 32 masters x S slaves
+        om, os_ = O.team_ids(S, O.INTER_WARP, len(m))
+        assert_exact(m, om, f"inter master S={S}")
+        assert_exact(s, os_, f"inter slave S={S}")
+
+
+def test_read_from_master_broadcast():
+    # every team member receives its master's value
+    for S in SS:
+        out = C.cudanp_debug_broadcast(S, C.INTRA_WARP)
+        t = np.arange(len(out))
+        assert_exact(out, (1000 * (t - t % S) + 7).astype(np.int32), f"intra S={S}")
+        out = C.cudanp_debug_broadcast(S, C.INTER_WARP)
+        t = np.arange(len(out))
+        assert_exact(out, (1000 * (t % 32) + 7).astype(np.int32), f"inter S={S}")
+
+
+# ------------------------------------------------------------------ batched reduce
+REDUCE_SHAPES = [(0, 7), (1, 1), (3, 0), (33, 5), (70, 12), (257, 32), (300, 33), (129, 80),
+                 (200, 150), (97, 256), (1100, 64)]
+
+
+def _reduce_cases():
+    # (dtype, op, kind, exact)
+    return [(C.F32, C.SUM, "f32_unit", False), (C.F32, C.SUM, "f32_int4", True),
+            (C.F32, C.MAX, "f32_signed", True), (C.I32, C.SUM, "i32_full", True),
+            (C.I32, C.MAX, "i32_full", True)]
+
+
+@pytest.mark.parametrize("case", _reduce_cases(), ids=lambda c: f"{c[0]}-{c[1]}-{c[2]}")
+def test_reduce_parity(case):
+    dtype, op, kind, exact = case
+    for N, L in REDUCE_SHAPES:
+        x = synth.items(N, L, kind)
+        ini = synth.init(N, kind)
+        ref = O.reduce(x, op=op)
+        ref_i = O.reduce(x, op=op, init=ini)
+        xd, inid = dev(x), dev(ini)
+        for S, dist, map_ in itertools.product(SS, DISTS, MAPS):
+            what = f"reduce {kind} op={op} N={N} L={L} S={S} dist={dist} map={map_}"
+            got = host(C.cudanp_batched_loop_reduce(xd, op=op, S=S, dist=dist, map=map_))
+            got_i = host(C.cudanp_batched_loop_reduce(xd, inid, op=op, S=S, dist=dist, map=map_))
+            if exact:
+                assert_exact(got, ref, what)
+                assert_exact(got_i, ref_i, what + " init")
+            else:
+                assert_rel(got, ref, L, what)
+                assert_rel(got_i, ref_i, L, what + " init")
+
+
+def test_reduce_scalar_path_misaligned():
+    # a base pointer off 16-byte alignment takes the scalar (V=1) path
+    N, L = 300, 64
+    x = synth.items(N + 1, L, "i32_full").reshape(-1)
+    xd = dev(x)
+    view = xd[1:1 + N * L].view(N, L)
+    assert view.data_ptr() % 16 != 0
+    ref = O.reduce(x[1:1 + N * L].reshape(N, L))
+    for S, dist, map_ in itertools.product(SS, DISTS, MAPS):
+        assert_exact(host(C.cudanp_batched_loop_reduce(view, S=S, dist=dist, map=map_)), ref,
+                     f"misaligned S={S} dist={dist} map={map_}")
+
+
+def test_reduce_int32_wrap_and_closed_forms():
+    x = np.full((64, 8), 1 << 30, np.int32)
+    for S in SS:
+        assert (host(C.cudanp_batched_loop_reduce(dev(x), S=S)) == 0).all()
+    ones = torch.ones(100, 256, dtype=torch.int32, device="cuda")
+    for S in SS:
+        assert (host(C.cudanp_batched_loop_reduce(ones, S=S)) == 256).all()
+    # L = 0 -> init or the identity
+    e = torch.empty(5, 0, dtype=torch.float32, device="cuda")
+    assert (host(C.cudanp_batched_loop_reduce(e, op=C.MAX)) == -np.inf).all()
+    ini = dev(np.arange(5, dtype=np.float32))
+    assert (host(C.cudanp_batched_loop_reduce(e, ini)) == np.arange(5)).all()
+
+
+# ------------------------------------------------------------------ batched scan
+SCAN_SHAPES = [(0, 8), (1, 1), (33, 5), (70, 12), (100, 64), (41, 80), (37, 150), (64, 256),
+               (20, 1024), (9, 1000)]
+
+
+@pytest.mark.parametrize("case", [(C.I32, "i32_small", True), (C.F32, "f32_int4", True),
+                                  (C.F32, "f32_unit", False)], ids=lambda c: c[1])
+def test_scan_parity(case):
+    dtype, kind, exact = case
+    for N, L in SCAN_SHAPES:
+        B_ = 1 << 15
+        x = synth.items(N, L, kind, B=B_)
+        ini = synth.init(N, kind, B=B_)
+        ref = O.scan(x)
+        ref_i = O.scan(x, init=ini)
+        xd, inid = dev(x), dev(ini)
+        for S, dist, map_ in itertools.product(SS, DISTS, MAPS):
+            what = f"scan {kind} N={N} L={L} S={S} dist={dist} map={map_}"
+            got = host(C.cudanp_batched_loop_scan(xd, S=S, dist=dist, map=map_))
+            got_i = host(C.cudanp_batched_loop_scan(xd, inid, S=S, dist=dist, map=map_))
+            if exact:
+                assert_exact(got, ref, what)
+                assert_exact(got_i, ref_i, what + " init")
+            else:
+                assert_rel(got, ref, L, what)
+                assert_rel(got_i, ref_i, L, what + " init")
+
+
+def test_scan_closed_forms_and_L0():
+    for S in SS:
+        ones = torch.ones(50, 1024, dtype=torch.int32, device="cuda")
+        got = host(C.cudanp_batched_loop_scan(ones, S=S))
+        assert (got == np.arange(1, 1025)).all()
+    out = torch.full((4, 0), 7, dtype=torch.int32, device="cuda")
+    C.cudanp_batched_loop_scan(torch.empty(4, 0, dtype=torch.int32, device="cuda"), out=out)
+
+
+def test_scan_misaligned_output():
+    N, L = 50, 64
+    x = synth.items(N, L, "i32_small")
+    xd = dev(x)
+    buf = torch.zeros(N * L + 1, dtype=torch.int32, device="cuda")
+    out = buf[1:].view(N, L)
+    for S, dist, map_ in itertools.product(SS, DISTS, MAPS):
+        C.cudanp_batched_loop_scan(xd, out=out, S=S, dist=dist, map=map_)
+        assert_exact(host(out), O.scan(x), f"misaligned out S={S} dist={dist} map={map_}")
+
+
+# ------------------------------------------------------------------ TMV / MV
+MAT_SHAPES = [(0, 8), (8, 0), (1, 1), (3, 5), (37, 131), (300, 260), (129, 512), (1024, 1024)]
+
+
+@pytest.mark.parametrize("kind", ["f32_unit", "f32_int4"])
+def test_tmv_parity(kind):
+    for h, w in MAT_SHAPES:
+        A = synth.matrix(h, w, kind)
+        x = synth.vector(h, kind)
+        ref = O.tmv(A, x, w) if h else np.zeros(w, np.float32)
+        Ad, xd = dev(A), dev(x)
+        for S, dist, map_ in itertools.product(SS, DISTS, MAPS):
+            what = f"tmv {kind} h={h} w={w} S={S} dist={dist} map={map_}"
+            got = host(C.cudanp_tmv(Ad, xd, S=S, dist=dist, map=map_)) if w else np.zeros(0, np.float32)
+            if kind == "f32_int4":
+                assert_exact(got, ref, what)
+            else:
+                assert_rel(got, ref, h, what)
+
+
+@pytest.mark.parametrize("kind", ["f32_unit", "f32_int4"])
+def test_mv_parity(kind):
+    for h, w in MAT_SHAPES:
+        A = synth.matrix(h, w, kind)
+        x = synth.vector(w, kind)
+        ref = O.mv(A, x, w) if h else np.zeros(0, np.float32)
+        Ad, xd = dev(A), dev(x)
+        for S, dist, map_ in itertools.product(SS, DISTS, MAPS):
+            what = f"mv {kind} h={h} w={w} S={S} dist={dist} map={map_}"
+            got = host(C.cudanp_mv(Ad, xd, S=S, dist=dist, map=map_)) if h else np.zeros(0, np.float32)
+            if kind == "f32_int4":
+                assert_exact(got, ref, what)
+            else:
+                assert_rel(got, ref, w, what)
+
+
+def test_matvec_padded_lda_and_scalar_path():
+    h, w, lda = 70, 45, 52   # w % 4 != 0 -> scalar path; lda > w
+    full = synth.matrix(h, lda, "f32_int4")
+    A = full.copy()
+    A[:, w:] = np.nan
+    x_t = synth.vector(h, "f32_int4")
+    x_m = synth.vector(w, "f32_int4")
+    Ad = dev(A)
+    for S, dist, map_ in itertools.product(SS, DISTS, MAPS):
+        got = host(C.cudanp_tmv(Ad, dev(x_t), S=S, dist=dist, map=map_, n_outer=w))
+        assert_exact(got, O.tmv(A, x_t, w), f"tmv lda S={S} dist={dist} map={map_}")
+        got = host(C.cudanp_mv(Ad, dev(x_m), S=S, dist=dist, map=map_, n_inner=w))
+        assert_exact(got, O.mv(A, x_m, w), f"mv lda S={S} dist={dist} map={map_}")
+
+
+def test_tmv_closed_forms():
+    h, w = 1024, 512
+    x = synth.vector(h, "f32_unit")
+    ones = torch.ones(h, w, device="cuda")
+    ref = O.tmv(np.ones((h, w), np.float32), x)
+    A = synth.matrix(h, w, "f32_signed")
+    for S in SS:
+        assert_rel(host(C.cudanp_tmv(ones, dev(x), S=S)), ref, h, f"ones S={S}")
+        e = np.zeros(h, np.float32)
+        e[77] = 1
+        assert_exact(host(C.cudanp_tmv(dev(A), dev(e), S=S)), A[77], f"e_k S={S}")
+
+
+# ------------------------------------------------------------------ comparison kernels
+@pytest.mark.parametrize("impl", [C.S1_LITERAL, C.DP_THREAD, C.DP_BLOCK])
+def test_variants_parity(impl):
+    C.cudanp_dp_set_pending_launch_limit(1 << 16)
+    C.cudanp_dp_error_count(reset=True)
+    h, w = 300, 260
+    A = synth.matrix(h, w, "f32_int4")
+    xt, xm = synth.vector(h, "f32_int4"), synth.vector(w, "f32_int4")
+    assert_exact(host(C.cudanp_tmv_variant(impl, dev(A), dev(xt))), O.tmv(A, xt), f"tmv impl={impl}")
+    assert_exact(host(C.cudanp_mv_variant(impl, dev(A), dev(xm))), O.mv(A, xm), f"mv impl={impl}")
+    Au = synth.matrix(h, w, "f32_unit")
+    xu = synth.vector(h, "f32_unit")
+    assert_rel(host(C.cudanp_tmv_variant(impl, dev(Au), dev(xu))), O.tmv(Au, xu), h, "tmv unit")
+    for N, L in [(1, 1), (300, 33), (1000, 64), (77, 1000)]:
+        for dtype, op, kind in [(C.I32, C.SUM, "i32_full"), (C.F32, C.MAX, "f32_signed"),
+                                (C.I32, C.MAX, "i32_full")]:
+            x = synth.items(N, L, kind)
+            ini = synth.init(N, kind)
+            got = host(C.cudanp_batched_loop_reduce_variant(impl, dev(x), dev(ini), op=op))
+            assert_exact(got, O.reduce(x, op=op, init=ini), f"reduce impl={impl} N={N} L={L}")
+        x = synth.items(N, L, "f32_unit")
+        got = host(C.cudanp_batched_loop_reduce_variant(impl, dev(x)))
+        assert_rel(got, O.reduce(x), L, f"reduce f32 impl={impl}")
+        xi = synth.items(N, L, "i32_small")
+        ini = synth.init(N, "i32_small")
+        got = host(C.cudanp_batched_loop_scan_variant(impl, dev(xi), dev(ini)))
+        assert_exact(got, O.scan(xi, init=ini), f"scan impl={impl} N={N} L={L}")
+        x = synth.items(N, L, "f32_unit")
+        assert_rel(host(C.cudanp_batched_loop_scan_variant(impl, dev(x))), O.scan(x), L, "scan f32")
+    assert C.cudanp_dp_error_count(reset=True) == 0
+
+
+# ------------------------------------------------------------------ full-size, bench configuration
+def _gen_matrix(h, w, kind):
+    A = torch.empty(h, w, dtype=torch.float32, device="cuda")
+    C.cudanp_generate(A, kind, stream_id=1)
+    return A
+
+
+def _gen_vec(n, kind, stream_id=2, dtype=torch.float32):
+    v = torch.empty(n, dtype=dtype, device="cuda")
+    C.cudanp_generate(v, kind, stream_id=stream_id)
+    return v
+
+
+def test_full_size_C2_tmv_mv_sampled():
+    """C2: 16384 x 16384 fp32, every S x dist x map (bench's sweep), sampled
+    against the oracle computing each sampled output from the generator."""
+    n = 16384
+    A = _gen_matrix(n, n, "f32_unit")
+    x = _gen_vec(n, "f32_unit")
+    rng = np.random.default_rng(0)
+    idx = np.unique(np.concatenate([rng.integers(0, n, 256), [0, 1, n - 2, n - 1]]))
+    ref_t = O.tmv_gen(n, n, idx)
+    ref_m = O.mv_gen(n, n, idx)
+    for S, dist, map_ in itertools.product(SS, DISTS, MAPS):
+        yt = host(C.cudanp_tmv(A, x, S=S, dist=dist, map=map_))
+        assert_rel(yt[idx], ref_t, n, f"C2 tmv S={S} dist={dist} map={map_}")
+        ym = host(C.cudanp_mv(A, x, S=S, dist=dist, map=map_))
+        assert_rel(ym[idx], ref_m, n, f"C2 mv S={S} dist={dist} map={map_}")
+    # exact-data invariant at full size: every variant gives identical bits (P3/P4)
+    C.cudanp_generate(A, "f32_int4", stream_id=1)
+    C.cudanp_generate(x, "f32_int4", stream_id=2)
+    base = host(C.cudanp_tmv(A, x, S=1))
+    assert_exact(base[idx], O.tmv_gen(n, n, idx, "f32_int4", "f32_int4"), "C2 tmv int4")
+    for S, dist, map_ in itertools.product(SS, DISTS, MAPS):
+        assert_exact(host(C.cudanp_tmv(A, x, S=S, dist=dist, map=map_)), base, f"P4 S={S}")
+    del A
+    torch.cuda.empty_cache()
+
+
+def test_full_size_C1_tmv_all_outputs():
+    n = 1024
+    A = _gen_matrix(n, n, "f32_unit")
+    x = _gen_vec(n, "f32_unit")
+    ref = O.tmv(host(A), host(x))
+    for S, dist, map_ in itertools.product(SS, DISTS, MAPS):
+        assert_rel(host(C.cudanp_tmv(A, x, S=S, dist=dist, map=map_)), ref, n, f"C1 S={S}")
+    assert_rel(host(C.cudanp_tmv_variant(C.S1_LITERAL, A, x)), ref, n, "C1 literal")
+
+
+def test_full_size_C3_reduce_sampled():
+    N = 1 << 22
+    rng = np.random.default_rng(1)
+    items = np.unique(np.concatenate([rng.integers(0, N, 2048), [0, N - 1]]))
+    for L in (32, 256):
+        x = torch.empty(N, L, dtype=torch.float32, device="cuda")
+        C.cudanp_generate(x, "f32_unit", stream_id=1)
+        ref = O.reduce_gen(L, items, O.F32, "f32_unit")
+        for S, dist in itertools.product(SS, DISTS):
+            got = host(C.cudanp_batched_loop_reduce(x, S=S, dist=dist, map=C.INTRA_WARP))
+            assert_rel(got[items], ref, L, f"C3 L={L} S={S} dist={dist}")
+        del x
+        xi = torch.empty(N, L, dtype=torch.int32, device="cuda")
+        C.cudanp_generate(xi, "i32_full", stream_id=1)
+        ref = O.reduce_gen(L, items, O.I32, "i32_full", op=O.MAX)
+        for S in SS:
+            got = host(C.cudanp_batched_loop_reduce(xi, op=C.MAX, S=S))
+            assert_exact(got[items], ref, f"C3 i32 max L={L} S={S}")
+        del xi
+        torch.cuda.empty_cache()
+
+
+def test_full_size_C4_scan_sampled():
+    N, L = 1 << 21, 256
+    rng = np.random.default_rng(2)
+    items = np.unique(np.concatenate([rng.integers(0, N, 512), [0, N - 1]]))
+    x = torch.empty(N, L, dtype=torch.int32, device="cuda")
+    C.cudanp_generate(x, "i32_small", stream_id=1, B=1 << 15)
+    ref = O.scan_gen(L, items, O.I32, "i32_small", B=1 << 15)
+    out = torch.empty_like(x)
+    for S, dist in itertools.product(SS, DISTS):
+        C.cudanp_batched_loop_scan(x, out=out, S=S, dist=dist, map=C.INTRA_WARP)
+        got = host(out[torch.from_numpy(items).cuda()])
+        assert_exact(got, ref, f"C4 scan S={S} dist={dist}")
+    del x, out
+    torch.cuda.empty_cache()
