@@ -51,6 +51,11 @@ def parse():
     ap.add_argument("--n", type=int, default=H, help="matrix size (default 16384 = C2)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=5)
+    ap.add_argument("--no-sweep", action="store_true",
+                    help="skip the autotune sweep and comparisons (for ncu launch lists); "
+                         "use --tmv-cfg / --mv-cfg")
+    ap.add_argument("--tmv-cfg", default="32,block,inter")
+    ap.add_argument("--mv-cfg", default="16,cyclic,intra")
     return ap.parse_args()
 
 
@@ -208,19 +213,27 @@ def run_cudanp(args):
 
     # ---- autotune sweep: every S x dist x map, per op
     sweep = {"tmv": {}, "mv": {}}
+    cfgs = [(S, d, m) for S in C.SLAVE_SIZES for d in (C.CYCLIC, C.BLOCK)
+            for m in (C.INTRA_WARP, C.INTER_WARP)]
+    if args.no_sweep:
+        def parse_cfg(s):
+            S, d, m = s.split(",")
+            return (int(S), {"cyclic": C.CYCLIC, "block": C.BLOCK}[d],
+                    {"intra": C.INTRA_WARP, "inter": C.INTER_WARP}[m])
+        cfg_of = {"tmv": [parse_cfg(args.tmv_cfg)], "mv": [parse_cfg(args.mv_cfg)]}
+    else:
+        cfg_of = {"tmv": cfgs, "mv": cfgs}
     for op, fn_np, nbytes in (("tmv", lambda S, d, m: C.cudanp_tmv(A_t, x_t, y_t, S=S, dist=d, map=m), bytes_t),
                               ("mv", lambda S, d, m: C.cudanp_mv(A_m, x_m, y_m, S=S, dist=d, map=m), bytes_m)):
-        for S in C.SLAVE_SIZES:
-            for d in (C.CYCLIC, C.BLOCK):
-                for m in (C.INTRA_WARP, C.INTER_WARP):
-                    ms = time_op(lambda: fn_np(S, d, m))
-                    ms = max_over_ranks(ms, world)
-                    sweep[op][(S, d, m)] = ms
+        for (S, d, m) in cfg_of[op]:
+            ms = time_op(lambda: fn_np(S, d, m))
+            ms = max_over_ranks(ms, world)
+            sweep[op][(S, d, m)] = ms
     best = {op: min(sweep[op], key=sweep[op].get) for op in sweep}
-    # literal S=1 (Fig 2) and DP (per-CTA) comparison, once each
+    # literal S=1 (Fig 2) and DP (per-CTA / per-thread) comparison, once each
     comp = {}
     C.cudanp_dp_set_pending_launch_limit(1 << 16)
-    for op, fn in (("tmv_s1_literal", lambda: C.cudanp_tmv_variant(C.S1_LITERAL, A_t, x_t, y_t)),
+    for op, fn in () if args.no_sweep else (("tmv_s1_literal", lambda: C.cudanp_tmv_variant(C.S1_LITERAL, A_t, x_t, y_t)),
                    ("mv_s1_literal", lambda: C.cudanp_mv_variant(C.S1_LITERAL, A_m, x_m, y_m)),
                    ("tmv_dp_block", lambda: C.cudanp_tmv_variant(C.DP_BLOCK, A_t, x_t, y_t)),
                    ("mv_dp_block", lambda: C.cudanp_mv_variant(C.DP_BLOCK, A_m, x_m, y_m)),
@@ -337,9 +350,11 @@ def run_cudanp(args):
 
     per_S = {}
     for op, nb in (("tmv", bytes_t), ("mv", bytes_m)):
-        s1 = min(v for (S, d, m), v in sweep[op].items() if S == 1)
+        s1 = min([v for (S, d, m), v in sweep[op].items() if S == 1] or [float("nan")])
         for S in C.SLAVE_SIZES:
             cand = {k: v for k, v in sweep[op].items() if k[0] == S}
+            if not cand:
+                continue
             k = min(cand, key=cand.get)
             per_S.setdefault(str(S), {})[op] = {
                 "gbs": gbs(nb, cand[k]), "ms": round(cand[k], 4),
@@ -348,8 +363,8 @@ def run_cudanp(args):
                 "map": "intra" if k[2] == C.INTRA_WARP else "inter",
                 "all": {f"{'cyc' if d == C.CYCLIC else 'blk'}/{'intra' if m == C.INTRA_WARP else 'inter'}":
                         gbs(nb, v) for (SS, d, m), v in cand.items()}}
-    s1_tmv = min(v for (S, d, m), v in sweep["tmv"].items() if S == 1)
-    s1_mv = min(v for (S, d, m), v in sweep["mv"].items() if S == 1)
+    s1_tmv = min([v for (S, d, m), v in sweep["tmv"].items() if S == 1] or [float("nan")])
+    s1_mv = min([v for (S, d, m), v in sweep["mv"].items() if S == 1] or [float("nan")])
 
     line = {
         "metric": METRIC, "value": round(value, 2), "unit": "GB/s", "n_gpus": world,

@@ -61,40 +61,48 @@ def _run(cmd: list[str]) -> None:
         sys.stderr.write(r.stderr)
 
 
-def build(force: bool = False, jobs: int | None = None, verbose: bool = False) -> str:
-    if not force and not stale():
+def build(force: bool = False, jobs: int | None = None, verbose: bool = False,
+          defines: tuple[str, ...] = (), out: str | None = None) -> str:
+    """Build libcudanp.so.  `defines`/`out` build an experiment variant (e.g.
+    -DCUDANP_TMV_U=4) into another file and build directory."""
+    lib = out or LIB
+    if not force and not defines and out is None and not stale():
         return LIB
-    os.makedirs(BUILD, exist_ok=True)
+    bdir = BUILD if not defines else BUILD + "_" + "_".join(d.replace("=", "") for d in defines)
+    os.makedirs(bdir, exist_ok=True)
+    dflags = ["-D" + d for d in defines]
     cc = nvcc()
     objs, cmds = [], []
     for s in SOURCES:
-        o = os.path.join(BUILD, s.replace(".cu", ".o"))
+        o = os.path.join(bdir, s.replace(".cu", ".o"))
         objs.append(o)
-        cmds.append([cc, *ARCH, *NVFLAGS, "-c", os.path.join(CSRC, s), "-o", o])
+        cmds.append([cc, *ARCH, *NVFLAGS, *dflags, "-c", os.path.join(CSRC, s), "-o", o])
     rdc_objs = []
     for s in RDC_SOURCES:
-        o = os.path.join(BUILD, s.replace(".cu", ".o"))
+        o = os.path.join(bdir, s.replace(".cu", ".o"))
         rdc_objs.append(o)
-        cmds.append([cc, *ARCH, *NVFLAGS, "-rdc=true", "-c", os.path.join(CSRC, s), "-o", o])
+        cmds.append([cc, *ARCH, *NVFLAGS, *dflags, "-rdc=true", "-c", os.path.join(CSRC, s), "-o", o])
     with ThreadPoolExecutor(max_workers=jobs or os.cpu_count() or 4) as ex:
         list(ex.map(_run, cmds))
-    dlink = os.path.join(BUILD, "dp_dlink.o")
+    dlink = os.path.join(bdir, "dp_dlink.o")
     _run([cc, *ARCH, "-Xcompiler", "-fPIC", "-dlink", *rdc_objs, "-o", dlink, "-lcudadevrt"])
-    tmp = LIB + f".tmp{os.getpid()}"
+    tmp = lib + f".tmp{os.getpid()}"
     _run([cc, *ARCH, "-shared", "-Xcompiler", "-fPIC", "-o", tmp, *objs, *rdc_objs, dlink,
           "-lcudadevrt", "-cudart", "static"])
-    os.replace(tmp, LIB)
+    os.replace(tmp, lib)
     if verbose:
-        print("built", LIB)
-    return LIB
+        print("built", lib)
+    return lib
 
 
 def main() -> None:
     ap = argparse.ArgumentParser()
     ap.add_argument("--force", action="store_true")
     ap.add_argument("-j", type=int, default=None)
+    ap.add_argument("-D", dest="defines", action="append", default=[])
+    ap.add_argument("--out", default=None)
     a = ap.parse_args()
-    build(force=a.force, jobs=a.j, verbose=True)
+    build(force=a.force, jobs=a.j, verbose=True, defines=tuple(a.defines), out=a.out)
 
 
 if __name__ == "__main__":

@@ -109,8 +109,19 @@ static int check_mv_args(const float* A, int64_t lda, const float* x, float* y, 
   return CUDANP_OK;
 }
 
+// TMV masters are columns: 128-bit loads give each thread 4 adjacent
+// masters (R19), which divides the CTA count by 4.  Measured on B200 (C1
+// 1024^2 vs C2 16384^2, profiles/): V=4 wins as long as the 4-wide grid has at
+// least half an SM's worth of CTAs per SM pair (>= SMs/2 CTAs); for narrower
+// matrices one master per thread (plus 8-master CTAs, np_matvec.cu) spreads
+// the few columns over more SMs.
 static bool tmv_vec(const float* A, int64_t lda, const float* y, int64_t w) {
-  return (w % 4 == 0) && (lda % 4 == 0) && aligned16(A) && aligned16(y);
+  const bool aligned = (w % 4 == 0) && (lda % 4 == 0) && aligned16(A) && aligned16(y);
+#if defined(CUDANP_TMV_VEC_ALWAYS)
+  return aligned;
+#else
+  return aligned && 2 * ((w + 127) / 128) >= sm_count();
+#endif
 }
 static bool mv_vec(const float* A, int64_t lda, const float* x, int64_t w) {
   return (w % 4 == 0) && (lda % 4 == 0) && aligned16(A) && aligned16(x);

@@ -49,6 +49,10 @@ template <> __device__ __forceinline__ int32_t OpMax::identity<int32_t>() { retu
 template <class T> struct V4 { T x, y, z, w; };
 
 // Streaming 128-bit load through the read-only path (LDG.E.128.CONSTANT).
+// The asm stays `volatile`: a non-volatile asm with no memory operand counts
+// as side-effect free, so the compiler may speculate it past the bound checks
+// of the loop (an out-of-bounds load).  Load batching comes from the register
+// budget given in __launch_bounds__, not from dropping volatile.
 template <class T>
 __device__ __forceinline__ V4<T> ldg4(const T* p) {
   V4<T> r;

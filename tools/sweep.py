@@ -1,0 +1,248 @@
+#!/usr/bin/env python
+"""Sweep every config of BASELINE.json (C1-C5 at G=1) over S x dist x map,
+plus the S=1 literal (Fig 2) and dynamic-parallelism comparison kernels --
+the analog of the paper's Figs 11, 13, 14 and its DP comparison.
+
+    python tools/sweep.py [--configs C1,C2,C3,C4,C5] [--out gpurun_out/sweep.jsonl]
+
+One JSON record per (config, op, dtype, L, S, dist, map, impl): median time,
+algorithmic bytes, GB/s, fraction of the measured HBM peak, speedup vs the
+best S=1 NP-path kernel ("tuned S=1") and vs the literal Fig 2 kernel.
+Timing: CUDA events on the launching stream, 2 warm-ups, median of reps.
+Inputs >= 512 MB exceed the 126 MB L2; C1 (4 MiB) is timed as a CUDA graph
+of 64 launches over 64 distinct copies (256 MiB) so every launch reads cold.
+"""
+from __future__ import annotations
+
+import argparse
+import itertools
+import json
+import os
+import statistics
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import torch  # noqa: E402
+
+from paper_conf_ppopp_yangz14_b200 import cudanp as C  # noqa: E402
+
+PEAK = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json"))).get("hbm_gbs", 6537.0) \
+    if os.path.exists(os.path.join(ROOT, "MEASURED_PEAKS.json")) else 6537.0
+DN = {C.CYCLIC: "cyclic", C.BLOCK: "block"}
+MN = {C.INTRA_WARP: "intra", C.INTER_WARP: "inter"}
+OUT = None
+
+
+def emit(rec):
+    rec["frac_hbm"] = round(rec["gbs"] / PEAK, 4) if rec.get("gbs") else None
+    line = json.dumps(rec)
+    print(line, flush=True)
+    if OUT:
+        OUT.write(line + "\n")
+        OUT.flush()
+
+
+def time_ms(fn, reps=5, warm=2):
+    st = torch.cuda.current_stream()
+    for _ in range(warm):
+        fn()
+    ts = []
+    for _ in range(reps):
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(st)
+        fn()
+        b.record(st)
+        b.synchronize()
+        ts.append(a.elapsed_time(b))
+    return statistics.median(ts), min(ts)
+
+
+def graph_time_ms(fns, reps=5):
+    """Capture a CUDA graph calling every fn once; return per-launch time."""
+    s = torch.cuda.Stream()
+    s.wait_stream(torch.cuda.current_stream())
+    with torch.cuda.stream(s):
+        for f in fns:
+            f()
+    torch.cuda.current_stream().wait_stream(s)
+    torch.cuda.synchronize()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g):
+        for f in fns:
+            f()
+    g.replay()
+    torch.cuda.synchronize()
+    ts = []
+    for _ in range(reps):
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record()
+        g.replay()
+        b.record()
+        b.synchronize()
+        ts.append(a.elapsed_time(b) / len(fns))
+    return statistics.median(ts), min(ts)
+
+
+def sweep_np(cfg, op, nbytes, run, extra, s1_ref=None, literal=None, comps=()):
+    """run(S, dist, map) -> (median_ms, min_ms)."""
+    res = {}
+    for S, d, m in itertools.product(C.SLAVE_SIZES, (C.CYCLIC, C.BLOCK), (C.INTRA_WARP, C.INTER_WARP)):
+        res[(S, d, m)] = run(S, d, m)
+    s1 = min(v[0] for k, v in res.items() if k[0] == 1)
+    for (S, d, m), (med, mn) in res.items():
+        rec = {"config": cfg, "op": op, **extra, "S": S, "dist": DN[d], "map": MN[m], "impl": "np",
+               "t_median_us": round(med * 1e3, 2), "t_min_us": round(mn * 1e3, 2),
+               "alg_bytes": nbytes, "gbs": round(nbytes / (med * 1e-3) / 1e9, 1),
+               "speedup_vs_s1_tuned": round(s1 / med, 3)}
+        if literal:
+            rec["speedup_vs_s1_literal"] = round(literal / med, 3)
+        emit(rec)
+    best = min(res, key=lambda k: res[k][0])
+    for name, t in comps:
+        emit({"config": cfg, "op": op, **extra, "impl": name, "t_median_us": round(t * 1e3, 2),
+              "alg_bytes": nbytes, "gbs": round(nbytes / (t * 1e-3) / 1e9, 1),
+              "speedup_of_best_np": round(t / res[best][0], 3)})
+    bS, bd, bm = best
+    emit({"config": cfg, "op": op, **extra, "impl": "best_np", "S": bS, "dist": DN[bd], "map": MN[bm],
+          "t_median_us": round(res[best][0] * 1e3, 2), "alg_bytes": nbytes,
+          "gbs": round(nbytes / (res[best][0] * 1e-3) / 1e9, 1),
+          "speedup_vs_s1_tuned": round(s1 / res[best][0], 3),
+          **({"speedup_vs_s1_literal": round(literal / res[best][0], 3)} if literal else {})})
+    return res, best
+
+
+def gen(shape, kind, dtype=torch.float32, stream_id=1, B=1 << 20):
+    t = torch.empty(*shape, dtype=dtype, device="cuda")
+    C.cudanp_generate(t, kind, stream_id=stream_id, B=B)
+    return t
+
+
+def c1():
+    n, copies = 1024, 64
+    As = [gen((n, n), "f32_unit") for _ in range(copies)]
+    x = gen((n,), "f32_unit", stream_id=2)
+    ys = [torch.empty(n, device="cuda") for _ in range(copies)]
+    nb = 4 * n * n + 8 * n
+
+    def run(S, d, m):
+        return graph_time_ms([lambda i=i: C.cudanp_tmv(As[i], x, ys[i], S=S, dist=d, map=m)
+                              for i in range(copies)])
+    lit = graph_time_ms([lambda i=i: C.cudanp_tmv_variant(C.S1_LITERAL, As[i], x, ys[i]) for i in range(copies)])[0]
+    comps = [("s1_literal", lit)]
+    for impl, name in ((C.DP_BLOCK, "dp_block"), (C.DP_THREAD, "dp_thread")):
+        comps.append((name, time_ms(lambda: C.cudanp_tmv_variant(impl, As[0], x, ys[0]), reps=5)[0]))
+    sweep_np("C1", "tmv", nb, run, {"dtype": "f32", "N": n, "L": n}, literal=lit, comps=comps)
+
+
+def c2():
+    n = 16384
+    A = gen((n, n), "f32_unit")
+    x = gen((n,), "f32_unit", stream_id=2)
+    y = torch.empty(n, device="cuda")
+    nb = 4 * n * n + 8 * n
+    for op, fnp, fv in (("tmv", C.cudanp_tmv, C.cudanp_tmv_variant), ("mv", C.cudanp_mv, C.cudanp_mv_variant)):
+        lit = time_ms(lambda: fv(C.S1_LITERAL, A, x, y), reps=3)[0]
+        comps = [("s1_literal", lit)]
+        for impl, name in ((C.DP_BLOCK, "dp_block"), (C.DP_THREAD, "dp_thread")):
+            comps.append((name, time_ms(lambda: fv(impl, A, x, y), reps=3, warm=1)[0]))
+        sweep_np("C2", op, nb, lambda S, d, m: time_ms(lambda: fnp(A, x, y, S=S, dist=d, map=m)),
+                 {"dtype": "f32", "N": n, "L": n}, literal=lit, comps=comps)
+    del A
+
+
+def c3(Ls=(32, 64, 128, 256, 80, 150)):
+    N = 1 << 22
+    for L in Ls:
+        for dtype, op, kind, tdt in ((C.F32, C.SUM, "f32_unit", torch.float32),
+                                     (C.F32, C.MAX, "f32_signed", torch.float32),
+                                     (C.I32, C.SUM, "i32_small", torch.int32),
+                                     (C.I32, C.MAX, "i32_full", torch.int32)):
+            x = gen((N, L), kind, tdt)
+            out = torch.empty(N, dtype=tdt, device="cuda")
+            nb = 4 * N * L + 4 * N
+            lit = time_ms(lambda: C.cudanp_batched_loop_reduce_variant(C.S1_LITERAL, x, None, out, op=op))[0]
+            comps = [("s1_literal", lit),
+                     ("dp_block", time_ms(lambda: C.cudanp_batched_loop_reduce_variant(C.DP_BLOCK, x, None, out, op=op), reps=3, warm=1)[0])]
+            # DP per thread: one device launch per item -> measured on a 65,536-item prefix
+            Np = 65536
+            xp, op_ = x[:Np], out[:Np]
+            tp = time_ms(lambda: C.cudanp_batched_loop_reduce_variant(C.DP_THREAD, xp, None, op_, op=op), reps=3, warm=1)[0]
+            comps.append(("dp_thread_prefix65536_scaled", tp * N / Np))
+            sweep_np("C3", "reduce", nb,
+                     lambda S, d, m: time_ms(lambda: C.cudanp_batched_loop_reduce(x, None, out, op=op, S=S, dist=d, map=m)),
+                     {"dtype": "f32" if dtype == C.F32 else "i32", "opname": "sum" if op == C.SUM else "max",
+                      "N": N, "L": L}, literal=lit, comps=comps)
+            del x, out
+            torch.cuda.empty_cache()
+
+
+def c4(Ls=(64, 128, 256, 512, 1024)):
+    N = 1 << 21
+    for L in Ls:
+        for dtype, kind, tdt in ((C.I32, "i32_small", torch.int32), (C.F32, "f32_unit", torch.float32)):
+            x = gen((N, L), kind, tdt, B=1 << 15)
+            out = torch.empty_like(x)
+            nb = 8 * N * L
+            lit = time_ms(lambda: C.cudanp_batched_loop_scan_variant(C.S1_LITERAL, x, None, out), reps=3)[0]
+            comps = [("s1_literal", lit),
+                     ("dp_block", time_ms(lambda: C.cudanp_batched_loop_scan_variant(C.DP_BLOCK, x, None, out), reps=3, warm=1)[0])]
+            Np = 65536
+            xp, op_ = x[:Np], out[:Np]
+            tp = time_ms(lambda: C.cudanp_batched_loop_scan_variant(C.DP_THREAD, xp, None, op_), reps=3, warm=1)[0]
+            comps.append(("dp_thread_prefix65536_scaled", tp * N / Np))
+            sweep_np("C4", "scan", nb,
+                     lambda S, d, m: time_ms(lambda: C.cudanp_batched_loop_scan(x, None, out, S=S, dist=d, map=m), reps=3),
+                     {"dtype": "f32" if dtype == C.F32 else "i32", "N": N, "L": L}, literal=lit, comps=comps)
+            del x, out
+            torch.cuda.empty_cache()
+
+
+def c5():
+    n = 65536
+    A = gen((n, n), "f32_unit")
+    x = gen((n,), "f32_unit", stream_id=2)
+    y = torch.empty(n, device="cuda")
+    nb = 4 * n * n + 8 * n
+    for S, d in itertools.product((8, 16, 32), (C.CYCLIC, C.BLOCK)):
+        med, mn = time_ms(lambda: C.cudanp_tmv(A, x, y, S=S, dist=d, map=C.INTER_WARP), reps=3)
+        emit({"config": "C5", "op": "tmv", "dtype": "f32", "N": n, "L": n, "G": 1, "S": S, "dist": DN[d],
+              "map": "inter", "impl": "np", "t_median_us": round(med * 1e3, 1), "alg_bytes": nb,
+              "gbs": round(nb / (med * 1e-3) / 1e9, 1)})
+    del A
+    torch.cuda.empty_cache()
+    N, L = 1 << 26, 64
+    xr = gen((N, L), "f32_unit")
+    out = torch.empty(N, device="cuda")
+    nb = 4 * N * L + 4 * N
+    for S, d in itertools.product((4, 8, 16), (C.CYCLIC, C.BLOCK)):
+        med, mn = time_ms(lambda: C.cudanp_batched_loop_reduce(xr, None, out, S=S, dist=d, map=C.INTRA_WARP), reps=3)
+        emit({"config": "C5", "op": "reduce", "dtype": "f32", "N": N, "L": L, "G": 1, "S": S, "dist": DN[d],
+              "map": "intra", "impl": "np", "t_median_us": round(med * 1e3, 1), "alg_bytes": nb,
+              "gbs": round(nb / (med * 1e-3) / 1e9, 1)})
+    del xr, out
+    torch.cuda.empty_cache()
+
+
+def main():
+    global OUT
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--configs", default="C1,C2,C3,C4,C5")
+    ap.add_argument("--out", default=os.path.join(ROOT, "gpurun_out", "sweep.jsonl"))
+    ap.add_argument("--lib", default=None, help="alternative libcudanp.so (build experiments)")
+    a = ap.parse_args()
+    os.makedirs(os.path.dirname(a.out), exist_ok=True)
+    OUT = open(a.out, "w")
+    C.load(a.lib) if a.lib else C.load()
+    C.cudanp_dp_set_pending_launch_limit(1 << 17)
+    t0 = time.time()
+    for c in a.configs.split(","):
+        {"C1": c1, "C2": c2, "C3": c3, "C4": c4, "C5": c5}[c.strip()]()
+        print(f"# {c} done at {time.time() - t0:.0f}s", file=sys.stderr, flush=True)
+    print(f"# dp launch errors: {C.cudanp_dp_error_count(reset=True)}", file=sys.stderr)
+
+
+if __name__ == "__main__":
+    main()
