@@ -93,6 +93,22 @@ int cudanp_batched_loop_scan(const void* in, const void* init, void* out,
                              int64_t n_outer, int64_t n_inner, int dtype,
                              int S, int dist, int map, void* stream);
 
+/* Ragged (runtime-bounded) loop-reduce over CSR segments (
+ * P:193 "valid if the loop bound is determined at the runtime"):
+ * out[n] = init[n] (op) fold_{offsets[n] <= i < offsets[n+1]} in[i], n < N.
+ * offsets: N+1 int64 device values (8-byte aligned), non-decreasing; a
+ * decreasing pair is treated as an empty loop.  The master of item n loads
+ * its two bounds and broadcasts them with read_from_master;
+ * the team streams the segment (head <= 3 scalars, 128-bit aligned body,
+ * tail <= 3 scalars).  in and offsets must be non-NULL when N > 0.  dtype,
+ * op, init, S, dist, map as for cudanp_batched_loop_reduce. */
+int cudanp_ragged_loop_reduce(const void* in, const int64_t* offsets, const void* init, void* out,
+                              int64_t n_outer, int dtype, int op, int S, int dist, int map,
+                              void* stream);
+/* Comparison: one thread per segment, serial loop (Fig 2 style). */
+int cudanp_ragged_loop_reduce_literal(const void* in, const int64_t* offsets, const void* init,
+                                      void* out, int64_t n_outer, int dtype, int op, void* stream);
+
 /* ------------------------------------------------------------------------
  * Comparison kernels.  Same operands as the NP
  * call; `impl` selects:

@@ -70,6 +70,8 @@ def lib():
                 "orc_reduce_i32": (None, [_vp, _vp, _vp, _i64, _i64, _int]),
                 "orc_scan_f32": (None, [_vp, _vp, _vp, _i64, _i64]),
                 "orc_scan_i32": (None, [_vp, _vp, _vp, _i64, _i64]),
+                "orc_ragged_reduce_f32": (None, [_vp, _vp, _vp, _vp, _i64, _int]),
+                "orc_ragged_reduce_i32": (None, [_vp, _vp, _vp, _vp, _i64, _int]),
                 "orc_tmv_gen": (None, [_u64, _int, _int, _i64, _i64, _vp, _i64, _vp]),
                 "orc_mv_gen": (None, [_u64, _int, _int, _i64, _i64, _vp, _i64, _vp]),
                 "orc_reduce_gen": (None, [_u64, _int, _int, _i64, _int, _i64, _int, _vp, _i64, _vp]),
@@ -170,6 +172,21 @@ def scan(x: np.ndarray, init: np.ndarray | None = None) -> np.ndarray:
         lib().orc_scan_i32(_p(x), _p(init), _p(out), N, L)
     else:
         raise TypeError(x.dtype)
+    return out
+
+
+def ragged_reduce(x: np.ndarray, offsets: np.ndarray, op: int = SUM,
+                  init: np.ndarray | None = None) -> np.ndarray:
+    """out[n] = init[n] (op) fold_{offsets[n] <= i < offsets[n+1]} x[i] (P:193, P:209)."""
+    x = np.ascontiguousarray(x)
+    offsets = np.ascontiguousarray(offsets, np.int64)
+    N = len(offsets) - 1
+    out = np.empty(N, x.dtype)
+    if init is not None:
+        init = np.ascontiguousarray(init, x.dtype)
+    f = {np.dtype(np.float32): lib().orc_ragged_reduce_f32,
+         np.dtype(np.int32): lib().orc_ragged_reduce_i32}[x.dtype]
+    f(_p(x), _p(offsets), _p(init), _p(out), N, op)
     return out
 
 

@@ -29,6 +29,9 @@ int dp_mv(bool, const float*, int64_t, const float*, float*, int64_t, int64_t, c
 int dp_reduce(bool, const void*, const void*, void*, int64_t, int64_t, int, int, cudaStream_t);
 int dp_scan(bool, const void*, const void*, void*, int64_t, int64_t, int, cudaStream_t);
 int dp_error_count(int, int64_t*);
+int ragged_np(const void*, const int64_t*, const void*, void*, int64_t, int, int, int, int, int,
+              cudaStream_t);
+int ragged_literal(const void*, const int64_t*, const void*, void*, int64_t, int, int, cudaStream_t);
 
 static thread_local char g_err[512] = "";
 
@@ -268,6 +271,35 @@ int cudanp_batched_loop_scan(const void* in, const void* init, void* out, int64_
   const bool vec = (n_inner % 4 == 0) && aligned16(in) && aligned16(out);
   return scan_np(in, init, out, n_outer, n_inner, dtype, S, dist, resolve_map(map, false), vec,
                  as_stream(stream), nullptr);
+}
+
+// ---------------------------------------------------------------- ragged (f1)
+static int check_ragged(const void* in, const int64_t* off, void* out, int64_t N, int S, int dist,
+                        int map, int dtype, int op) {
+  int rc = check_common(S, dist, map, N, 0);
+  if (rc) return rc;
+  rc = check_dtype_op(dtype, op);
+  if (rc) return rc;
+  if (N > 0 && (!in || !off || !out)) return fail_invalid("in, offsets or out is NULL");
+  if (((uintptr_t)off & 7u) != 0) return fail_invalid("offsets must be 8-byte aligned");
+  if (((uintptr_t)in & 3u) != 0) return fail_invalid("in must be 4-byte aligned");
+  return CUDANP_OK;
+}
+
+int cudanp_ragged_loop_reduce(const void* in, const int64_t* offsets, const void* init, void* out,
+                              int64_t n_outer, int dtype, int op, int S, int dist, int map,
+                              void* stream) {
+  int rc = check_ragged(in, offsets, out, n_outer, S, dist, map, dtype, op);
+  if (rc) return rc;
+  return ragged_np(in, offsets, init, out, n_outer, dtype, op, S, dist, resolve_map(map, false),
+                   as_stream(stream));
+}
+
+int cudanp_ragged_loop_reduce_literal(const void* in, const int64_t* offsets, const void* init,
+                                      void* out, int64_t n_outer, int dtype, int op, void* stream) {
+  int rc = check_ragged(in, offsets, out, n_outer, 1, 0, 0, dtype, op);
+  if (rc) return rc;
+  return ragged_literal(in, offsets, init, out, n_outer, dtype, op, as_stream(stream));
 }
 
 // ---------------------------------------------------------------- variants

@@ -38,6 +38,8 @@ _SIGS = {
     "cudanp_mv": [_vp, _i64, _vp, _vp, _i64, _i64, _int, _int, _int, _vp],
     "cudanp_batched_loop_reduce": [_vp, _vp, _vp, _i64, _i64, _int, _int, _int, _int, _int, _vp],
     "cudanp_batched_loop_scan": [_vp, _vp, _vp, _i64, _i64, _int, _int, _int, _int, _vp],
+    "cudanp_ragged_loop_reduce": [_vp, _vp, _vp, _vp, _i64, _int, _int, _int, _int, _int, _vp],
+    "cudanp_ragged_loop_reduce_literal": [_vp, _vp, _vp, _vp, _i64, _int, _int, _vp],
     "cudanp_tmv_variant": [_int, _vp, _i64, _vp, _vp, _i64, _i64, _vp],
     "cudanp_mv_variant": [_int, _vp, _i64, _vp, _vp, _i64, _i64, _vp],
     "cudanp_batched_loop_reduce_variant": [_int, _vp, _vp, _vp, _i64, _i64, _int, _int, _vp],
@@ -167,6 +169,33 @@ def cudanp_batched_loop_scan(x, init=None, out=None, *, S=8, dist=CYCLIC, map=AU
     _check(load().cudanp_batched_loop_scan(_ptr(x), _ptr(init), _ptr(out), N, L, _dtype_code(x),
                                            S, dist, map, _stream(stream)),
            "cudanp_batched_loop_scan")
+    return out
+
+
+def cudanp_ragged_loop_reduce(x, offsets, init=None, out=None, *, op=SUM, S=8, dist=CYCLIC,
+                              map=AUTO, stream=None):
+    """out[n] = init[n] (op) fold_{offsets[n] <= i < offsets[n+1]} x[i] (P:193).
+    x: 1-D fp32/int32; offsets: 1-D int64 of N+1 entries."""
+    import torch
+    if offsets.dtype != torch.int64:
+        raise TypeError("offsets must be int64")
+    N = offsets.shape[0] - 1
+    if out is None:
+        out = torch.empty(N, dtype=x.dtype, device=x.device)
+    _check(load().cudanp_ragged_loop_reduce(_ptr(x), _ptr(offsets), _ptr(init), _ptr(out), N,
+                                            _dtype_code(x), op, S, dist, map, _stream(stream)),
+           "cudanp_ragged_loop_reduce")
+    return out
+
+
+def cudanp_ragged_loop_reduce_literal(x, offsets, init=None, out=None, *, op=SUM, stream=None):
+    import torch
+    N = offsets.shape[0] - 1
+    if out is None:
+        out = torch.empty(N, dtype=x.dtype, device=x.device)
+    _check(load().cudanp_ragged_loop_reduce_literal(_ptr(x), _ptr(offsets), _ptr(init), _ptr(out),
+                                                    N, _dtype_code(x), op, _stream(stream)),
+           "cudanp_ragged_loop_reduce_literal")
     return out
 
 

@@ -86,3 +86,26 @@ def items(N: int, L: int, kind: str, B: int = 1 << 20, seed: int = SEED, n0: int
 
 def init(N: int, kind: str, B: int = 1 << 20, seed: int = SEED, n0: int = 0):
     return gen(STREAM_INIT, kind, n0, N, B, seed)
+
+
+STREAM_LEN = 4
+
+
+def lengths(N: int, mean: int, dist: str = "uniform", seed: int = SEED, cap: int | None = None):
+    """Per-item loop trip counts (structure of a ragged workload):
+    'uniform' -> integers in [0, 2*mean]; 'exp' -> floor(-mean*ln(u)), an
+    exponential (skewed) mix capped at `cap` (default 16*mean)."""
+    h = hash64(STREAM_LEN, np.arange(N, dtype=np.uint64), seed)
+    if dist == "uniform":
+        return ((h >> np.uint64(32)) % np.uint64(2 * mean + 1)).astype(np.int64)
+    if dist == "exp":
+        u = ((h >> np.uint64(11)).astype(np.float64) + 1.0) * 2.0 ** -53
+        L = np.floor(-mean * np.log(u)).astype(np.int64)
+        return np.minimum(L, cap if cap is not None else 16 * mean)
+    raise ValueError(dist)
+
+
+def offsets_from_lengths(lens):
+    off = np.zeros(len(lens) + 1, np.int64)
+    np.cumsum(lens, out=off[1:])
+    return off

@@ -370,3 +370,43 @@ def test_team_ids_reject(orc):
         orc.team_ids(3, orc.INTRA_WARP, 32)
     with pytest.raises(ValueError):
         orc.owner_map(4, 0, orc.CYCLIC)
+
+
+# ------------------------------------------------------------------ ragged (f1)
+def test_ragged_equal_lengths_is_batched_reduce(orc):
+    # second formulation: equal segment lengths L reduce to the batched op
+    N, L = 37, 13
+    for kind, dt in [("f32_signed", np.float32), ("i32_full", np.int32)]:
+        x = synth.items(N, L, kind)
+        off = np.arange(N + 1, dtype=np.int64) * L
+        for op in (orc.SUM, orc.MAX):
+            assert orc.ragged_reduce(x.reshape(-1), off, op=op).tobytes() == orc.reduce(x, op=op).tobytes()
+
+
+def test_ragged_bruteforce_and_empty(orc):
+    lens = synth.lengths(60, 7)
+    assert (lens == 0).any()
+    off = synth.offsets_from_lengths(lens)
+    x = synth.gen(1, "f32_signed", 0, int(off[-1]))
+    y = orc.ragged_reduce(x, off)
+    for n in range(60):
+        s = sum((Fraction(float(v)) for v in x[off[n]:off[n + 1]]), Fraction(0))
+        assert y[n] == np.float32(float(s))
+    ym = orc.ragged_reduce(x, off, op=orc.MAX)
+    for n in range(60):
+        seg = x[off[n]:off[n + 1]]
+        assert ym[n] == (seg.max() if len(seg) else -np.inf)
+    ini = synth.init(60, "f32_int4")
+    yi = orc.ragged_reduce(x, off, init=ini)
+    assert (yi[lens == 0] == ini[lens == 0]).all()
+    # decreasing offset pair -> empty loop
+    off2 = np.array([0, 5, 3, 8], np.int64)
+    xi = np.arange(8, dtype=np.int32)
+    assert orc.ragged_reduce(xi, off2).tolist() == [10, 0, 3 + 4 + 5 + 6 + 7]
+
+
+def test_ragged_lengths_distributions():
+    u = synth.lengths(100000, 64, "uniform")
+    assert u.min() == 0 and u.max() == 128 and abs(u.mean() - 64) < 1
+    e = synth.lengths(100000, 64, "exp")
+    assert e.min() == 0 and e.max() <= 16 * 64 and abs(e.mean() - 64) < 2

@@ -226,10 +226,29 @@ def c5():
     torch.cuda.empty_cache()
 
 
+def r1(means=(16, 64, 256)):
+    """f1: ragged CSR segments, N = 4M items, uniform and exponential lengths."""
+    import synth
+    N = 1 << 22
+    for mean in means:
+        for dist in ("uniform", "exp"):
+            off = torch.from_numpy(synth.offsets_from_lengths(synth.lengths(N, mean, dist))).cuda()
+            total = int(off[-1].item())
+            x = gen((total,), "f32_unit")
+            out = torch.empty(N, device="cuda")
+            nb = 4 * total + 8 * (N + 1) + 4 * N
+            lit = time_ms(lambda: C.cudanp_ragged_loop_reduce_literal(x, off, None, out))[0]
+            sweep_np("R1", "ragged_reduce", nb,
+                     lambda S, d, m: time_ms(lambda: C.cudanp_ragged_loop_reduce(x, off, None, out, S=S, dist=d, map=m)),
+                     {"dtype": "f32", "N": N, "L": f"{dist}{mean}"}, literal=lit, comps=[("s1_literal", lit)])
+            del x, out, off
+            torch.cuda.empty_cache()
+
+
 def main():
     global OUT
     ap = argparse.ArgumentParser()
-    ap.add_argument("--configs", default="C1,C2,C3,C4,C5")
+    ap.add_argument("--configs", default="C1,C2,C3,C4,C5,R1")
     ap.add_argument("--out", default=os.path.join(ROOT, "gpurun_out", "sweep.jsonl"))
     ap.add_argument("--lib", default=None, help="alternative libcudanp.so (build experiments)")
     a = ap.parse_args()
@@ -239,7 +258,7 @@ def main():
     C.cudanp_dp_set_pending_launch_limit(1 << 17)
     t0 = time.time()
     for c in a.configs.split(","):
-        {"C1": c1, "C2": c2, "C3": c3, "C4": c4, "C5": c5}[c.strip()]()
+        {"C1": c1, "C2": c2, "C3": c3, "C4": c4, "C5": c5, "R1": r1}[c.strip()]()
         print(f"# {c} done at {time.time() - t0:.0f}s", file=sys.stderr, flush=True)
     print(f"# dp launch errors: {C.cudanp_dp_error_count(reset=True)}", file=sys.stderr)
 
