@@ -109,6 +109,27 @@ int cudanp_ragged_loop_reduce(const void* in, const int64_t* offsets, const void
 int cudanp_ragged_loop_reduce_literal(const void* in, const int64_t* offsets, const void* init,
                                       void* out, int64_t n_outer, int dtype, int op, void* stream);
 
+/* Multi-section items, the LE kernel of Figs 5-6 (SURVEY §8(f)
+ * f2): per item n with L = n_inner points Grad[i] = in(n, i):
+ *   sum = reduction(Grad); ave = sum / L;
+ *   var = reduction((Grad-ave)^2); ep = reduction(Grad-ave);
+ *   if ((ave*ave)/var > threshold) gicov[n] = ave / sqrt(var)   (master only)
+ * gicov[n] is left untouched when the test fails.  ave, var,
+ * ep (N floats each) may be NULL.  layout 0: in[n*L + i] (item-major);
+ * layout 1: in[i*N + n] (point-major).  Grad stays in the slaves' registers
+ * between the loops (Fig 6c) when ceil(L/S) <= 32.  S: 1,2,4,8,16,32 for
+ * both maps, and also 3,5,10,15 for CUDANP_MAP_INTER_WARP (Fig 12);
+ * a non-power-of-two S with the intra-warp map returns
+ * CUDANP_ERR_UNSUPPORTED.  L must be >= 1 when N > 0. */
+int cudanp_le_gicov(const float* in, float* gicov, float* ave, float* var, float* ep,
+                    int64_t n_outer, int64_t n_inner, float threshold, int layout, int S,
+                    int dist, int map, void* stream);
+/* Comparison: Fig 5 as written, one thread per item, Grad in a per-thread
+ * local-memory array when L <= 256. */
+int cudanp_le_gicov_literal(const float* in, float* gicov, float* ave, float* var, float* ep,
+                            int64_t n_outer, int64_t n_inner, float threshold, int layout,
+                            void* stream);
+
 /* ------------------------------------------------------------------------
  * Comparison kernels.  Same operands as the NP
  * call; `impl` selects:

@@ -72,6 +72,7 @@ def lib():
                 "orc_scan_i32": (None, [_vp, _vp, _vp, _i64, _i64]),
                 "orc_ragged_reduce_f32": (None, [_vp, _vp, _vp, _vp, _i64, _int]),
                 "orc_ragged_reduce_i32": (None, [_vp, _vp, _vp, _vp, _i64, _int]),
+                "orc_le_gicov": (None, [_vp, _vp, _vp, _vp, _vp, _i64, _i64, ctypes.c_float, _int]),
                 "orc_tmv_gen": (None, [_u64, _int, _int, _i64, _i64, _vp, _i64, _vp]),
                 "orc_mv_gen": (None, [_u64, _int, _int, _i64, _i64, _vp, _i64, _vp]),
                 "orc_reduce_gen": (None, [_u64, _int, _int, _i64, _int, _i64, _int, _vp, _i64, _vp]),
@@ -188,6 +189,18 @@ def ragged_reduce(x: np.ndarray, offsets: np.ndarray, op: int = SUM,
          np.dtype(np.int32): lib().orc_ragged_reduce_i32}[x.dtype]
     f(_p(x), _p(offsets), _p(init), _p(out), N, op)
     return out
+
+
+def le_gicov(x: np.ndarray, thr: float, layout: int = 0, gicov_fill: float = -1.0):
+    """Fig 5: per item, ave, var, ep and the conditional gicov.
+    x is (N, L) for layout 0 (item-major) or (L, N) for layout 1 (point-major).
+    Items whose test fails keep gicov_fill."""
+    x = np.ascontiguousarray(x, np.float32)
+    N, L = (x.shape if layout == 0 else x.shape[::-1])
+    g = np.full(N, gicov_fill, np.float32)
+    a, v, e = (np.empty(N, np.float32) for _ in range(3))
+    lib().orc_le_gicov(_p(x), _p(g), _p(a), _p(v), _p(e), N, L, thr, layout)
+    return g, a, v, e
 
 
 def tmv_gen(h: int, w: int, cols, kindA="f32_unit", kindx="f32_unit", seed: int = SEED) -> np.ndarray:

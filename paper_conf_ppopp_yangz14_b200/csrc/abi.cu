@@ -32,6 +32,10 @@ int dp_error_count(int, int64_t*);
 int ragged_np(const void*, const int64_t*, const void*, void*, int64_t, int, int, int, int, int,
               cudaStream_t);
 int ragged_literal(const void*, const int64_t*, const void*, void*, int64_t, int, int, cudaStream_t);
+int le_np(const float*, float*, float*, float*, float*, int64_t, int64_t, float, int, int, int, int,
+          cudaStream_t);
+int le_literal(const float*, float*, float*, float*, float*, int64_t, int64_t, float, int,
+               cudaStream_t);
 
 static thread_local char g_err[512] = "";
 
@@ -300,6 +304,38 @@ int cudanp_ragged_loop_reduce_literal(const void* in, const int64_t* offsets, co
   int rc = check_ragged(in, offsets, out, n_outer, 1, 0, 0, dtype, op);
   if (rc) return rc;
   return ragged_literal(in, offsets, init, out, n_outer, dtype, op, as_stream(stream));
+}
+
+// ---------------------------------------------------------------- LE multi-section (f2)
+static int check_le(const float* in, float* gicov, int64_t N, int64_t L, int layout, int S,
+                    int dist, int map) {
+  if (S < 1 || S > 32) return fail_invalid("S must be one of 1,2,3,4,5,8,10,15,16,32");
+  int rc = check_common(1, dist, map, N, L);
+  if (rc) return rc;
+  if (layout != 0 && layout != 1) return fail_invalid("layout");
+  if (N > 0 && L < 1) return fail_invalid("n_inner must be >= 1 (ave = sum / L)");
+  if (N > 0 && (!in || !gicov)) return fail_invalid("in or gicov is NULL");
+  return CUDANP_OK;
+}
+
+int cudanp_le_gicov(const float* in, float* gicov, float* ave, float* var, float* ep,
+                    int64_t n_outer, int64_t n_inner, float threshold, int layout, int S, int dist,
+                    int map, void* stream) {
+  int rc = check_le(in, gicov, n_outer, n_inner, layout, S, dist, map);
+  if (rc) return rc;
+  // MAP_AUTO: keep the masters' accesses coalesced: point-major
+  // data -> inter-warp (the paper's LE choice); item-major -> intra.
+  const int m = map != CUDANP_MAP_AUTO ? map : (layout ? MAP_INTER : MAP_INTRA);
+  return le_np(in, gicov, ave, var, ep, n_outer, n_inner, threshold, layout, S, dist, m,
+               as_stream(stream));
+}
+
+int cudanp_le_gicov_literal(const float* in, float* gicov, float* ave, float* var, float* ep,
+                            int64_t n_outer, int64_t n_inner, float threshold, int layout,
+                            void* stream) {
+  int rc = check_le(in, gicov, n_outer, n_inner, layout, 1, 0, 0);
+  if (rc) return rc;
+  return le_literal(in, gicov, ave, var, ep, n_outer, n_inner, threshold, layout, as_stream(stream));
 }
 
 // ---------------------------------------------------------------- variants

@@ -40,6 +40,9 @@ _SIGS = {
     "cudanp_batched_loop_scan": [_vp, _vp, _vp, _i64, _i64, _int, _int, _int, _int, _vp],
     "cudanp_ragged_loop_reduce": [_vp, _vp, _vp, _vp, _i64, _int, _int, _int, _int, _int, _vp],
     "cudanp_ragged_loop_reduce_literal": [_vp, _vp, _vp, _vp, _i64, _int, _int, _vp],
+    "cudanp_le_gicov": [_vp, _vp, _vp, _vp, _vp, _i64, _i64, ctypes.c_float, _int, _int, _int,
+                        _int, _vp],
+    "cudanp_le_gicov_literal": [_vp, _vp, _vp, _vp, _vp, _i64, _i64, ctypes.c_float, _int, _vp],
     "cudanp_tmv_variant": [_int, _vp, _i64, _vp, _vp, _i64, _i64, _vp],
     "cudanp_mv_variant": [_int, _vp, _i64, _vp, _vp, _i64, _i64, _vp],
     "cudanp_batched_loop_reduce_variant": [_int, _vp, _vp, _vp, _i64, _i64, _int, _int, _vp],
@@ -197,6 +200,27 @@ def cudanp_ragged_loop_reduce_literal(x, offsets, init=None, out=None, *, op=SUM
                                                     N, _dtype_code(x), op, _stream(stream)),
            "cudanp_ragged_loop_reduce_literal")
     return out
+
+
+def cudanp_le_gicov(x, threshold, gicov=None, *, layout=0, S=8, dist=CYCLIC, map=AUTO,
+                    want_stats=True, literal=False, stream=None):
+    """LE multi-section item (Figs 5-6): returns (gicov, ave, var, ep).
+    x: (N, L) when layout == 0, (L, N) when layout == 1.  gicov entries whose
+    test fails are left as given (default: filled with -1)."""
+    import torch
+    N, L = (x.shape if layout == 0 else x.shape[::-1])
+    if gicov is None:
+        gicov = torch.full((N,), -1.0, dtype=torch.float32, device=x.device)
+    stats = [torch.empty(N, dtype=torch.float32, device=x.device) for _ in range(3)] \
+        if want_stats else [None, None, None]
+    if literal:
+        rc = load().cudanp_le_gicov_literal(_ptr(x), _ptr(gicov), *(_ptr(t) for t in stats), N, L,
+                                            threshold, layout, _stream(stream))
+    else:
+        rc = load().cudanp_le_gicov(_ptr(x), _ptr(gicov), *(_ptr(t) for t in stats), N, L,
+                                    threshold, layout, S, dist, map, _stream(stream))
+    _check(rc, "cudanp_le_gicov")
+    return (gicov, *stats)
 
 
 # ---------------------------------------------------------------- comparison kernels

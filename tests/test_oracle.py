@@ -410,3 +410,38 @@ def test_ragged_lengths_distributions():
     assert u.min() == 0 and u.max() == 128 and abs(u.mean() - 64) < 1
     e = synth.lengths(100000, 64, "exp")
     assert e.min() == 0 and e.max() <= 16 * 64 and abs(e.mean() - 64) < 2
+
+
+# ------------------------------------------------------------------ LE multi-section (f2)
+def test_le_closed_forms(orc):
+    # two-valued items a,b alternating (L even): ave=(a+b)/2, var=L((a-b)/2)^2, ep=0
+    N, L = 5, 150
+    a = np.arange(1, N + 1, dtype=np.float32)[:, None]
+    x = np.where(np.arange(L)[None, :] % 2 == 0, a, 3 * a).astype(np.float32)
+    g, ave, var, ep = orc.le_gicov(x, thr=0.0)
+    assert (ave == 2 * a[:, 0]).all()
+    assert (var == L * a[:, 0] ** 2).all()
+    assert (ep == 0).all()
+    assert (g == np.float32(2 * a[:, 0]) / np.sqrt(np.float32(L * a[:, 0] ** 2))).all()
+    # constant items: var = 0 -> ratio inf > thr -> gicov = ave/0 = inf
+    g, ave, var, ep = orc.le_gicov(np.full((3, 8), 0.25, np.float32), thr=1e30)
+    assert (var == 0).all() and np.isinf(g).all()
+    # a threshold no item passes leaves gicov untouched
+    g, *_ = orc.le_gicov(x, thr=np.float32(1e30), gicov_fill=-7.0)
+    assert (g == -7).all()
+
+
+def test_le_bruteforce_and_layout(orc):
+    x = synth.items(9, 23, "f32_signed")
+    g, ave, var, ep = orc.le_gicov(x, thr=0.0)
+    for n in range(9):
+        s = sum(Fraction(float(v)) for v in x[n])
+        a32 = np.float32(np.float32(float(s)) / np.float32(23))
+        assert ave[n] == a32
+        ts = [Fraction(float(v)) - Fraction(float(a32)) for v in x[n]]
+        assert var[n] == np.float32(float(sum(t * t for t in ts)))
+        assert ep[n] == np.float32(float(sum(ts)))
+    # point-major layout of the transpose is the same computation
+    g2, a2, v2, e2 = orc.le_gicov(np.ascontiguousarray(x.T), thr=0.0, layout=1)
+    assert (a2 == ave).all() and (v2 == var).all() and (e2 == ep).all()
+    assert np.array_equal(g2, g)

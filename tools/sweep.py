@@ -245,10 +245,53 @@ def r1(means=(16, 64, 256)):
             torch.cuda.empty_cache()
 
 
+def f2(L=150):
+    """f2: LE multi-section items (Figs 5-6), N = 2M items x 150 points, both
+    layouts, every map x dist x S including the non-power-of-two inter-warp S
+    of Fig 12 (3, 5, 10, 15)."""
+    N = 1 << 21
+    for layout in (0, 1):
+        x = gen((N, L) if layout == 0 else (L, N), "f32_unit")
+        g = torch.empty(N, device="cuda")
+        st = [torch.empty(N, device="cuda") for _ in range(3)]
+        nb = 4 * N * L + 4 * N * 4
+        def run(S, d, m):
+            return time_ms(lambda: C.load().cudanp_le_gicov(x.data_ptr(), g.data_ptr(), *(t.data_ptr() for t in st),
+                                                           N, L, 0.02, layout, S, d, m, None))
+        lit = time_ms(lambda: C.load().cudanp_le_gicov_literal(x.data_ptr(), g.data_ptr(), *(t.data_ptr() for t in st),
+                                                               N, L, 0.02, layout, None))[0]
+        res = {}
+        for S in (1, 2, 3, 4, 5, 8, 10, 15, 16, 32):
+            for d in (C.CYCLIC, C.BLOCK):
+                for m in (C.INTRA_WARP, C.INTER_WARP):
+                    if m == C.INTRA_WARP and S & (S - 1):
+                        continue
+                    res[(S, d, m)] = run(S, d, m)
+        s1 = min(v[0] for k, v in res.items() if k[0] == 1)
+        for (S, d, m), (med, mn) in res.items():
+            emit({"config": "F2", "op": "le_gicov", "dtype": "f32", "N": N, "L": L,
+                  "layout": "point-major" if layout else "item-major", "S": S, "dist": DN[d], "map": MN[m],
+                  "impl": "np", "t_median_us": round(med * 1e3, 2), "alg_bytes": nb,
+                  "gbs": round(nb / (med * 1e-3) / 1e9, 1), "speedup_vs_s1_tuned": round(s1 / med, 3),
+                  "speedup_vs_s1_literal": round(lit / med, 3)})
+        best = min(res, key=lambda k: res[k][0])
+        emit({"config": "F2", "op": "le_gicov", "dtype": "f32", "N": N, "L": f"{L}/{'pm' if layout else 'im'}",
+              "impl": "s1_literal", "t_median_us": round(lit * 1e3, 2), "alg_bytes": nb,
+              "gbs": round(nb / (lit * 1e-3) / 1e9, 1)})
+        emit({"config": "F2", "op": "le_gicov", "dtype": "f32", "N": N, "L": f"{L}/{'pm' if layout else 'im'}",
+              "impl": "best_np", "S": best[0], "dist": DN[best[1]], "map": MN[best[2]],
+              "t_median_us": round(res[best][0] * 1e3, 2), "alg_bytes": nb,
+              "gbs": round(nb / (res[best][0] * 1e-3) / 1e9, 1),
+              "speedup_vs_s1_tuned": round(s1 / res[best][0], 3),
+              "speedup_vs_s1_literal": round(lit / res[best][0], 3)})
+        del x, g, st
+        torch.cuda.empty_cache()
+
+
 def main():
     global OUT
     ap = argparse.ArgumentParser()
-    ap.add_argument("--configs", default="C1,C2,C3,C4,C5,R1")
+    ap.add_argument("--configs", default="C1,C2,C3,C4,C5,R1,F2")
     ap.add_argument("--out", default=os.path.join(ROOT, "gpurun_out", "sweep.jsonl"))
     ap.add_argument("--lib", default=None, help="alternative libcudanp.so (build experiments)")
     a = ap.parse_args()
@@ -258,7 +301,7 @@ def main():
     C.cudanp_dp_set_pending_launch_limit(1 << 17)
     t0 = time.time()
     for c in a.configs.split(","):
-        {"C1": c1, "C2": c2, "C3": c3, "C4": c4, "C5": c5, "R1": r1}[c.strip()]()
+        {"C1": c1, "C2": c2, "C3": c3, "C4": c4, "C5": c5, "R1": r1, "F2": f2}[c.strip()]()
         print(f"# {c} done at {time.time() - t0:.0f}s", file=sys.stderr, flush=True)
     print(f"# dp launch errors: {C.cudanp_dp_error_count(reset=True)}", file=sys.stderr)
 
