@@ -165,6 +165,15 @@ int cudanp_dp_set_pending_launch_limit(size_t n);
  * (synchronizes the device); reset = 1 clears the counter. */
 int cudanp_dp_error_count(int reset, int64_t* count_out);
 
+/* Memory-copy microbenchmark of Fig 1: copies
+ * `total` floats in -> out.  variant 0: plain grid-stride copy kernel built
+ * without relocatable device code; 1: the same kernel built with -rdc (the
+ * "dynamic-parallelism-enabled kernel overhead"); 2: dynamic
+ * parallelism -- a parent kernel of m threads, each launching a child grid
+ * of n = total/m threads that copies n floats (m must divide total). */
+int cudanp_dp_memcopy(const float* in, float* out, int64_t total, int64_t m, int variant,
+                      void* stream);
+
 /* ------------------------------------------------------------------------
  * Launch shape actually used (the paper's resource analysis, Table 1 P:96,
  * and autotune space P:384): for an NP call with these arguments,

@@ -29,6 +29,7 @@ int dp_mv(bool, const float*, int64_t, const float*, float*, int64_t, int64_t, c
 int dp_reduce(bool, const void*, const void*, void*, int64_t, int64_t, int, int, cudaStream_t);
 int dp_scan(bool, const void*, const void*, void*, int64_t, int64_t, int, cudaStream_t);
 int dp_error_count(int, int64_t*);
+int dp_memcopy(const float*, float*, int64_t, int64_t, int, cudaStream_t);
 int ragged_np(const void*, const int64_t*, const void*, void*, int64_t, int, int, int, int, int,
               cudaStream_t);
 int ragged_literal(const void*, const int64_t*, const void*, void*, int64_t, int, int, cudaStream_t);
@@ -164,6 +165,15 @@ __global__ void generate_kernel(void* out, int64_t rows, int64_t cols, int64_t l
       default: break;
     }
   }
+}
+
+// ---------------------------------------------------------------- memcopy (Fig 1 baseline)
+// The plain copy kernel, compiled WITHOUT -rdc ("baseline ... without
+// dynamic parallelism").
+__global__ void memcopy_kernel(const float* __restrict__ in, float* __restrict__ out, int64_t total) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < total;
+       i += (int64_t)gridDim.x * blockDim.x)
+    out[i] = in[i];
 }
 
 // ---------------------------------------------------------------- debug kernels
@@ -393,6 +403,19 @@ int cudanp_dp_set_pending_launch_limit(size_t n) {
 }
 
 int cudanp_dp_error_count(int reset, int64_t* count_out) { return dp_error_count(reset, count_out); }
+
+int cudanp_dp_memcopy(const float* in, float* out, int64_t total, int64_t m, int variant,
+                      void* stream) {
+  if (total < 0 || (total > 0 && (!in || !out))) return fail_invalid("memcopy sizes/pointers");
+  if (variant < 0 || variant > 2) return fail_invalid("memcopy variant");
+  if (variant == 2 && (m < 1 || total % m != 0)) return fail_invalid("m must divide total");
+  if (total == 0) return CUDANP_OK;
+  if (variant == 0) {
+    memcopy_kernel<<<(unsigned)(sm_count() * 8), 256, 0, as_stream(stream)>>>(in, out, total);
+    return check_launch("memcopy launch");
+  }
+  return dp_memcopy(in, out, total, m, variant, as_stream(stream));
+}
 
 // ---------------------------------------------------------------- launch info
 int cudanp_launch_info(int op_kind, int64_t n_outer, int64_t n_inner, int dtype, int op, int S,

@@ -190,6 +190,44 @@ __global__ void dp_scan_parent(const T* in, const T* init, T* out, int64_t N, in
   }
 }
 
+// ---------------------------------------------------------------- memcopy microbenchmark (Fig 1)
+// copy m*n floats; the parent kernel has m threads and each launches
+// a child grid of n threads that copies n floats.  memcopy_rdc_kernel is the
+// plain copy compiled inside this -rdc translation unit, i.e. the "dynamic-
+// parallelism-enabled kernel overhead" case; the same kernel without
+// -rdc lives in abi.cu.
+__global__ void memcopy_rdc_kernel(const float* __restrict__ in, float* __restrict__ out,
+                                   int64_t total) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < total;
+       i += (int64_t)gridDim.x * blockDim.x)
+    out[i] = in[i];
+}
+
+__global__ void dp_memcopy_child(const float* __restrict__ in, float* __restrict__ out, int64_t n) {
+  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < n) out[i] = in[i];
+}
+
+__global__ void dp_memcopy_parent(const float* in, float* out, int64_t m, int64_t n) {
+  const int64_t p = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (p >= m) return;
+  const int64_t base = p * n;
+  const unsigned blocks = (unsigned)((n + 255) / 256);
+  dp_memcopy_child<<<blocks, n < 256 ? (unsigned)((n + 31) / 32 * 32) : 256u, 0,
+                     cudaStreamFireAndForget>>>(in + base, out + base, n);
+  note_launch();
+}
+
+int dp_memcopy(const float* in, float* out, int64_t total, int64_t m, int variant, cudaStream_t st) {
+  if (total == 0) return CUDANP_OK;
+  if (variant == 1) {
+    memcopy_rdc_kernel<<<(unsigned)(sm_count() * 8), 256, 0, st>>>(in, out, total);
+  } else {
+    dp_memcopy_parent<<<(unsigned)((m + 127) / 128), 128, 0, st>>>(in, out, m, total / m);
+  }
+  return check_launch("dp_memcopy launch");
+}
+
 // ---------------------------------------------------------------- host side
 constexpr int kParentBlock = 128;
 

@@ -49,6 +49,7 @@ _SIGS = {
     "cudanp_batched_loop_scan_variant": [_int, _vp, _vp, _vp, _i64, _i64, _int, _vp],
     "cudanp_dp_set_pending_launch_limit": [_sz],
     "cudanp_dp_error_count": [_int, ctypes.POINTER(_i64)],
+    "cudanp_dp_memcopy": [_vp, _vp, _i64, _i64, _int, _vp],
     "cudanp_launch_info": [_int, _i64, _i64, _int, _int, _int, _int, _int, _int,
                            ctypes.POINTER(_int), ctypes.POINTER(_i64), ctypes.POINTER(_int),
                            ctypes.POINTER(_int), ctypes.POINTER(_int)],
@@ -276,6 +277,17 @@ def cudanp_dp_error_count(reset: bool = True) -> int:
     c = _i64(0)
     _check(load().cudanp_dp_error_count(int(reset), ctypes.byref(c)), "cudanp_dp_error_count")
     return c.value
+
+
+def cudanp_dp_memcopy(x, out=None, *, m=1, variant=2, stream=None):
+    """Fig 1 memcopy: variant 0 plain, 1 plain built with -rdc, 2 DP
+    with m parent threads each launching a child of numel/m threads."""
+    import torch
+    if out is None:
+        out = torch.empty_like(x)
+    _check(load().cudanp_dp_memcopy(_ptr(x), _ptr(out), x.numel(), m, variant, _stream(stream)),
+           "cudanp_dp_memcopy")
+    return out
 
 
 # ---------------------------------------------------------------- support

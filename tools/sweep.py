@@ -288,10 +288,28 @@ def f2(L=150):
         torch.cuda.empty_cache()
 
 
+def f3(total=1 << 26):
+    """f3: Fig 1 on B200 -- copy 64M floats; plain kernel without and
+    with -rdc, and DP with m parent threads x n = total/m child threads."""
+    x = gen((total,), "f32_unit")
+    out = torch.empty_like(x)
+    nb = 8 * total
+    for variant, name in ((0, "plain"), (1, "plain_rdc")):
+        med, mn = time_ms(lambda: C.cudanp_dp_memcopy(x, out, variant=variant))
+        emit({"config": "F3", "op": "memcopy", "impl": name, "m": 1, "n": total,
+              "t_median_us": round(med * 1e3, 2), "alg_bytes": nb, "gbs": round(nb / (med * 1e-3) / 1e9, 1)})
+    for m in (1, 4, 16, 64, 256, 1024, 4096, 16384, 65536):
+        med, mn = time_ms(lambda: C.cudanp_dp_memcopy(x, out, m=m, variant=2), reps=3, warm=1)
+        emit({"config": "F3", "op": "memcopy", "impl": "dp", "m": m, "n": total // m,
+              "t_median_us": round(med * 1e3, 2), "alg_bytes": nb, "gbs": round(nb / (med * 1e-3) / 1e9, 1)})
+    del x, out
+    torch.cuda.empty_cache()
+
+
 def main():
     global OUT
     ap = argparse.ArgumentParser()
-    ap.add_argument("--configs", default="C1,C2,C3,C4,C5,R1,F2")
+    ap.add_argument("--configs", default="C1,C2,C3,C4,C5,R1,F2,F3")
     ap.add_argument("--out", default=os.path.join(ROOT, "gpurun_out", "sweep.jsonl"))
     ap.add_argument("--lib", default=None, help="alternative libcudanp.so (build experiments)")
     a = ap.parse_args()
@@ -301,7 +319,7 @@ def main():
     C.cudanp_dp_set_pending_launch_limit(1 << 17)
     t0 = time.time()
     for c in a.configs.split(","):
-        {"C1": c1, "C2": c2, "C3": c3, "C4": c4, "C5": c5, "R1": r1, "F2": f2}[c.strip()]()
+        {"C1": c1, "C2": c2, "C3": c3, "C4": c4, "C5": c5, "R1": r1, "F2": f2, "F3": f3}[c.strip()]()
         print(f"# {c} done at {time.time() - t0:.0f}s", file=sys.stderr, flush=True)
     print(f"# dp launch errors: {C.cudanp_dp_error_count(reset=True)}", file=sys.stderr)
 
