@@ -54,6 +54,9 @@ def parse():
     ap.add_argument("--no-sweep", action="store_true",
                     help="skip the autotune sweep and comparisons (for ncu launch lists); "
                          "use --tmv-cfg / --mv-cfg")
+    ap.add_argument("--gather", choices=["nccl", "fused"], default="nccl",
+                    help="N > 1: gather outputs to rank 0 with NCCL send/recv, or fused into the "
+                         "kernels' master stores through CUDA IPC over NVLink (SURVEY f4)")
     ap.add_argument("--tmv-cfg", default="32,block,inter")
     ap.add_argument("--mv-cfg", default="16,cyclic,intra")
     return ap.parse_args()
@@ -247,21 +250,31 @@ def run_cudanp(args):
     y_root = torch.empty(n * world, dtype=torch.float32, device="cuda") if rank == 0 else None
     ym_root = torch.empty(n * world, dtype=torch.float32, device="cuda") if rank == 0 else None
 
+    fused = world > 1 and args.gather == "fused"
+    if fused:
+        fg_t = P.FusedGather(y_root, n * world, rank, world)
+        fg_m = P.FusedGather(ym_root, n * world, rank, world)
+        out_t, out_m = fg_t.out_ptr(), fg_m.out_ptr()
+    else:
+        out_t, out_m = y_t, y_m
+
     def step(evs=None):
         if evs:
             evs[0].record(st)
-        C.cudanp_tmv(A_t, x_t, y_t, S=St, dist=dt, map=mt)
+        C.cudanp_tmv(A_t, x_t, out_t, S=St, dist=dt, map=mt, n_outer=wt)
         if evs:
             evs[1].record(st)
-        C.cudanp_mv(A_m, x_m, y_m, S=Sm, dist=dm, map=mm)
+        C.cudanp_mv(A_m, x_m, out_m, S=Sm, dist=dm, map=mm)
         if evs:
             evs[2].record(st)
-        if world > 1:
+        if world > 1 and not fused:
             P.gather_to_root(y_t, y_root, n * world, rank, world)
             P.gather_to_root(y_m, ym_root, n * world, rank, world)
 
     for _ in range(args.warmup):
         step()
+    if fused:
+        fg_t.finish()
     clocks = ClockSampler(local)
     clocks.start()
     time.sleep(0.3)
@@ -274,7 +287,7 @@ def run_cudanp(args):
         step(per_step[k])
     e1.record(st)
     torch.cuda.synchronize()
-    barrier(world)
+    barrier(world)   # with --gather fused this is also the stores' completion point
     clk = clocks.stop()
     ms = max_over_ranks(e0.elapsed_time(e1) / args.steps, world)
     t_tmv = statistics.mean(ev[0].elapsed_time(ev[1]) for ev in per_step)
@@ -378,7 +391,9 @@ def run_cudanp(args):
                     "map": "intra" if mt == 1 else "inter"},
             "mv": {"S": Sm, "dist": "cyclic" if dm == 0 else "block",
                    "map": "intra" if mm == 1 else "inter"},
-            "parallelism": f"dp{world}: contiguous outer-item shards + NCCL gather to rank 0"
+            "parallelism": (f"dp{world}: contiguous outer-item shards + "
+                            + ("gather fused into the master stores (CUDA IPC over NVLink)"
+                               if fused else "NCCL send/recv gather to rank 0"))
                            if world > 1 else "single GPU",
             "l2": "no flush: each matrix is 1 GiB > 126 MB L2",
             "step": "cudanp_tmv + cudanp_mv (+ gather when n_gpus > 1)",

@@ -193,6 +193,21 @@ int cudanp_launch_info(int op_kind, int64_t n_outer, int64_t n_inner, int dtype,
  * ---------------------------------------------------------------------- */
 int cudanp_shard_range(int64_t n_outer, int nranks, int rank, int64_t* begin, int64_t* end);
 
+/* Fused gather over NVLink: CUDA IPC lets rank g's kernel
+ * epilogue store its outputs straight into rank 0's result buffer, so the
+ * master's store *is* the gather -- pass the opened pointer (plus the
+ * shard's begin) as the `y`/`out` argument of any call above.
+ * cudanp_ipc_get_handle: handle_out receives 64 bytes (cudaIpcMemHandle_t) of
+ *   the allocation holding dev_ptr and *offset_out its byte offset in it.
+ * cudanp_ipc_open: maps a handle from another process of the same node;
+ *   *dev_ptr_out = mapped base + offset.  Peer access is enabled lazily.
+ * cudanp_ipc_close: unmaps (pass the pointer and offset from ipc_open).
+ * The caller orders the writes (stream sync + a barrier) before the owner
+ * reads the buffer. */
+int cudanp_ipc_get_handle(const void* dev_ptr, void* handle_out, int64_t* offset_out);
+int cudanp_ipc_open(const void* handle, int64_t offset, void** dev_ptr_out);
+int cudanp_ipc_close(void* dev_ptr, int64_t offset);
+
 /* ------------------------------------------------------------------------
  * Test and benchmark support (not part of the method).
  * ---------------------------------------------------------------------- */

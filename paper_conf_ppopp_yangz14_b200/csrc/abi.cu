@@ -448,6 +448,64 @@ int cudanp_launch_info(int op_kind, int64_t n_outer, int64_t n_inner, int dtype,
   return CUDANP_OK;
 }
 
+// ---------------------------------------------------------------- CUDA IPC (f4)
+// cuMemGetAddressRange through the runtime's driver entry point, so the
+// library needs no link-time libcuda (it must load on GPU-less build hosts).
+typedef int (*MemGetAddressRangeFn)(unsigned long long*, size_t*, unsigned long long);
+
+static int alloc_base(const void* ptr, char** base) {
+  static MemGetAddressRangeFn fn = nullptr;
+  if (!fn) {
+    void* f = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuMemGetAddressRange", &f, cudaEnableDefault, &q) != cudaSuccess ||
+        !f) {
+      cudaGetLastError();
+      set_error("cuMemGetAddressRange entry point unavailable");
+      return CUDANP_ERR_CUDA;
+    }
+    fn = (MemGetAddressRangeFn)f;
+  }
+  unsigned long long b = 0;
+  size_t sz = 0;
+  if (fn(&b, &sz, (unsigned long long)(uintptr_t)ptr) != 0) {
+    set_error("cuMemGetAddressRange failed (not a device allocation?)");
+    return CUDANP_ERR_CUDA;
+  }
+  *base = (char*)(uintptr_t)b;
+  return CUDANP_OK;
+}
+
+int cudanp_ipc_get_handle(const void* dev_ptr, void* handle_out, int64_t* offset_out) {
+  if (!dev_ptr || !handle_out || !offset_out) return fail_invalid("ipc_get_handle arguments");
+  char* base = nullptr;
+  int rc = alloc_base(dev_ptr, &base);
+  if (rc) return rc;
+  cudaIpcMemHandle_t h;
+  if (cudaIpcGetMemHandle(&h, base) != cudaSuccess) return check_launch("cudaIpcGetMemHandle");
+  memcpy(handle_out, &h, sizeof(h));
+  *offset_out = (int64_t)((const char*)dev_ptr - base);
+  return CUDANP_OK;
+}
+
+int cudanp_ipc_open(const void* handle, int64_t offset, void** dev_ptr_out) {
+  if (!handle || !dev_ptr_out || offset < 0) return fail_invalid("ipc_open arguments");
+  cudaIpcMemHandle_t h;
+  memcpy(&h, handle, sizeof(h));
+  void* base = nullptr;
+  if (cudaIpcOpenMemHandle(&base, h, cudaIpcMemLazyEnablePeerAccess) != cudaSuccess)
+    return check_launch("cudaIpcOpenMemHandle");
+  *dev_ptr_out = (char*)base + offset;
+  return CUDANP_OK;
+}
+
+int cudanp_ipc_close(void* dev_ptr, int64_t offset) {
+  if (!dev_ptr || offset < 0) return fail_invalid("ipc_close arguments");
+  if (cudaIpcCloseMemHandle((char*)dev_ptr - offset) != cudaSuccess)
+    return check_launch("cudaIpcCloseMemHandle");
+  return CUDANP_OK;
+}
+
 // ---------------------------------------------------------------- sharding
 int cudanp_shard_range(int64_t n_outer, int nranks, int rank, int64_t* begin, int64_t* end) {
   if (n_outer < 0 || nranks < 1 || rank < 0 || rank >= nranks || !begin || !end)

@@ -54,6 +54,9 @@ _SIGS = {
                            ctypes.POINTER(_int), ctypes.POINTER(_i64), ctypes.POINTER(_int),
                            ctypes.POINTER(_int), ctypes.POINTER(_int)],
     "cudanp_shard_range": [_i64, _int, _int, ctypes.POINTER(_i64), ctypes.POINTER(_i64)],
+    "cudanp_ipc_get_handle": [_vp, _vp, ctypes.POINTER(_i64)],
+    "cudanp_ipc_open": [_vp, _i64, ctypes.POINTER(_vp)],
+    "cudanp_ipc_close": [_vp, _i64],
     "cudanp_generate": [_vp, _i64, _i64, _i64, _i64, _i64, _i64, _int, _int, _i64, _u64, _vp],
     "cudanp_debug_owner_map": [_i64, _int, _int, _int, _P32],
     "cudanp_debug_team_ids": [_int, _int, _P32, _P32, ctypes.POINTER(_int)],
@@ -110,8 +113,12 @@ def _stream(stream) -> int | None:
 
 
 def _ptr(t) -> int | None:
+    """Device pointer of a CUDA tensor, or a raw device address passed as int
+    (e.g. an IPC-mapped peer buffer, cudanp_ipc_open)."""
     if t is None:
         return None
+    if isinstance(t, int):
+        return t or None
     if not t.is_cuda:
         raise ValueError("tensor must be on a CUDA device (the library takes device pointers)")
     return t.data_ptr() or None
@@ -300,6 +307,24 @@ def cudanp_launch_info(op_kind: str, n_outer: int, n_inner: int, *, dtype=F32, o
                                      ctypes.byref(s), ctypes.byref(m)), "cudanp_launch_info")
     return {"block_threads": b.value, "grid_ctas": g.value, "regs_per_thread": r.value,
             "smem_bytes": s.value, "map": {1: "intra_warp", 2: "inter_warp"}.get(m.value, "?")}
+
+
+def cudanp_ipc_get_handle(t) -> tuple[bytes, int]:
+    """(64-byte IPC handle of t's allocation, byte offset of t in it)."""
+    buf = ctypes.create_string_buffer(64)
+    off = _i64()
+    _check(load().cudanp_ipc_get_handle(_ptr(t), buf, ctypes.byref(off)), "cudanp_ipc_get_handle")
+    return buf.raw, off.value
+
+
+def cudanp_ipc_open(handle: bytes, offset: int) -> int:
+    p = _vp()
+    _check(load().cudanp_ipc_open(handle, offset, ctypes.byref(p)), "cudanp_ipc_open")
+    return p.value
+
+
+def cudanp_ipc_close(ptr: int, offset: int) -> None:
+    _check(load().cudanp_ipc_close(ptr, offset), "cudanp_ipc_close")
 
 
 def cudanp_shard_range(n_outer: int, nranks: int, rank: int) -> tuple[int, int]:

@@ -41,3 +41,47 @@ def gather_to_root(local, root_buf, n_total: int, rank: int, world: int, root: i
         for r in dist.batch_isend_irecv(ops):
             r.wait()
     return root_buf if rank == root else None
+
+
+class FusedGather:
+    """Gather fused into the kernels' master stores.
+
+    Rank 0 exports its result buffer through CUDA IPC; every other rank maps
+    it once, and then passes ``out_ptr()`` -- rank 0's buffer at the start of
+    its own shard -- as the output pointer of a cudanp call, so each master
+    thread's store lands in rank 0's HBM over NVLink with no separate
+    collective.  ``finish()`` orders the stores before rank 0 reads:
+    stream synchronize + a process-group barrier.
+    """
+
+    def __init__(self, root_buf, n_total: int, rank: int, world: int, elem_bytes: int = 4,
+                 root: int = 0):
+        import torch.distributed as dist
+        self.rank, self.world, self.root = rank, world, root
+        self.begin, self.end = shard(n_total, world, rank)
+        obj = [None]
+        if rank == root:
+            obj = [C.cudanp_ipc_get_handle(root_buf)]
+            self.base = root_buf.data_ptr()
+        dist.broadcast_object_list(obj, src=root)
+        self.handle, self.offset = obj[0]
+        if rank != root:
+            self.mapped = C.cudanp_ipc_open(self.handle, self.offset)
+            self.base = self.mapped
+        else:
+            self.mapped = None
+        self.elem_bytes = elem_bytes
+
+    def out_ptr(self) -> int:
+        return self.base + self.begin * self.elem_bytes
+
+    def finish(self):
+        import torch
+        import torch.distributed as dist
+        torch.cuda.current_stream().synchronize()
+        dist.barrier()
+
+    def close(self):
+        if self.mapped is not None:
+            C.cudanp_ipc_close(self.mapped, self.offset)
+            self.mapped = None
