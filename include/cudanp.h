@@ -85,6 +85,19 @@ int cudanp_batched_loop_reduce(const void* in, const void* init, void* out,
                                int64_t n_outer, int64_t n_inner, int dtype, int op,
                                int S, int dist, int map, void* stream);
 
+/* Team-reduction backend ablation (Fig 16: shfl vs shared
+ * memory for the reduction under intra-warp NP; plus sm_100a redux.sync):
+ * the batched loop-reduce with the intra-warp map and cyclic distribution,
+ * combining the team's partials with backend 0 = shfl-xor butterfly (what
+ * cudanp_batched_loop_reduce uses), 1 = shared memory (each lane writes a
+ * slot, the master folds its team's S slots), 2 = redux.sync over the team's
+ * lane mask (int32 add/max, fp32 max; fp32 sum -> CUDANP_ERR_UNSUPPORTED).
+ * Built for the 128-bit path only: L % 4 == 0 and `in` 16-byte aligned, else
+ * CUDANP_ERR_UNSUPPORTED. */
+int cudanp_batched_loop_reduce_backend(const void* in, const void* init, void* out,
+                                       int64_t n_outer, int64_t n_inner, int dtype, int op,
+                                       int S, int backend, void* stream);
+
 /* Batched inclusive scan (scan clause; inclusive per R1):
  * out[n*L + k] = init[n] + sum_{i<=k} in[n*L + i].  init may be NULL (0);
  * when given, the master loads it and broadcasts it to its slaves with

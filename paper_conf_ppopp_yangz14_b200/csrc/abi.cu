@@ -15,6 +15,8 @@ namespace cudanp {
 int reduce_np(const void*, const void*, void*, int64_t, int64_t, int, int, int, int, int, bool,
               cudaStream_t, LaunchInfo*);
 int reduce_literal(const void*, const void*, void*, int64_t, int64_t, int, int, cudaStream_t);
+int reduce_backend(const void*, const void*, void*, int64_t, int64_t, int, int, int, int,
+                   cudaStream_t);
 int scan_np(const void*, const void*, void*, int64_t, int64_t, int, int, int, int, bool,
             cudaStream_t, LaunchInfo*);
 int scan_literal(const void*, const void*, void*, int64_t, int64_t, int, cudaStream_t);
@@ -276,6 +278,19 @@ int cudanp_batched_loop_reduce(const void* in, const void* init, void* out, int6
   const bool vec = (n_inner % 4 == 0) && aligned16(in);
   return reduce_np(in, init, out, n_outer, n_inner, dtype, op, S, dist, resolve_map(map, false),
                    vec, as_stream(stream), nullptr);
+}
+
+int cudanp_batched_loop_reduce_backend(const void* in, const void* init, void* out,
+                                       int64_t n_outer, int64_t n_inner, int dtype, int op, int S,
+                                       int backend, void* stream) {
+  int rc = check_batched(in, out, n_outer, n_inner, S, 0, CUDANP_MAP_INTRA_WARP, dtype, op, true);
+  if (rc) return rc;
+  if (backend < 0 || backend > 2) return fail_invalid("backend");
+  if (!((n_inner % 4 == 0) && aligned16(in))) {
+    set_error("backend ablation is built for the 128-bit path only (L %% 4 == 0, 16-byte aligned)");
+    return CUDANP_ERR_UNSUPPORTED;
+  }
+  return reduce_backend(in, init, out, n_outer, n_inner, dtype, op, S, backend, as_stream(stream));
 }
 
 int cudanp_batched_loop_scan(const void* in, const void* init, void* out, int64_t n_outer,

@@ -15,6 +15,8 @@
 #include "common.cuh"
 #include "np_team.cuh"
 
+#include <type_traits>
+
 namespace cudanp {
 
 constexpr int kReduceBlock = 256;  // intra-warp CTA: 8 warps
@@ -29,14 +31,25 @@ __device__ __forceinline__ V4<T> op4(V4<T> a, V4<T> b) {
   return {Op::apply(a.x, b.x), Op::apply(a.y, b.y), Op::apply(a.z, b.z), Op::apply(a.w, b.w)};
 }
 
+// Team-reduction backend (the Fig 16 ablation): 0 = shfl
+// butterfly (default), 1 = shared memory, 2 = redux.sync.
+enum { RB_SHFL = 0, RB_SMEM = 1, RB_REDUX = 2 };
+
+template <class T, class Op>
+__device__ __forceinline__ T redux_op(T v, unsigned mask) {
+  if constexpr (std::is_same<Op, OpSum>::value) return Redux::sum(v, mask);
+  else return Redux::max(v, mask);
+}
+
 // ---------------------------------------------------------------- intra-warp
 // Team = S lanes; a warp holds TPW = 32/S teams = TPW items ("warp tile").
 // Each warp processes K consecutive warp tiles per step of a grid-stride
 // loop, so a lane has K independent rows in flight.
-template <class T, class Op, int S, int DIST, bool VEC>
+template <class T, class Op, int S, int DIST, bool VEC, int RB = RB_SHFL>
 __global__ void __launch_bounds__(kReduceBlock)
 reduce_intra_kernel(const T* __restrict__ in, const T* __restrict__ init, T* __restrict__ out,
                     int64_t N, int64_t L) {
+  __shared__ T slots[RB == RB_SMEM ? kReduceBlock : 1];
   constexpr int TPW = 32 / S;
   constexpr int K = kReduceK;
   const IntraTeam<S> team;
@@ -95,7 +108,10 @@ reduce_intra_kernel(const T* __restrict__ in, const T* __restrict__ init, T* __r
     // epilogue: combine with init[n] and store.
 #pragma unroll
     for (int k = 0; k < K; ++k) {
-      const T res = team.template reduce<Op>(part[k]);
+      T res;
+      if constexpr (RB == RB_SMEM) res = team.template reduce_smem<Op>(part[k], slots + (threadIdx.x & ~31));
+      else if constexpr (RB == RB_REDUX) res = redux_op<T, Op>(part[k], team.segment_mask());
+      else res = team.template reduce<Op>(part[k]);
       if (team.is_master() && item[k] < N)
         out[item[k]] = init ? Op::apply(init[item[k]], res) : res;
     }
@@ -224,6 +240,45 @@ int reduce_np(const void* in, const void* init, void* out, int64_t N, int64_t L,
   return op == CUDANP_SUM
              ? dispatch_reduce_t<int32_t, OpSum>(in, init, out, N, L, S, dist, map, vec, st, info)
              : dispatch_reduce_t<int32_t, OpMax>(in, init, out, N, L, S, dist, map, vec, st, info);
+}
+
+// Fig 16 ablation entry: intra-warp, cyclic, 128-bit path, chosen backend.
+template <class T, class Op, int RB>
+static int launch_reduce_backend(const void* in, const void* init, void* out, int64_t N, int64_t L,
+                                 int S, cudaStream_t st) {
+  CUDANP_DISPATCH_S(S, {
+    auto kern = reduce_intra_kernel<T, Op, kS, DIST_CYCLIC, true, RB>;
+    constexpr int TPW = 32 / kS;
+    const int64_t ntiles = (N + TPW - 1) / TPW;
+    const int64_t per_cta = (kReduceBlock / 32) * kReduceK;
+    const int64_t grid = persistent_grid(kern, kReduceBlock, 0, (ntiles + per_cta - 1) / per_cta);
+    if (N == 0) return CUDANP_OK;
+    kern<<<(unsigned)grid, kReduceBlock, 0, st>>>((const T*)in, (const T*)init, (T*)out, N, L);
+    return check_launch("batched_loop_reduce_backend launch");
+  });
+  return CUDANP_OK;
+}
+
+template <class T, class Op>
+static int reduce_backend_t(const void* in, const void* init, void* out, int64_t N, int64_t L, int S,
+                            int backend, cudaStream_t st) {
+  if (backend == RB_SHFL) return launch_reduce_backend<T, Op, RB_SHFL>(in, init, out, N, L, S, st);
+  if (backend == RB_SMEM) return launch_reduce_backend<T, Op, RB_SMEM>(in, init, out, N, L, S, st);
+  if constexpr (std::is_same<T, float>::value && std::is_same<Op, OpSum>::value) {
+    set_error("redux.sync has no fp32 add (fp32 min/max and int32 add/max only)");
+    return CUDANP_ERR_UNSUPPORTED;
+  } else {
+    return launch_reduce_backend<T, Op, RB_REDUX>(in, init, out, N, L, S, st);
+  }
+}
+
+int reduce_backend(const void* in, const void* init, void* out, int64_t N, int64_t L, int dtype,
+                   int op, int S, int backend, cudaStream_t st) {
+  if (dtype == CUDANP_F32)
+    return op == CUDANP_SUM ? reduce_backend_t<float, OpSum>(in, init, out, N, L, S, backend, st)
+                            : reduce_backend_t<float, OpMax>(in, init, out, N, L, S, backend, st);
+  return op == CUDANP_SUM ? reduce_backend_t<int32_t, OpSum>(in, init, out, N, L, S, backend, st)
+                          : reduce_backend_t<int32_t, OpMax>(in, init, out, N, L, S, backend, st);
 }
 
 int reduce_literal(const void* in, const void* init, void* out, int64_t N, int64_t L, int dtype,

@@ -145,6 +145,26 @@ struct IntraTeam {
     for (int o = S / 2; o > 0; o >>= 1) v = Op::apply(v, __shfl_xor_sync(kFull, v, o, S));
     return v;
   }
+  // The same reduction through shared memory ("using shared memory";
+  // the Fig 16 comparison): every lane writes its partial to the
+  // warp's 32 slots and the master folds its team's S slots in slave order.
+  // Only the master's return value is meaningful.
+  template <class Op, class T>
+  __device__ __forceinline__ T reduce_smem(T v, T* slots /*[32] per warp*/) const {
+    slots[lane] = v;
+    __syncwarp();
+    T r = v;
+    if (slave == 0) {
+#pragma unroll
+      for (int k = 1; k < S; ++k) r = Op::apply(r, slots[lane + k]);
+    }
+    __syncwarp();
+    return r;
+  }
+  // Team mask for the width-S segment of this lane.
+  __device__ __forceinline__ unsigned segment_mask() const {
+    return S == 32 ? kFull : (((1u << S) - 1u) << (team * S));
+  }
   // Inclusive scan over the team ("similar approach to the CUDA SDK"):
   // Hillis-Steele with shfl_up inside each width-S segment.
   template <class T>
@@ -162,6 +182,23 @@ struct IntraTeam {
     if (S == 1) return T(0);
     T t = __shfl_up_sync(kFull, incl, 1, S);
     return slave == 0 ? T(0) : t;
+  }
+};
+
+// ---------------------------------------------------------------- redux.sync
+// Hardware warp reductions (sm_80+ integer, sm_100a fp32 min/max) over a
+// lane mask; segments of a width-S team each pass their own mask.
+struct Redux {
+  __device__ __forceinline__ static int32_t sum(int32_t v, unsigned mask) {
+    return (int32_t)__reduce_add_sync(mask, (unsigned)v);
+  }
+  __device__ __forceinline__ static int32_t max(int32_t v, unsigned mask) {
+    return __reduce_max_sync(mask, v);
+  }
+  __device__ __forceinline__ static float max(float v, unsigned mask) {
+    float r;
+    asm volatile("redux.sync.max.f32 %0, %1, %2;" : "=f"(r) : "f"(v), "r"(mask));
+    return r;
   }
 };
 

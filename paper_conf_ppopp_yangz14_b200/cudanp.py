@@ -38,6 +38,7 @@ _SIGS = {
     "cudanp_mv": [_vp, _i64, _vp, _vp, _i64, _i64, _int, _int, _int, _vp],
     "cudanp_batched_loop_reduce": [_vp, _vp, _vp, _i64, _i64, _int, _int, _int, _int, _int, _vp],
     "cudanp_batched_loop_scan": [_vp, _vp, _vp, _i64, _i64, _int, _int, _int, _int, _vp],
+    "cudanp_batched_loop_reduce_backend": [_vp, _vp, _vp, _i64, _i64, _int, _int, _int, _int, _vp],
     "cudanp_ragged_loop_reduce": [_vp, _vp, _vp, _vp, _i64, _int, _int, _int, _int, _int, _vp],
     "cudanp_ragged_loop_reduce_literal": [_vp, _vp, _vp, _vp, _i64, _int, _int, _vp],
     "cudanp_le_gicov": [_vp, _vp, _vp, _vp, _vp, _i64, _i64, ctypes.c_float, _int, _int, _int,
@@ -168,6 +169,24 @@ def cudanp_batched_loop_reduce(x, init=None, out=None, *, op=SUM, S=8, dist=CYCL
     _check(load().cudanp_batched_loop_reduce(_ptr(x), _ptr(init), _ptr(out), N, L, _dtype_code(x),
                                              op, S, dist, map, _stream(stream)),
            "cudanp_batched_loop_reduce")
+    return out
+
+
+SHFL, SMEM, REDUX = 0, 1, 2
+
+
+def cudanp_batched_loop_reduce_backend(x, init=None, out=None, *, op=SUM, S=8, backend=SHFL,
+                                       stream=None):
+    """Fig 16 ablation: intra-warp cyclic reduce with the team reduction done by
+    shfl (0), shared memory (1) or redux.sync (2)."""
+    import torch
+    N, L = x.shape
+    if out is None:
+        out = torch.empty(N, dtype=x.dtype, device=x.device)
+    _check(load().cudanp_batched_loop_reduce_backend(_ptr(x), _ptr(init), _ptr(out), N, L,
+                                                     _dtype_code(x), op, S, backend,
+                                                     _stream(stream)),
+           "cudanp_batched_loop_reduce_backend")
     return out
 
 

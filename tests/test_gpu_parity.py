@@ -420,3 +420,26 @@ def test_full_size_C4_scan_sampled():
         assert_exact(got, ref, f"C4 scan S={S} dist={dist}")
     del x, out
     torch.cuda.empty_cache()
+
+
+# ------------------------------------------------------------------ Fig 16 ablation backends
+@pytest.mark.parametrize("backend", [C.SHFL, C.SMEM, C.REDUX])
+def test_reduce_backend_parity(backend):
+    for N, L in [(1, 4), (70, 12), (300, 32), (97, 256), (1100, 64)]:
+        for dtype, op, kind, exact in [(C.I32, C.SUM, "i32_full", True), (C.I32, C.MAX, "i32_full", True),
+                                       (C.F32, C.MAX, "f32_signed", True), (C.F32, C.SUM, "f32_unit", False)]:
+            x = synth.items(N, L, kind)
+            ini = synth.init(N, kind)
+            ref = O.reduce(x, op=op, init=ini)
+            for S in SS:
+                what = f"backend={backend} {kind} op={op} N={N} L={L} S={S}"
+                if backend == C.REDUX and dtype == C.F32 and op == C.SUM:
+                    with pytest.raises(C.CudanpError) as ei:
+                        C.cudanp_batched_loop_reduce_backend(dev(x), dev(ini), op=op, S=S, backend=backend)
+                    assert ei.value.status == C.ERR_UNSUPPORTED
+                    continue
+                got = host(C.cudanp_batched_loop_reduce_backend(dev(x), dev(ini), op=op, S=S, backend=backend))
+                if exact:
+                    assert_exact(got, ref, what)
+                else:
+                    assert_rel(got, ref, L, what)

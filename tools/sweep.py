@@ -306,10 +306,31 @@ def f3(total=1 << 26):
     torch.cuda.empty_cache()
 
 
+def e9(Ls=(32, 64, 128)):
+    """Fig 16 analog: team reduction by shfl vs shared memory vs
+    redux.sync under intra-warp NP (cyclic), C3 shapes."""
+    N = 1 << 22
+    for L in Ls:
+        for dtype, op, kind, tdt in ((C.I32, C.SUM, "i32_small", torch.int32),
+                                     (C.F32, C.MAX, "f32_signed", torch.float32)):
+            x = gen((N, L), kind, tdt)
+            out = torch.empty(N, dtype=tdt, device="cuda")
+            nb = 4 * N * L + 4 * N
+            for S in C.SLAVE_SIZES:
+                for be, name in ((C.SHFL, "shfl"), (C.SMEM, "smem"), (C.REDUX, "redux")):
+                    med, mn = time_ms(lambda: C.cudanp_batched_loop_reduce_backend(x, None, out, op=op, S=S, backend=be))
+                    emit({"config": "E9", "op": "reduce", "dtype": "f32" if dtype == C.F32 else "i32",
+                          "opname": "sum" if op == C.SUM else "max", "N": N, "L": L, "S": S,
+                          "backend": name, "impl": "np", "t_median_us": round(med * 1e3, 2),
+                          "alg_bytes": nb, "gbs": round(nb / (med * 1e-3) / 1e9, 1)})
+            del x, out
+            torch.cuda.empty_cache()
+
+
 def main():
     global OUT
     ap = argparse.ArgumentParser()
-    ap.add_argument("--configs", default="C1,C2,C3,C4,C5,R1,F2,F3")
+    ap.add_argument("--configs", default="C1,C2,C3,C4,C5,R1,F2,F3,E9")
     ap.add_argument("--out", default=os.path.join(ROOT, "gpurun_out", "sweep.jsonl"))
     ap.add_argument("--lib", default=None, help="alternative libcudanp.so (build experiments)")
     a = ap.parse_args()
@@ -319,7 +340,7 @@ def main():
     C.cudanp_dp_set_pending_launch_limit(1 << 17)
     t0 = time.time()
     for c in a.configs.split(","):
-        {"C1": c1, "C2": c2, "C3": c3, "C4": c4, "C5": c5, "R1": r1, "F2": f2, "F3": f3}[c.strip()]()
+        {"C1": c1, "C2": c2, "C3": c3, "C4": c4, "C5": c5, "R1": r1, "F2": f2, "F3": f3, "E9": e9}[c.strip()]()
         print(f"# {c} done at {time.time() - t0:.0f}s", file=sys.stderr, flush=True)
     print(f"# dp launch errors: {C.cudanp_dp_error_count(reset=True)}", file=sys.stderr)
 
