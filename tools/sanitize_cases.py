@@ -1,0 +1,72 @@
+#!/usr/bin/env python
+"""Small launches of every kernel family for compute-sanitizer
+(memcheck / racecheck / synccheck):
+
+    compute-sanitizer --tool racecheck python tools/sanitize_cases.py
+
+Shapes are tiny but ragged (several teams, partial warps/CTAs, tails), and
+cover both maps, both distributions, every S, the smem broadcast / reduce /
+scan barriers of the inter-warp teams and every masked shuffle.
+"""
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+
+import synth  # noqa: E402
+from paper_conf_ppopp_yangz14_b200 import cudanp as C  # noqa: E402
+
+
+def dev(a):
+    return torch.from_numpy(np.ascontiguousarray(a)).cuda()
+
+
+def main():
+    C.load()
+    quick = "--quick" in sys.argv
+    Ss = (1, 8, 32) if quick else C.SLAVE_SIZES
+    A = dev(synth.matrix(37, 70, "f32_unit"))
+    A4 = dev(synth.matrix(37, 68, "f32_unit"))
+    xt, xm, xm4 = dev(synth.vector(37)), dev(synth.vector(70)), dev(synth.vector(68))
+    Xf = dev(synth.items(70, 36, "f32_unit"))
+    Xi = dev(synth.items(70, 37, "i32_small"))
+    Xi4 = dev(synth.items(70, 36, "i32_small"))
+    inif, inii = dev(synth.init(70, "f32_unit")), dev(synth.init(70, "i32_small"))
+    lens = synth.lengths(50, 9)
+    off = dev(synth.offsets_from_lengths(lens))
+    xr = dev(synth.gen(1, "f32_unit", 0, int(lens.sum()) + 3))
+    le = dev(synth.items(40, 30, "f32_unit"))
+    for S in Ss:
+        for d in (C.CYCLIC, C.BLOCK):
+            for m in (C.INTRA_WARP, C.INTER_WARP):
+                C.cudanp_tmv(A, xt, S=S, dist=d, map=m, n_outer=70)
+                C.cudanp_tmv(A4, xt, S=S, dist=d, map=m)
+                C.cudanp_mv(A, xm, S=S, dist=d, map=m)
+                C.cudanp_mv(A4, xm4, S=S, dist=d, map=m)
+                for X, ini in ((Xf, inif), (Xi, inii)):
+                    C.cudanp_batched_loop_reduce(X, ini, op=C.SUM, S=S, dist=d, map=m)
+                    C.cudanp_batched_loop_reduce(X, None, op=C.MAX, S=S, dist=d, map=m)
+                    C.cudanp_batched_loop_scan(X, ini, S=S, dist=d, map=m)
+                C.cudanp_ragged_loop_reduce(xr, off, S=S, dist=d, map=m)
+                C.cudanp_le_gicov(le, 0.01, S=S, dist=d, map=m)
+        for be in (C.SHFL, C.SMEM, C.REDUX):
+            C.cudanp_batched_loop_reduce_backend(Xi4, inii, S=S, backend=be)
+    for S in (3, 5, 10, 15):
+        C.cudanp_le_gicov(le, 0.01, S=S, map=C.INTER_WARP, layout=0)
+    if not quick:
+        C.cudanp_dp_set_pending_launch_limit(1 << 12)
+        for impl in (C.S1_LITERAL, C.DP_THREAD, C.DP_BLOCK):
+            C.cudanp_tmv_variant(impl, A, xt, n_outer=70)
+            C.cudanp_mv_variant(impl, A, xm)
+            C.cudanp_batched_loop_reduce_variant(impl, Xi, inii)
+            C.cudanp_batched_loop_scan_variant(impl, Xf, inif)
+    torch.cuda.synchronize()
+    print("sanitize cases done")
+
+
+if __name__ == "__main__":
+    main()
