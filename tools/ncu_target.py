@@ -19,7 +19,10 @@ from paper_conf_ppopp_yangz14_b200 import cudanp as C  # noqa: E402
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--op", required=True, choices=["tmv", "mv", "reduce", "scan", "tmv_literal",
-                                                    "mv_literal", "reduce_literal", "scan_literal"])
+                                                    "mv_literal", "reduce_literal", "scan_literal",
+                                                    "ragged", "le"])
+    ap.add_argument("--lens", default="uniform", help="ragged: length distribution")
+    ap.add_argument("--layout", type=int, default=0, help="le: 0 item-major, 1 point-major")
     ap.add_argument("--S", type=int, default=8)
     ap.add_argument("--dist", default="cyclic")
     ap.add_argument("--map", default="auto")
@@ -32,7 +35,18 @@ def main():
     d = {"cyclic": C.CYCLIC, "block": C.BLOCK}[a.dist]
     m = {"auto": C.AUTO, "intra": C.INTRA_WARP, "inter": C.INTER_WARP}[a.map]
     C.load()
-    if a.op.startswith(("tmv", "mv")):
+    if a.op == "ragged":
+        import synth
+        off = torch.from_numpy(synth.offsets_from_lengths(synth.lengths(a.N, a.L, a.lens))).cuda()
+        X = torch.empty(int(off[-1].item()), device="cuda")
+        C.cudanp_generate(X, "f32_unit")
+        o1 = torch.empty(a.N, device="cuda")
+        fns = {"ragged": lambda: C.cudanp_ragged_loop_reduce(X, off, None, o1, S=a.S, dist=d, map=m)}
+    elif a.op == "le":
+        X = torch.empty(*((a.N, a.L) if a.layout == 0 else (a.L, a.N)), device="cuda")
+        C.cudanp_generate(X, "f32_unit")
+        fns = {"le": lambda: C.cudanp_le_gicov(X, 0.02, layout=a.layout, S=a.S, dist=d, map=m)}
+    elif a.op.startswith(("tmv", "mv")):
         A = torch.empty(a.n, a.n, device="cuda")
         C.cudanp_generate(A, "f32_unit")
         x = torch.empty(a.n, device="cuda")

@@ -28,6 +28,7 @@ def dev(a):
 def main():
     C.load()
     quick = "--quick" in sys.argv
+    no_dp = "--no-dp" in sys.argv  # racecheck/synccheck do not support dynamic parallelism
     Ss = (1, 8, 32) if quick else C.SLAVE_SIZES
     A = dev(synth.matrix(37, 70, "f32_unit"))
     A4 = dev(synth.matrix(37, 68, "f32_unit"))
@@ -59,7 +60,7 @@ def main():
         C.cudanp_le_gicov(le, 0.01, S=S, map=C.INTER_WARP, layout=0)
     if not quick:
         C.cudanp_dp_set_pending_launch_limit(1 << 12)
-        for impl in (C.S1_LITERAL, C.DP_THREAD, C.DP_BLOCK):
+        for impl in (C.S1_LITERAL,) if no_dp else (C.S1_LITERAL, C.DP_THREAD, C.DP_BLOCK):
             C.cudanp_tmv_variant(impl, A, xt, n_outer=70)
             C.cudanp_mv_variant(impl, A, xm)
             C.cudanp_batched_loop_reduce_variant(impl, Xi, inii)
