@@ -34,23 +34,30 @@ __device__ __forceinline__ V4<T> op4r(V4<T> a, V4<T> b) {
   return {Op::apply(a.x, b.x), Op::apply(a.y, b.y), Op::apply(a.z, b.z), Op::apply(a.w, b.w)};
 }
 
-// Split [b, e) into head [b, hb), aligned body units [hb, hb + 4*nu), tail.
-template <class T>
-__device__ __forceinline__ void split_segment(const T* in, int64_t b, int64_t e, int64_t& hb,
-                                              int64_t& nu) {
-  const int mis = (int)(((uintptr_t)(in + b) >> 2) & 3);  // 4-byte elements past a 16-byte line
-  int64_t head = (4 - mis) & 3;
-  if (head > e - b) head = e - b;
-  hb = b + head;
-  nu = (e - hb) >> 2;
-}
-
-// Trip count of slave `s` over n units for the distribution.
-template <int S, int DIST>
-__device__ __forceinline__ int64_t trips_of(const Range<S, DIST>& r) {
-  if (r.end <= r.begin) return 0;
-  return DIST == DIST_CYCLIC ? (r.end - r.begin + S - 1) / S : r.end - r.begin;
-}
+// One slave's view of a segment [b, b+len): head (< 4 scalars up to the next
+// 16-byte boundary), aligned body of nu 128-bit units dealt over the team by
+// the distribution, tail (< 4 scalars).  All index math is done once per item
+// and the body walks a pointer; per-element 64-bit arithmetic made the first
+// version instruction-bound (ncu: 4 B per warp instruction).
+template <class T, int S, int DIST>
+struct SegShare {
+  const T* body;      // this slave's first body unit
+  int64_t step;       // elements between its consecutive units
+  int cnt;            // body units it owns
+  int head, tail;     // segment head/tail lengths
+  __device__ __forceinline__ SegShare(const T* in, int64_t b, int64_t len, int slave) {
+    const int mis = (int)(((uintptr_t)(in + b) >> 2) & 3);  // elements past a 16-byte line
+    int64_t h = (4 - mis) & 3;
+    if (h > len) h = len;
+    const int64_t nu = (len - h) >> 2;
+    head = (int)h;
+    tail = (int)(len - h - 4 * nu);
+    const Range<S, DIST> r(nu, 4 * nu, 4, slave);
+    cnt = r.end > r.begin ? (int)((r.end - r.begin + r.step - 1) / r.step) : 0;
+    body = in + b + h + 4 * r.begin;
+    step = 4 * r.step;
+  }
+};
 
 // ---------------------------------------------------------------- intra-warp
 template <class T, class Op, int S, int DIST>
@@ -66,52 +73,56 @@ ragged_intra_kernel(const T* __restrict__ in, const int64_t* __restrict__ off,
   const T id = Op::template identity<T>();
 
   for (int64_t t0 = warp * K; t0 < ntiles; t0 += nwarps * K) {
-    int64_t item[K], hb[K], nu[K], e[K], rb[K], re[K], rs[K];
+    int64_t item[K];
+    const T* p[K];
+    int64_t pstep[K];
+    int cnt[K];
     T part[K];
-    int64_t trips = 0;
+    int trips = 0;
 #pragma unroll
     for (int k = 0; k < K; ++k) {
       item[k] = (t0 + k) * TPW + team.team;
       // Sequential section (master only): read the loop bounds ...
-      int64_t b0 = 0, e0 = 0;
+      int64_t b0 = 0, l0 = 0;
       if (team.is_master() && item[k] < N) {
         b0 = off[item[k]];
-        e0 = off[item[k] + 1];
-        if (e0 < b0) e0 = b0;  // a decreasing offset pair is an empty loop
+        l0 = off[item[k] + 1] - b0;
+        if (l0 < 0) l0 = 0;  // a decreasing offset pair is an empty loop
       }
       // ... and broadcast them to the slaves.
       const int64_t b = team.read_from_master(b0);
-      e[k] = team.read_from_master(e0);
-      split_segment(in, b, e[k], hb[k], nu[k]);
-      const Range<S, DIST> r(nu[k], 4 * nu[k], 4, team.slave);
-      rb[k] = r.begin; re[k] = r.end; rs[k] = r.step;
-      trips = max(trips, trips_of(r));
-      // head elements (<= 3), dealt cyclically
+      const int64_t len = team.read_from_master(l0);
+      const SegShare<T, S, DIST> sh(in, b, len, team.slave);
+      p[k] = sh.body;
+      pstep[k] = sh.step;
+      cnt[k] = sh.cnt;
+      trips = max(trips, sh.cnt);
+      // head and tail scalars (< 4 each), dealt over the first slaves
       part[k] = id;
-      for (int64_t i = b + team.slave; i < hb[k]; i += S) part[k] = Op::apply(part[k], in[i]);
+      for (int i = team.slave; i < sh.head; i += S) part[k] = Op::apply(part[k], in[b + i]);
+      const T* tl = in + b + sh.head + 4 * ((len - sh.head) >> 2);
+      for (int i = team.slave; i < sh.tail; i += S) part[k] = Op::apply(part[k], tl[i]);
     }
-    trips = __reduce_max_sync(kFull, (unsigned)trips);  // warp-uniform trip count
+    trips = (int)__reduce_max_sync(kFull, (unsigned)trips);  // warp-uniform trip count
     V4<T> acc[K];
 #pragma unroll
     for (int k = 0; k < K; ++k) acc[k] = {id, id, id, id};
 #pragma unroll kRaggedUnroll
-    for (int64_t j = 0; j < trips; ++j) {
+    for (int j = 0; j < trips; ++j) {
       V4<T> v[K];
 #pragma unroll
       for (int k = 0; k < K; ++k) {
-        const int64_t u = rb[k] + j * rs[k];
-        if (u < re[k]) v[k] = ldg4(in + hb[k] + 4 * u);
+        if (j < cnt[k]) v[k] = ldg4(p[k]);
         else v[k] = {id, id, id, id};
+        p[k] += pstep[k];
       }
 #pragma unroll
       for (int k = 0; k < K; ++k) acc[k] = op4r<T, Op>(acc[k], v[k]);
     }
 #pragma unroll
     for (int k = 0; k < K; ++k) {
-      const int64_t tb = hb[k] + 4 * nu[k];
-      T p = Op::apply(part[k], Op::apply(Op::apply(acc[k].x, acc[k].y), Op::apply(acc[k].z, acc[k].w)));
-      for (int64_t i = tb + team.slave; i < e[k]; i += S) p = Op::apply(p, in[i]);  // tail (<= 3)
-      const T res = team.template reduce<Op>(p);
+      const T pk = Op::apply(part[k], Op::apply(Op::apply(acc[k].x, acc[k].y), Op::apply(acc[k].z, acc[k].w)));
+      const T res = team.template reduce<Op>(pk);
       if (team.is_master() && item[k] < N) out[item[k]] = init ? Op::apply(init[item[k]], res) : res;
     }
   }
@@ -123,7 +134,7 @@ template <class T, class Op, int S, int DIST>
 __global__ void __launch_bounds__(32 * S)
 ragged_inter_kernel(const T* __restrict__ in, const int64_t* __restrict__ off,
                     const T* __restrict__ init, T* __restrict__ out, int64_t N) {
-  __shared__ int64_t slot_b[32], slot_e[32];
+  __shared__ int64_t slot_b[32], slot_l[32];
   __shared__ T red[S][33];
   const InterTeam<S> team;
   const int64_t ngroups = (N + 31) / 32;
@@ -131,34 +142,34 @@ ragged_inter_kernel(const T* __restrict__ in, const int64_t* __restrict__ off,
   for (int64_t g = blockIdx.x; g < ngroups; g += gridDim.x) {
     const int64_t item = g * 32 + team.master;
     const bool ok = item < N;
-    int64_t b0 = 0, e0 = 0;
+    int64_t b0 = 0, l0 = 0;
     if (team.is_master() && ok) {
       b0 = off[item];
-      e0 = off[item + 1];
-      if (e0 < b0) e0 = b0;
+      l0 = off[item + 1] - b0;
+      if (l0 < 0) l0 = 0;
     }
     const int64_t b = team.read_from_master(b0, slot_b);
-    const int64_t e = team.read_from_master(e0, slot_e);
-    int64_t hb, nu;
-    split_segment(in, b, e, hb, nu);
-    const Range<S, DIST> r(nu, 4 * nu, 4, team.slave);
-    T p = id;
-    for (int64_t i = b + team.slave; i < hb; i += S) p = Op::apply(p, in[i]);
+    const int64_t len = team.read_from_master(l0, slot_l);
+    const SegShare<T, S, DIST> sh(in, b, len, team.slave);
+    T pv = id;
+    for (int i = team.slave; i < sh.head; i += S) pv = Op::apply(pv, in[b + i]);
+    const T* tl = in + b + sh.head + 4 * ((len - sh.head) >> 2);
+    for (int i = team.slave; i < sh.tail; i += S) pv = Op::apply(pv, tl[i]);
     V4<T> acc = {id, id, id, id};
-    for (int64_t u = r.begin; u < r.end; u += r.step) acc = op4r<T, Op>(acc, ldg4(in + hb + 4 * u));
-    p = Op::apply(p, Op::apply(Op::apply(acc.x, acc.y), Op::apply(acc.z, acc.w)));
-    const int64_t tb = hb + 4 * nu;
-    for (int64_t i = tb + team.slave; i < e; i += S) p = Op::apply(p, in[i]);
+    const T* q = sh.body;
+#pragma unroll 4
+    for (int c = 0; c < sh.cnt; ++c, q += sh.step) acc = op4r<T, Op>(acc, ldg4(q));
+    pv = Op::apply(pv, Op::apply(Op::apply(acc.x, acc.y), Op::apply(acc.z, acc.w)));
     if (S == 1) {
-      if (ok) out[item] = init ? Op::apply(init[item], p) : p;
+      if (ok) out[item] = init ? Op::apply(init[item], pv) : pv;
       continue;
     }
-    red[team.slave][team.master] = p;
+    red[team.slave][team.master] = pv;
     __syncthreads();
     if (team.is_master() && ok) {
       T res = red[0][team.master];
 #pragma unroll
-      for (int s = 1; s < S; ++s) res = Op::apply(res, red[s][team.master]);
+      for (int s2 = 1; s2 < S; ++s2) res = Op::apply(res, red[s2][team.master]);
       out[item] = init ? Op::apply(init[item], res) : res;
     }
     __syncthreads();
