@@ -133,6 +133,46 @@ def tmv_serial_f32(A: np.ndarray, x: np.ndarray) -> np.ndarray:
     return y
 
 
+def tmv_parallel(A: np.ndarray, x: np.ndarray, threads: int) -> np.ndarray:
+    """orc_tmv over `threads` contiguous column ranges in parallel (outer items
+    are independent; the arithmetic per output is unchanged).  For the
+    all-core CPU baseline only."""
+    from concurrent.futures import ThreadPoolExecutor
+    A = np.ascontiguousarray(A, np.float32)
+    x = np.ascontiguousarray(x, np.float32)
+    h, lda = A.shape
+    y = np.empty(lda, np.float32)
+    bounds = [(g * lda // threads, (g + 1) * lda // threads) for g in range(threads)]
+    L = lib()
+
+    def run(b):
+        j0, j1 = b
+        if j1 > j0:
+            L.orc_tmv(A.ctypes.data + 4 * j0, lda, _p(x), y.ctypes.data + 4 * j0, j1 - j0, h)
+    with ThreadPoolExecutor(threads) as ex:
+        list(ex.map(run, bounds))
+    return y
+
+
+def mv_parallel(A: np.ndarray, x: np.ndarray, threads: int) -> np.ndarray:
+    """orc_mv over `threads` contiguous row ranges in parallel."""
+    from concurrent.futures import ThreadPoolExecutor
+    A = np.ascontiguousarray(A, np.float32)
+    x = np.ascontiguousarray(x, np.float32)
+    h, lda = A.shape
+    y = np.empty(h, np.float32)
+    bounds = [(g * h // threads, (g + 1) * h // threads) for g in range(threads)]
+    L = lib()
+
+    def run(b):
+        i0, i1 = b
+        if i1 > i0:
+            L.orc_mv(A.ctypes.data + 4 * i0 * lda, lda, _p(x), y.ctypes.data + 4 * i0, i1 - i0, lda)
+    with ThreadPoolExecutor(threads) as ex:
+        list(ex.map(run, bounds))
+    return y
+
+
 def mv(A: np.ndarray, x: np.ndarray, w: int | None = None) -> np.ndarray:
     """y[i] = sum_j A[i, j] * x[j]; A is (h, lda) row-major."""
     A = np.ascontiguousarray(A, np.float32)

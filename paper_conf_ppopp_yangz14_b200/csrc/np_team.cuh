@@ -57,7 +57,11 @@ template <class T>
 __device__ __forceinline__ V4<T> ldg4(const T* p) {
   V4<T> r;
   uint32_t a, b, c, d;
+#if defined(CUDANP_L2_256B_ALL)
+  asm volatile("ld.global.nc.L2::256B.v4.b32 {%0,%1,%2,%3}, [%4];"
+#else
   asm volatile("ld.global.nc.v4.b32 {%0,%1,%2,%3}, [%4];"
+#endif
                : "=r"(a), "=r"(b), "=r"(c), "=r"(d) : "l"(p));
   r.x = __builtin_bit_cast(T, a); r.y = __builtin_bit_cast(T, b);
   r.z = __builtin_bit_cast(T, c); r.w = __builtin_bit_cast(T, d);
@@ -68,7 +72,11 @@ template <class T>
 __device__ __forceinline__ V4<T> ldg4_stream(const T* p) {
   V4<T> r;
   uint32_t a, b, c, d;
+#if defined(CUDANP_L2_256B)
+  asm volatile("ld.global.nc.L1::no_allocate.L2::256B.v4.b32 {%0,%1,%2,%3}, [%4];"
+#else
   asm volatile("ld.global.nc.L1::no_allocate.v4.b32 {%0,%1,%2,%3}, [%4];"
+#endif
                : "=r"(a), "=r"(b), "=r"(c), "=r"(d) : "l"(p));
   r.x = __builtin_bit_cast(T, a); r.y = __builtin_bit_cast(T, b);
   r.z = __builtin_bit_cast(T, c); r.w = __builtin_bit_cast(T, d);

@@ -82,3 +82,38 @@ def test_fused_gather_equals_unsharded(world):
     assert np.array_equal(y, O.tmv(A, x))
     X = O.gen_i32(1, "i32_full", 0, N * L).reshape(N, L)
     assert np.array_equal(r, O.reduce(X))
+
+
+def _nccl_g1(q, port):
+    import torch.distributed as dist
+
+    import oracle as O
+    from paper_conf_ppopp_yangz14_b200 import cudanp as C
+    from paper_conf_ppopp_yangz14_b200 import parallel as P
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    torch.cuda.set_device(0)
+    dist.init_process_group("nccl", rank=0, world_size=1, device_id=torch.device("cuda", 0))
+    try:
+        A = torch.empty(H, W, device="cuda")
+        C.cudanp_generate(A, "f32_int4", stream_id=1)
+        x = torch.empty(H, device="cuda")
+        C.cudanp_generate(x, "f32_int4", stream_id=2)
+        y = C.cudanp_tmv(A, x, S=8)
+        root = torch.empty(W, device="cuda")
+        P.gather_to_root(y, root, W, 0, 1)
+        ref = O.tmv(O.gen_f32(1, "f32_int4", 0, H * W).reshape(H, W), O.gen_f32(2, "f32_int4", 0, H))
+        q.put(bool(np.array_equal(root.cpu().numpy(), ref)))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_nccl_world1_degenerate_gather():
+    # NCCL with G = 1 is a degenerate but real path
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    p = ctx.Process(target=_nccl_g1, args=(q, _port()))
+    p.start()
+    ok = q.get(timeout=300)
+    p.join(timeout=60)
+    assert ok and p.exitcode == 0

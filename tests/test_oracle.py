@@ -445,3 +445,12 @@ def test_le_bruteforce_and_layout(orc):
     g2, a2, v2, e2 = orc.le_gicov(np.ascontiguousarray(x.T), thr=0.0, layout=1)
     assert (a2 == ave).all() and (v2 == var).all() and (e2 == ep).all()
     assert np.array_equal(g2, g)
+
+
+def test_parallel_oracle_equals_serial(orc):
+    # the all-core CPU baseline splits outer items only: identical bits
+    A = synth.matrix(200, 301, "f32_unit")
+    x = synth.vector(200, "f32_unit")
+    assert orc.tmv_parallel(A, x, 7).tobytes() == orc.tmv(A, x).tobytes()
+    xm = synth.vector(301, "f32_unit")
+    assert orc.mv_parallel(A, xm, 5).tobytes() == orc.mv(A, xm).tobytes()

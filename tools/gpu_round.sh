@@ -9,6 +9,7 @@ timeout 900 python -m pytest tests -m gpu -q -rf --timeout 900 > $O/pytest_gpu_$
 timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > $O/smoke_$TAG.log 2>&1; echo SMOKE_RC=$? >> $O/smoke_$TAG.log
 timeout 600 python bench.py --impl reference --steps 5 --warmup 1 > $O/bench_ref_$TAG.json 2> $O/bench_ref_$TAG.err
 timeout 600 python bench.py > $O/bench_$TAG.json 2> $O/bench_$TAG.err; echo BENCH_RC=$? >> $O/bench_$TAG.err
+timeout 120 python tools/resource_table.py $TAG > /dev/null 2>&1
 timeout 1500 python tools/sweep.py --out $O/sweep_$TAG.jsonl > $O/sweep_$TAG.log 2>&1; echo SWEEP_RC=$? >> $O/sweep_$TAG.log
 TCFG=$(python -c "import json;d=json.load(open('$O/bench_$TAG.json'));c=d['config']['tmv'];print(f\"{c['S']},{c['dist']},{c['map']}\")" 2>/dev/null || echo 32,block,inter)
 MCFG=$(python -c "import json;d=json.load(open('$O/bench_$TAG.json'));c=d['config']['mv'];print(f\"{c['S']},{c['dist']},{c['map']}\")" 2>/dev/null || echo 32,cyclic,intra)
