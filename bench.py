@@ -141,12 +141,17 @@ def dist_init(ngpus):
     local = int(os.environ.get("LOCAL_RANK", "0"))
     if world != ngpus:
         raise SystemExit(f"--gpus {ngpus} but WORLD_SIZE={world}")
+    # CUDANP_BENCH_BACKEND=gloo (testing only): lets several ranks share one GPU
+    # to exercise the multi-rank logic where NCCL refuses duplicate devices.
+    backend = os.environ.get("CUDANP_BENCH_BACKEND", "nccl")
+    dev = local % max(torch.cuda.device_count(), 1)
+    torch.cuda.set_device(dev)
     if world > 1:
-        torch.cuda.set_device(local)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    else:
-        torch.cuda.set_device(0)
-    return rank, world, local
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", dev))
+        else:
+            dist.init_process_group(backend)
+    return rank, world, dev
 
 
 def barrier(world):
@@ -160,7 +165,8 @@ def max_over_ranks(v: float, world: int) -> float:
         return v
     import torch
     import torch.distributed as dist
-    t = torch.tensor([v], dtype=torch.float64, device="cuda")
+    dev = "cuda" if dist.get_backend() == "nccl" else "cpu"
+    t = torch.tensor([v], dtype=torch.float64, device=dev)
     dist.all_reduce(t, op=dist.ReduceOp.MAX)
     return float(t.item())
 
