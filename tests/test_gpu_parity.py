@@ -443,3 +443,33 @@ def test_reduce_backend_parity(backend):
                     assert_exact(got, ref, what)
                 else:
                     assert_rel(got, ref, L, what)
+
+
+# ------------------------------------------------------------------ edge shapes around team/tile sizes
+def test_edge_shapes_per_S():
+    """N around the masters per CTA / warp tile (31, 32, 33, tile +- 1) and L
+    around S and 4S (S-1, S, S+1, 4S-1, 4S, 4S+1): every tail of the team,
+    warp-tile and vector-unit logic (SURVEY §4 test plan item 2)."""
+    for S in SS:
+        tile = 8 * (32 // S) * 4  # intra-warp reduce: 8 warps x (32/S) items x K=4 tiles
+        Ns = sorted({1, 31, 32, 33, tile - 1, tile, tile + 1})
+        Ls = sorted({max(S - 1, 0), S, S + 1, 4 * S - 1, 4 * S, 4 * S + 1})
+        for N in Ns:
+            for L in Ls:
+                x = synth.items(N, L, "i32_full", seed=N * 131 + L)
+                ini = synth.init(N, "i32_full", seed=L)
+                rr, rs = O.reduce(x, init=ini), O.scan(x, init=ini)
+                xd, inid = dev(x), dev(ini)
+                for dist, map_ in itertools.product(DISTS, MAPS):
+                    what = f"edge S={S} N={N} L={L} dist={dist} map={map_}"
+                    assert_exact(host(C.cudanp_batched_loop_reduce(xd, inid, S=S, dist=dist, map=map_)), rr, what)
+                    assert_exact(host(C.cudanp_batched_loop_scan(xd, inid, S=S, dist=dist, map=map_)), rs, what)
+        # TMV/MV widths around 32*V column strips and 8-master CTAs
+        for w in (31, 32, 33, 127, 128, 129):
+            h = 4 * S + 1
+            A = synth.matrix(h, w, "f32_int4", seed=w)
+            xt, xm = synth.vector(h, "f32_int4"), synth.vector(w, "f32_int4")
+            for dist, map_ in itertools.product(DISTS, MAPS):
+                what = f"edge matvec S={S} h={h} w={w} dist={dist} map={map_}"
+                assert_exact(host(C.cudanp_tmv(dev(A), dev(xt), S=S, dist=dist, map=map_)), O.tmv(A, xt), what)
+                assert_exact(host(C.cudanp_mv(dev(A), dev(xm), S=S, dist=dist, map=map_)), O.mv(A, xm), what)
