@@ -8,9 +8,11 @@ import sys
 
 def main(path, out=None):
     recs = [json.loads(l) for l in open(path) if l.strip()]
+    special = [r for r in recs if r["config"] in ("F3", "E9")]
+    recs = [r for r in recs if r["config"] not in ("F3", "E9")]
     groups = collections.OrderedDict()
     for r in recs:
-        key = (r["config"], r["op"], r.get("dtype"), r.get("opname", ""), r.get("L"))
+        key = (r["config"], r["op"], r.get("dtype"), r.get("opname", "") or r.get("layout", ""), r.get("L"))
         groups.setdefault(key, []).append(r)
     lines = ["| config | op | dtype | L | S=1 | S=2 | S=4 | S=8 | S=16 | S=32 | best (S,dist,map) | best GB/s | % HBM | vs tuned S=1 | vs literal S=1 | vs DP-CTA | vs DP-thread |",
              "|---|---|---|---|---|---|---|---|---|---|---|---|---|---|---|---|---|"]
@@ -38,6 +40,20 @@ def main(path, out=None):
             + f" | {b['S']},{b['dist']},{b['map']} | {b['gbs']:.0f} | {100 * b['gbs'] / 6537:.1f} | "
             + f"{b.get('speedup_vs_s1_tuned', float('nan')):.2f}x | {vs('s1_literal')} | {vs('dp_block')} | "
             + (vs(dp_thr) if dp_thr else "—") + " |")
+    f3 = [r for r in special if r["config"] == "F3"]
+    if f3:
+        lines += ["", "F3 — Fig 1 memcopy (64M floats): impl, m parents x n children, GB/s", "",
+                  "| impl | m | n | GB/s |", "|---|---|---|---|"]
+        lines += [f"| {r['impl']} | {r['m']} | {r['n']} | {r['gbs']:.0f} |" for r in f3]
+    e9 = [r for r in special if r["config"] == "E9"]
+    if e9:
+        t = collections.OrderedDict()
+        for r in e9:
+            t.setdefault((r["dtype"], r["opname"], r["L"], r["S"]), {})[r["backend"]] = r["gbs"]
+        lines += ["", "E9 — Fig 16 analog: team reduction backend (GB/s)", "",
+                  "| dtype | op | L | S | shfl | smem | redux |", "|---|---|---|---|---|---|---|"]
+        lines += [f"| {k[0]} | {k[1]} | {k[2]} | {k[3]} | {v.get('shfl', 0):.0f} | {v.get('smem', 0):.0f} | "
+                  f"{v.get('redux', 0):.0f} |" for k, v in t.items()]
     txt = "\n".join(lines)
     print(txt)
     if out:
