@@ -473,3 +473,28 @@ def test_edge_shapes_per_S():
                 what = f"edge matvec S={S} h={h} w={w} dist={dist} map={map_}"
                 assert_exact(host(C.cudanp_tmv(dev(A), dev(xt), S=S, dist=dist, map=map_)), O.tmv(A, xt), what)
                 assert_exact(host(C.cudanp_mv(dev(A), dev(xm), S=S, dist=dist, map=map_)), O.mv(A, xm), what)
+
+
+def test_full_size_C5_single_gpu_sampled():
+    """C5 at G=1: TMV 65536^2 (16 GiB) and the 64M-item reduce, sampled."""
+    n = 65536
+    A = _gen_matrix(n, n, "f32_unit")
+    x = _gen_vec(n, "f32_unit")
+    rng = np.random.default_rng(11)
+    cols = np.unique(np.concatenate([rng.integers(0, n, 128), [0, n - 1]]))
+    ref = O.tmv_gen(n, n, cols)
+    for S, dist in itertools.product((8, 16, 32), DISTS):
+        y = host(C.cudanp_tmv(A, x, S=S, dist=dist, map=C.INTER_WARP))
+        assert_rel(y[cols], ref, n, f"C5 tmv S={S} dist={dist}")
+    del A
+    torch.cuda.empty_cache()
+    N, L = 1 << 26, 64
+    X = torch.empty(N, L, device="cuda")
+    C.cudanp_generate(X, "f32_unit", stream_id=1)
+    items = np.unique(np.concatenate([rng.integers(0, N, 2048), [0, N - 1]]))
+    ref = O.reduce_gen(L, items, O.F32, "f32_unit")
+    for S, dist in itertools.product((4, 8, 16), DISTS):
+        got = host(C.cudanp_batched_loop_reduce(X, S=S, dist=dist, map=C.INTRA_WARP))
+        assert_rel(got[items], ref, L, f"C5 reduce S={S} dist={dist}")
+    del X
+    torch.cuda.empty_cache()

@@ -275,11 +275,11 @@ def f2(L=150):
                   "gbs": round(nb / (med * 1e-3) / 1e9, 1), "speedup_vs_s1_tuned": round(s1 / med, 3),
                   "speedup_vs_s1_literal": round(lit / med, 3)})
         best = min(res, key=lambda k: res[k][0])
-        emit({"config": "F2", "op": "le_gicov", "dtype": "f32", "N": N, "L": f"{L}/{'pm' if layout else 'im'}",
-              "impl": "s1_literal", "t_median_us": round(lit * 1e3, 2), "alg_bytes": nb,
+        emit({"config": "F2", "op": "le_gicov", "dtype": "f32", "N": N, "L": L,
+              "layout": "point-major" if layout else "item-major", "impl": "s1_literal", "t_median_us": round(lit * 1e3, 2), "alg_bytes": nb,
               "gbs": round(nb / (lit * 1e-3) / 1e9, 1)})
-        emit({"config": "F2", "op": "le_gicov", "dtype": "f32", "N": N, "L": f"{L}/{'pm' if layout else 'im'}",
-              "impl": "best_np", "S": best[0], "dist": DN[best[1]], "map": MN[best[2]],
+        emit({"config": "F2", "op": "le_gicov", "dtype": "f32", "N": N, "L": L,
+              "layout": "point-major" if layout else "item-major", "impl": "best_np", "S": best[0], "dist": DN[best[1]], "map": MN[best[2]],
               "t_median_us": round(res[best][0] * 1e3, 2), "alg_bytes": nb,
               "gbs": round(nb / (res[best][0] * 1e-3) / 1e9, 1),
               "speedup_vs_s1_tuned": round(s1 / res[best][0], 3),
