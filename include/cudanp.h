@@ -69,6 +69,16 @@ typedef enum { CUDANP_SUM = 0, CUDANP_MAX = 1 } cudanp_op;
 int cudanp_tmv(const float* A, int64_t lda, const float* x, float* y,
                int64_t n_outer, int64_t n_inner, int S, int dist, int map, void* stream);
 
+/* TMV with TMA-staged tiles (north star: "TMA or cp.async staging where the
+ * access pattern is strided (as in y=A^T x)"): the inter-warp map of
+ * cudanp_tmv, with one elected thread streaming [32 rows x 128 columns]
+ * tiles of A into an 8-stage shared-memory ring (cp.async.bulk.tensor, an
+ * mbarrier per stage) that the S slave warps consume; cyclic or block rows.
+ * Needs A and y 16-byte aligned, lda % 4 == 0, n_outer % 4 == 0 and both
+ * sizes < 2^31, else CUDANP_ERR_UNSUPPORTED (cudanp_tmv handles any case). */
+int cudanp_tmv_tma(const float* A, int64_t lda, const float* x, float* y,
+                   int64_t n_outer, int64_t n_inner, int S, int dist, void* stream);
+
 /* MV (Table 1 "MV"): y[i] = sum_{j<n_inner} A[i*lda + j] * x[j],
  * for i < n_outer.  Master = row i; inner loop over the w = n_inner columns.
  * A: n_outer x lda fp32 (lda >= n_inner), x: n_inner, y: n_outer. */

@@ -32,6 +32,7 @@ int dp_reduce(bool, const void*, const void*, void*, int64_t, int64_t, int, int,
 int dp_scan(bool, const void*, const void*, void*, int64_t, int64_t, int, cudaStream_t);
 int dp_error_count(int, int64_t*);
 int dp_memcopy(const float*, float*, int64_t, int64_t, int, cudaStream_t);
+int tmv_tma(const float*, int64_t, const float*, float*, int64_t, int64_t, int, int, cudaStream_t);
 int ragged_np(const void*, const int64_t*, const void*, void*, int64_t, int, int, int, int, int,
               cudaStream_t);
 int ragged_literal(const void*, const int64_t*, const void*, void*, int64_t, int, int, cudaStream_t);
@@ -247,6 +248,21 @@ int cudanp_tmv(const float* A, int64_t lda, const float* x, float* y, int64_t n_
   if (rc) return rc;
   return tmv_np(A, lda, x, y, n_outer, n_inner, S, dist, resolve_map(map, true),
                 tmv_vec(A, lda, y, n_outer), as_stream(stream), nullptr);
+}
+
+int cudanp_tmv_tma(const float* A, int64_t lda, const float* x, float* y, int64_t n_outer,
+                   int64_t n_inner, int S, int dist, void* stream) {
+  int rc = check_tmv_args(A, lda, x, y, n_outer, n_inner, S, dist, CUDANP_MAP_INTER_WARP);
+  if (rc) return rc;
+  if (n_outer == 0) return CUDANP_OK;
+  if (n_inner == 0)  // nothing to stream: the plain kernel writes the zeros
+    return tmv_np(A, lda, x, y, n_outer, n_inner, S, dist, MAP_INTER, false, as_stream(stream), nullptr);
+  if (!(aligned16(A) && aligned16(y) && lda % 4 == 0 && n_outer % 4 == 0 &&
+        n_outer < (int64_t(1) << 31) && n_inner < (int64_t(1) << 31))) {
+    set_error("TMA path needs 16-byte aligned A and y, lda %% 4 == 0, n_outer %% 4 == 0, sizes < 2^31");
+    return CUDANP_ERR_UNSUPPORTED;
+  }
+  return tmv_tma(A, lda, x, y, n_outer, n_inner, S, dist, as_stream(stream));
 }
 
 int cudanp_mv(const float* A, int64_t lda, const float* x, float* y, int64_t n_outer,

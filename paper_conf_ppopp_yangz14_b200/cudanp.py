@@ -36,6 +36,7 @@ _P32 = ctypes.POINTER(ctypes.c_int32)
 _SIGS = {
     "cudanp_tmv": [_vp, _i64, _vp, _vp, _i64, _i64, _int, _int, _int, _vp],
     "cudanp_mv": [_vp, _i64, _vp, _vp, _i64, _i64, _int, _int, _int, _vp],
+    "cudanp_tmv_tma": [_vp, _i64, _vp, _vp, _i64, _i64, _int, _int, _vp],
     "cudanp_batched_loop_reduce": [_vp, _vp, _vp, _i64, _i64, _int, _int, _int, _int, _int, _vp],
     "cudanp_batched_loop_scan": [_vp, _vp, _vp, _i64, _i64, _int, _int, _int, _int, _vp],
     "cudanp_batched_loop_reduce_backend": [_vp, _vp, _vp, _i64, _i64, _int, _int, _int, _int, _vp],
@@ -144,6 +145,18 @@ def cudanp_tmv(A, x, y=None, *, S=32, dist=CYCLIC, map=AUTO, n_outer=None, strea
         y = torch.empty(w, dtype=torch.float32, device=A.device)
     _check(load().cudanp_tmv(_ptr(A), lda, _ptr(x), _ptr(y), w, h, S, dist, map, _stream(stream)),
            "cudanp_tmv")
+    return y
+
+
+def cudanp_tmv_tma(A, x, y=None, *, S=8, dist=CYCLIC, n_outer=None, stream=None):
+    """TMV with TMA-staged tiles (inter-warp map); same result contract as cudanp_tmv."""
+    import torch
+    h, lda = A.shape
+    w = lda if n_outer is None else n_outer
+    if y is None:
+        y = torch.empty(w, dtype=torch.float32, device=A.device)
+    _check(load().cudanp_tmv_tma(_ptr(A), lda, _ptr(x), _ptr(y), w, h, S, dist, _stream(stream)),
+           "cudanp_tmv_tma")
     return y
 
 

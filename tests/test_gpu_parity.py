@@ -498,3 +498,40 @@ def test_full_size_C5_single_gpu_sampled():
         assert_rel(got[items], ref, L, f"C5 reduce S={S} dist={dist}")
     del X
     torch.cuda.empty_cache()
+
+
+# ------------------------------------------------------------------ TMA-staged TMV
+def test_tmv_tma_parity():
+    for h, w in [(1, 4), (37, 128), (300, 260), (1000, 516), (1024, 1024), (4097, 132)]:
+        for kind in ("f32_int4", "f32_unit"):
+            A = synth.matrix(h, w, kind)
+            x = synth.vector(h, kind)
+            ref = O.tmv(A, x)
+            Ad, xd = dev(A), dev(x)
+            for S, dist in itertools.product(SS, DISTS):
+                got = host(C.cudanp_tmv_tma(Ad, xd, S=S, dist=dist))
+                what = f"tma h={h} w={w} {kind} S={S} dist={dist}"
+                if kind == "f32_int4":
+                    assert_exact(got, ref, what)
+                else:
+                    assert_rel(got, ref, h, what)
+    # padded lda, and the unsupported cases
+    A = synth.matrix(50, 72, "f32_int4")
+    xd = dev(synth.vector(50, "f32_int4"))
+    got = host(C.cudanp_tmv_tma(dev(A), xd, S=4, n_outer=64))
+    assert_exact(got, O.tmv(A, synth.vector(50, "f32_int4"), 64), "tma lda")
+    with pytest.raises(C.CudanpError) as ei:
+        C.cudanp_tmv_tma(dev(synth.matrix(5, 6, "f32_int4")), dev(synth.vector(5, "f32_int4")))
+    assert ei.value.status == C.ERR_UNSUPPORTED
+
+
+def test_tmv_tma_full_size_C2():
+    n = 16384
+    A = _gen_matrix(n, n, "f32_unit")
+    x = _gen_vec(n, "f32_unit")
+    cols = np.arange(0, n, 61)
+    ref = O.tmv_gen(n, n, cols)
+    for S, dist in itertools.product(SS, DISTS):
+        assert_rel(host(C.cudanp_tmv_tma(A, x, S=S, dist=dist))[cols], ref, n, f"C2 tma S={S} d={dist}")
+    del A
+    torch.cuda.empty_cache()

@@ -150,7 +150,19 @@ def c2():
             comps.append((name, time_ms(lambda: fv(impl, A, x, y), reps=3, warm=1)[0]))
         sweep_np("C2", op, nb, lambda S, d, m: time_ms(lambda: fnp(A, x, y, S=S, dist=d, map=m)),
                  {"dtype": "f32", "N": n, "L": n}, literal=lit, comps=comps)
+    tma_sweep("C2", A, x, y, n)
     del A
+
+
+def tma_sweep(cfg, A, x, y, n):
+    """TMA-staged TMV (cudanp_tmv_tma), every S x dist."""
+    nb = 4 * n * n + 8 * n
+    for S in C.SLAVE_SIZES:
+        for d in (C.CYCLIC, C.BLOCK):
+            med, mn = time_ms(lambda: C.cudanp_tmv_tma(A, x, y, S=S, dist=d))
+            emit({"config": cfg, "op": "tmv_tma", "dtype": "f32", "N": n, "L": n, "S": S, "dist": DN[d],
+                  "map": "inter", "impl": "np_tma", "t_median_us": round(med * 1e3, 2),
+                  "alg_bytes": nb, "gbs": round(nb / (med * 1e-3) / 1e9, 1)})
 
 
 def c3(Ls=(32, 64, 128, 256, 80, 150)):
@@ -206,6 +218,7 @@ def c5():
     x = gen((n,), "f32_unit", stream_id=2)
     y = torch.empty(n, device="cuda")
     nb = 4 * n * n + 8 * n
+    tma_sweep("C5", A, x, y, n)
     for S, d in itertools.product((8, 16, 32), (C.CYCLIC, C.BLOCK)):
         med, mn = time_ms(lambda: C.cudanp_tmv(A, x, y, S=S, dist=d, map=C.INTER_WARP), reps=3)
         emit({"config": "C5", "op": "tmv", "dtype": "f32", "N": n, "L": n, "G": 1, "S": S, "dist": DN[d],
