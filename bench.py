@@ -367,9 +367,16 @@ def run_cudanp(args):
     def gbs(nb, t):
         return round(nb / (t * 1e-3) / 1e9, 1)
 
+    # "tuned S=1" = the best no-NP kernel: the S=1 instantiations and the literal
+    def best_s1(op):
+        c = [v for (S, d, m), v in sweep[op].items() if S == 1]
+        if f"{op}_s1_literal" in comp:
+            c.append(comp[f"{op}_s1_literal"])
+        return min(c or [float("nan")])
+
     per_S = {}
     for op, nb in (("tmv", bytes_t), ("mv", bytes_m)):
-        s1 = min([v for (S, d, m), v in sweep[op].items() if S == 1] or [float("nan")])
+        s1 = best_s1(op)
         for S in C.SLAVE_SIZES:
             cand = {k: v for k, v in sweep[op].items() if k[0] == S}
             if not cand:
@@ -382,8 +389,7 @@ def run_cudanp(args):
                 "map": "intra" if k[2] == C.INTRA_WARP else "inter",
                 "all": {f"{'cyc' if d == C.CYCLIC else 'blk'}/{'intra' if m == C.INTRA_WARP else 'inter'}":
                         gbs(nb, v) for (SS, d, m), v in cand.items()}}
-    s1_tmv = min([v for (S, d, m), v in sweep["tmv"].items() if S == 1] or [float("nan")])
-    s1_mv = min([v for (S, d, m), v in sweep["mv"].items() if S == 1] or [float("nan")])
+    s1_tmv, s1_mv = best_s1("tmv"), best_s1("mv")
 
     line = {
         "metric": METRIC, "value": round(value, 2), "unit": "GB/s", "n_gpus": world,
