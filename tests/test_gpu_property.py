@@ -1,0 +1,80 @@
+"""Randomised parity (hypothesis): random N, L, S, dist, map, dtype, op,
+alignment and init against the oracle; integer data so every check is
+bit-exact regardless of the summation order."""
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+if not torch.cuda.is_available():
+    pytest.skip("needs a CUDA device", allow_module_level=True)
+from hypothesis import HealthCheck, given, settings
+from hypothesis import strategies as st
+
+import oracle as O
+import synth
+from paper_conf_ppopp_yangz14_b200 import build as B
+from paper_conf_ppopp_yangz14_b200 import cudanp as C
+from test_gpu_parity import assert_exact, dev, host
+
+pytestmark = pytest.mark.gpu
+B.build()
+C.load()
+
+S_ = st.sampled_from(C.SLAVE_SIZES)
+D_ = st.sampled_from([C.CYCLIC, C.BLOCK])
+M_ = st.sampled_from([C.INTRA_WARP, C.INTER_WARP, C.AUTO])
+CFG = settings(max_examples=150, deadline=None, suppress_health_check=list(HealthCheck))
+
+
+@CFG
+@given(N=st.integers(0, 700), L=st.integers(0, 300), S=S_, dist=D_, map_=M_,
+       op=st.sampled_from([C.SUM, C.MAX]), shift=st.integers(0, 3), use_init=st.booleans(),
+       seed=st.integers(0, 10**6))
+def test_reduce_random(N, L, S, dist, map_, op, shift, use_init, seed):
+    x = synth.gen(1, "i32_full", 0, N * L + shift, seed=seed)
+    xd = dev(x)[shift:].view(N, L) if N * L else dev(x)[: 0].view(N, L)
+    ini = synth.init(N, "i32_full", seed=seed)
+    ref = O.reduce(x[shift:].reshape(N, L), op=op, init=ini if use_init else None)
+    got = host(C.cudanp_batched_loop_reduce(xd, dev(ini) if use_init and N else None, op=op,
+                                            S=S, dist=dist, map=map_))
+    assert_exact(got, ref, f"N={N} L={L} S={S} dist={dist} map={map_} op={op} shift={shift}")
+
+
+@CFG
+@given(N=st.integers(0, 400), L=st.integers(0, 300), S=S_, dist=D_, map_=M_,
+       shift=st.integers(0, 3), use_init=st.booleans(), seed=st.integers(0, 10**6))
+def test_scan_random(N, L, S, dist, map_, shift, use_init, seed):
+    x = synth.gen(1, "i32_small", 0, N * L + shift, B=1 << 15, seed=seed)
+    xd = dev(x)[shift:].view(N, L) if N * L else dev(x)[: 0].view(N, L)
+    ini = synth.init(N, "i32_small", B=1 << 15, seed=seed)
+    ref = O.scan(x[shift:].reshape(N, L), init=ini if use_init else None)
+    got = host(C.cudanp_batched_loop_scan(xd, dev(ini) if use_init and N else None, S=S, dist=dist,
+                                          map=map_))
+    assert_exact(got, ref, f"N={N} L={L} S={S} dist={dist} map={map_} shift={shift}")
+
+
+@CFG
+@given(h=st.integers(0, 300), w=st.integers(1, 300), pad=st.integers(0, 5), S=S_, dist=D_,
+       map_=M_, seed=st.integers(0, 10**6))
+def test_matvec_random(h, w, pad, S, dist, map_, seed):
+    lda = w + pad
+    A = synth.matrix(h, lda, "f32_int4", seed=seed)
+    xt, xm = synth.vector(h, "f32_int4", seed=seed), synth.vector(w, "f32_int4", seed=seed)
+    Ad = dev(A)
+    what = f"h={h} w={w} lda={lda} S={S} dist={dist} map={map_}"
+    ref_t = O.tmv(A, xt, w) if h else np.zeros(w, np.float32)
+    assert_exact(host(C.cudanp_tmv(Ad, dev(xt), S=S, dist=dist, map=map_, n_outer=w)), ref_t, "tmv " + what)
+    if h:
+        assert_exact(host(C.cudanp_mv(Ad, dev(xm), S=S, dist=dist, map=map_, n_inner=w)),
+                     O.mv(A, xm, w), "mv " + what)
+
+
+@CFG
+@given(N=st.integers(1, 500), mean=st.integers(0, 80), S=S_, dist=D_, map_=M_,
+       op=st.sampled_from([C.SUM, C.MAX]), shift=st.integers(0, 3), seed=st.integers(0, 10**6))
+def test_ragged_random(N, mean, S, dist, map_, op, shift, seed):
+    lens = synth.lengths(N, mean, "exp", seed=seed)
+    off = synth.offsets_from_lengths(lens) + shift
+    x = synth.gen(1, "i32_full", 0, int(off[-1]) + 1, seed=seed)
+    got = host(C.cudanp_ragged_loop_reduce(dev(x), dev(off), op=op, S=S, dist=dist, map=map_))
+    assert_exact(got, O.ragged_reduce(x, off, op=op), f"N={N} mean={mean} S={S} d={dist} m={map_}")

@@ -454,3 +454,26 @@ def test_parallel_oracle_equals_serial(orc):
     assert orc.tmv_parallel(A, x, 7).tobytes() == orc.tmv(A, x).tobytes()
     xm = synth.vector(301, "f32_unit")
     assert orc.mv_parallel(A, xm, 5).tobytes() == orc.mv(A, xm).tobytes()
+
+
+# ------------------------------------------------------------------ randomised oracle invariants
+from hypothesis import given, settings  # noqa: E402
+from hypothesis import strategies as st  # noqa: E402
+
+
+@settings(max_examples=60, deadline=None)
+@given(N=st.integers(1, 30), L=st.integers(0, 40), seed=st.integers(0, 10**6))
+def test_oracle_invariants_random(orc, N, L, seed):
+    x = synth.items(N, L, "i32_full", seed=seed)
+    ini = synth.init(N, "i32_full", seed=seed)
+    r, sc = orc.reduce(x, init=ini), orc.scan(x, init=ini)
+    exact = [((int(i) + sum(int(v) for v in row) + (1 << 31)) % (1 << 32)) - (1 << 31) for i, row in zip(ini, x)]
+    assert r.tolist() == exact
+    if L:
+        assert (sc[:, -1] == r).all()
+    xf = synth.items(N, L, "f32_int4", seed=seed)
+    assert (orc.reduce(xf) == xf.astype(np.int64).sum(1)).all()
+    assert (orc.reduce(xf, op=orc.MAX) == (xf.max(1) if L else -np.inf)).all()
+    A = synth.matrix(N, L + 1, "f32_int4", seed=seed)
+    xv = synth.vector(N, "f32_int4", seed=seed)
+    assert orc.tmv(A, xv).tobytes() == orc.mv(np.ascontiguousarray(A.T), xv).tobytes()
