@@ -20,7 +20,10 @@
 namespace cudanp {
 
 constexpr int kReduceBlock = 256;  // intra-warp CTA: 8 warps
-constexpr int kReduceK = 4;        // warp tiles in flight per warp (intra)
+#ifndef CUDANP_REDUCE_K
+#define CUDANP_REDUCE_K 4
+#endif
+constexpr int kReduceK = CUDANP_REDUCE_K;  // warp tiles in flight per warp (intra)
 
 template <class T, class Op>
 __device__ __forceinline__ T fold4(V4<T> v) {

@@ -21,7 +21,10 @@
 namespace cudanp {
 
 constexpr int kScanBlock = 256;
-constexpr int kScanK = 2;  // warp tiles per warp step (intra)
+#ifndef CUDANP_SCAN_K
+#define CUDANP_SCAN_K 2
+#endif
+constexpr int kScanK = CUDANP_SCAN_K;  // warp tiles per warp step (intra)
 
 template <class T>
 __device__ __forceinline__ void local_scan4(V4<T>& v) {

@@ -283,9 +283,7 @@ def f2(L=150):
                     if m == C.INTRA_WARP and S & (S - 1):
                         continue
                     res[(S, d, m)] = run(S, d, m)
-        # "tuned S=1" = the best no-NP kernel: the S=1 NP-path instantiations and the
-    # Fig 2 literal, whichever is faster.
-    s1 = min([v[0] for k, v in res.items() if k[0] == 1] + ([literal] if literal else []))
+        s1 = min([v[0] for k, v in res.items() if k[0] == 1] + [lit])  # best no-NP kernel
         for (S, d, m), (med, mn) in res.items():
             emit({"config": "F2", "op": "le_gicov", "dtype": "f32", "N": N, "L": L,
                   "layout": "point-major" if layout else "item-major", "S": S, "dist": DN[d], "map": MN[m],
