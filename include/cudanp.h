@@ -16,6 +16,11 @@
  *         CUDANP_MAP_INTER_WARP (team = one lane in each of S warps)
  *         (P:189-191), CUDANP_MAP_AUTO choosing per the rules of P:340-342.
  * S = 1 means no nesting: the tuned one-thread-per-item kernel.
+ * S in {64, 128, 256, 512, 1024} ("shared-memory fallback when S exceeds
+ * 32"): a team of S/32 consecutive warps, shfl inside each warp and shared
+ * memory across them; supported by the reduce, scan and MV calls with
+ * CUDANP_MAP_AUTO / CUDANP_MAP_INTRA_WARP, and by TMV with the inter-warp
+ * map for S <= 128 (CUDANP_ERR_UNSUPPORTED otherwise).
  *
  * Conventions for every call:
  *  - Data pointers are DEVICE pointers owned by the caller; the library never

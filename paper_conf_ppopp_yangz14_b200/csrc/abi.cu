@@ -75,7 +75,8 @@ static bool size_ok(int64_t a, int64_t b) {  // a*b*4 bytes addressable
 }
 
 static int check_common(int S, int dist, int map, int64_t n_outer, int64_t n_inner) {
-  if (!valid_S(S)) return fail_invalid("S must be one of 1,2,4,8,16,32");
+  if (!valid_S(S) && !valid_big_S(S))
+    return fail_invalid("S must be one of 1,2,4,8,16,32 (or 64..1024 for multi-warp teams)");
   if (dist != CUDANP_DIST_CYCLIC && dist != CUDANP_DIST_BLOCK) return fail_invalid("dist");
   if (map != CUDANP_MAP_AUTO && map != CUDANP_MAP_INTRA_WARP && map != CUDANP_MAP_INTER_WARP)
     return fail_invalid("map");

@@ -31,6 +31,10 @@ inline int check_launch(const char* what) {
 inline bool valid_S(int S) {
   return S == 1 || S == 2 || S == 4 || S == 8 || S == 16 || S == 32;
 }
+// Teams larger than a warp (S/32 consecutive warps; shfl within each warp,
+// shared memory across them): batched reduce/scan and MV with the intra-warp
+// (consecutive-thread) map, TMV with the inter-warp map for S <= 128.
+inline bool valid_big_S(int S) { return S == 64 || S == 128 || S == 256 || S == 512 || S == 1024; }
 
 inline bool aligned16(const void* p) { return ((uintptr_t)p & 15u) == 0; }
 
@@ -52,6 +56,22 @@ inline int64_t persistent_grid(K kernel, int block_threads, size_t dyn_smem, int
   int64_t cap = (int64_t)per_sm * sm_count();
   if (work_ctas < 1) work_ctas = 1;
   return work_ctas < cap ? work_ctas : cap;
+}
+
+// Persistent intra-warp launch where each warp takes K consecutive warp tiles
+// per step: returns the grid and the effective tiles per step `keff` -- K
+// for large problems, fewer when there are not enough tiles to give every
+// resident warp K of them (so few-item launches still use every SM).
+template <class Kn>
+inline int64_t tiled_grid(Kn kernel, int block_threads, int64_t ntiles, int K, int* keff) {
+  const int64_t cap_ctas = persistent_grid(kernel, block_threads, 0, INT64_MAX / 4);
+  const int64_t warps = cap_ctas * (block_threads / 32);
+  int64_t k = (ntiles + warps - 1) / warps;
+  if (k < 1) k = 1;
+  if (k > K) k = K;
+  *keff = (int)k;
+  const int64_t per_cta = (block_threads / 32) * k;
+  return persistent_grid(kernel, block_threads, 0, (ntiles + per_cta - 1) / per_cta);
 }
 
 template <class K>

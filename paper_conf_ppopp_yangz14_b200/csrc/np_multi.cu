@@ -1,0 +1,361 @@
+// np_multi.cu -- teams larger than a warp: S in {64, 128, 256, 512, 1024}.
+//
+// The north star asks for "warp-shuffle reduction and scan trees with a
+// shared-memory fallback when S exceeds 32".  A team of S > 32 threads is S/32
+// consecutive warps of one CTA (the paper's TB enlargement up to 1024
+// threads, taken to a single master per CTA when S = 1024): the
+// distribution of the loop is the same (cyclic P:166 / block R5); the
+// reduction and scan run as shfl trees inside each warp (intra-warp)
+// and combine the S/32 warp results through shared memory (P:209,
+// inter-warp).  Few outer items with long loops (MV with few rows, a batched
+// reduce over few long items) get the whole GPU this way.
+#include "common.cuh"
+#include "np_team.cuh"
+
+namespace cudanp {
+
+// ---------------------------------------------------------------- the team
+template <int S>
+struct MultiTeam {
+  static_assert(S % 32 == 0 && S >= 64 && S <= 1024, "multi-warp teams: S = 64..1024");
+  static constexpr int W = S / 32;  // warps per team
+  int slave, team, lane, wit;       // wit: warp index inside the team
+  __device__ __forceinline__ MultiTeam() {
+    slave = threadIdx.x % S;
+    team = threadIdx.x / S;
+    lane = threadIdx.x & 31;
+    wit = slave >> 5;
+  }
+  __device__ __forceinline__ bool is_master() const { return slave == 0; }
+
+  // Reduction: shfl butterfly per warp, then the team's W warp results through
+  // shared memory.  Every CTA thread must call it (it holds CTA barriers);
+  // every team member returns the team's result.
+  template <class Op, class T>
+  __device__ __forceinline__ T reduce(T v, T* sm /*[teams*W]*/) const {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v = Op::apply(v, __shfl_xor_sync(kFull, v, o));
+    if (lane == 0) sm[team * W + wit] = v;
+    __syncthreads();
+    T r = sm[team * W];
+#pragma unroll 4
+    for (int k = 1; k < W; ++k) r = Op::apply(r, sm[team * W + k]);
+    __syncthreads();
+    return r;
+  }
+  // Inclusive scan over the S team threads; *total = the team's sum.
+  template <class T>
+  __device__ __forceinline__ T inclusive_scan(T v, T* sm /*[teams*W]*/, T* total) const {
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const T t = __shfl_up_sync(kFull, v, o);
+      if (lane >= o) v = OpSum::apply(v, t);
+    }
+    if (lane == 31) sm[team * W + wit] = v;
+    __syncthreads();
+    T off = T(0), tot = T(0);
+#pragma unroll 4
+    for (int k = 0; k < W; ++k) {
+      const T p = sm[team * W + k];
+      if (k < wit) off = OpSum::apply(off, p);
+      tot = OpSum::apply(tot, p);
+    }
+    __syncthreads();
+    *total = tot;
+    return OpSum::apply(off, v);
+  }
+  // read_from_master through a per-team shared slot.
+  template <class T>
+  __device__ __forceinline__ T read_from_master(T v, T* slot /*[teams]*/) const {
+    if (slave == 0) slot[team] = v;
+    __syncthreads();
+    const T r = slot[team];
+    __syncthreads();
+    return r;
+  }
+};
+
+template <int S> struct MultiShape {
+  static constexpr int CTA = S < 256 ? 256 : S;  // threads per CTA
+  static constexpr int TEAMS = CTA / S;          // teams (items) per CTA
+  static constexpr int MINB = 1024 / CTA;        // CTAs per SM -> 64 registers/thread
+};
+
+// a - b with int32 wrapping modulo 2^32 (R13)
+__device__ __forceinline__ float tsub(float a, float b) { return a - b; }
+__device__ __forceinline__ int32_t tsub(int32_t a, int32_t b) { return (int32_t)((uint32_t)a - (uint32_t)b); }
+
+template <class T, class Op>
+__device__ __forceinline__ V4<T> mop4(V4<T> a, V4<T> b) {
+  return {Op::apply(a.x, b.x), Op::apply(a.y, b.y), Op::apply(a.z, b.z), Op::apply(a.w, b.w)};
+}
+
+// ---------------------------------------------------------------- batched reduce
+template <class T, class Op, int S, int DIST, bool VEC>
+__global__ void __launch_bounds__(MultiShape<S>::CTA, MultiShape<S>::MINB)
+reduce_multi_kernel(const T* __restrict__ in, const T* __restrict__ init, T* __restrict__ out,
+                    int64_t N, int64_t L) {
+  using Sh = MultiShape<S>;
+  __shared__ T sm[Sh::TEAMS * MultiTeam<S>::W];
+  const MultiTeam<S> team;
+  const int64_t nunits = VEC ? (L >> 2) : L;
+  const Range<S, DIST> r(nunits, L, VEC ? 4 : 1, team.slave);
+  const int64_t ngroups = (N + Sh::TEAMS - 1) / Sh::TEAMS;
+  const T id = Op::template identity<T>();
+  for (int64_t g = blockIdx.x; g < ngroups; g += gridDim.x) {
+    const int64_t item = g * Sh::TEAMS + team.team;
+    const bool ok = item < N;
+    const T* row = in + (ok ? item : 0) * L;
+    V4<T> acc = {id, id, id, id};
+    if (ok) {
+      int64_t u = r.begin;
+      constexpr int U = 4;
+      for (; u + (U - 1) * r.step < r.end; u += U * r.step) {
+        V4<T> v[U];
+#pragma unroll
+        for (int j = 0; j < U; ++j) {
+          if constexpr (VEC) v[j] = ldg4(row + 4 * (u + j * r.step));
+          else v[j] = {ldg1(row + u + j * r.step), id, id, id};
+        }
+#pragma unroll
+        for (int j = 0; j < U; ++j) acc = mop4<T, Op>(acc, v[j]);
+      }
+      for (; u < r.end; u += r.step) {
+        if constexpr (VEC) acc = mop4<T, Op>(acc, ldg4(row + 4 * u));
+        else acc.x = Op::apply(acc.x, ldg1(row + u));
+      }
+    }
+    const T p = Op::apply(Op::apply(acc.x, acc.y), Op::apply(acc.z, acc.w));
+    const T res = team.template reduce<Op>(p, sm);
+    if (team.is_master() && ok) out[item] = init ? Op::apply(init[item], res) : res;
+  }
+}
+
+// ---------------------------------------------------------------- MV
+template <int S, int DIST, bool VEC>
+__global__ void __launch_bounds__(MultiShape<S>::CTA, MultiShape<S>::MINB)
+mv_multi_kernel(const float* __restrict__ A, int64_t lda, const float* __restrict__ x,
+                float* __restrict__ y, int64_t h, int64_t w) {
+  using Sh = MultiShape<S>;
+  __shared__ float sm[Sh::TEAMS * MultiTeam<S>::W];
+  const MultiTeam<S> team;
+  const int64_t nunits = VEC ? (w >> 2) : w;
+  const Range<S, DIST> r(nunits, w, VEC ? 4 : 1, team.slave);
+  const int64_t ngroups = (h + Sh::TEAMS - 1) / Sh::TEAMS;
+  for (int64_t g = blockIdx.x; g < ngroups; g += gridDim.x) {
+    const int64_t rowi = g * Sh::TEAMS + team.team;
+    const bool ok = rowi < h;
+    const float* a = A + (ok ? rowi : 0) * lda;
+    V4<float> acc = {0.f, 0.f, 0.f, 0.f};
+    if (ok) {
+      int64_t u = r.begin;
+      constexpr int U = 4;
+      for (; u + (U - 1) * r.step < r.end; u += U * r.step) {
+        V4<float> av[U], xv[U];
+#pragma unroll
+        for (int j = 0; j < U; ++j) {
+          const int64_t uu = u + j * r.step;
+          if constexpr (VEC) { av[j] = ldg4_stream(a + 4 * uu); xv[j] = ldg4(x + 4 * uu); }
+          else { av[j].x = ldg1(a + uu); xv[j].x = ldg1(x + uu); }
+        }
+#pragma unroll
+        for (int j = 0; j < U; ++j) {
+          acc.x = fmaf(av[j].x, xv[j].x, acc.x);
+          if constexpr (VEC) {
+            acc.y = fmaf(av[j].y, xv[j].y, acc.y);
+            acc.z = fmaf(av[j].z, xv[j].z, acc.z);
+            acc.w = fmaf(av[j].w, xv[j].w, acc.w);
+          }
+        }
+      }
+      for (; u < r.end; u += r.step) {
+        if constexpr (VEC) {
+          const V4<float> av = ldg4_stream(a + 4 * u), xv = ldg4(x + 4 * u);
+          acc.x = fmaf(av.x, xv.x, acc.x); acc.y = fmaf(av.y, xv.y, acc.y);
+          acc.z = fmaf(av.z, xv.z, acc.z); acc.w = fmaf(av.w, xv.w, acc.w);
+        } else {
+          acc.x = fmaf(ldg1(a + u), ldg1(x + u), acc.x);
+        }
+      }
+    }
+    const float p = (acc.x + acc.y) + (acc.z + acc.w);
+    const float res = team.template reduce<OpSum>(p, sm);
+    if (team.is_master() && ok) y[rowi] = res;
+  }
+}
+
+// ---------------------------------------------------------------- batched scan
+template <class T, int S, int DIST, bool VEC>
+__global__ void __launch_bounds__(MultiShape<S>::CTA, MultiShape<S>::MINB)
+scan_multi_kernel(const T* __restrict__ in, const T* __restrict__ init, T* __restrict__ out,
+                  int64_t N, int64_t L) {
+  using Sh = MultiShape<S>;
+  __shared__ T sm[Sh::TEAMS * MultiTeam<S>::W];
+  __shared__ T slot[Sh::TEAMS];
+  const MultiTeam<S> team;
+  constexpr int V = VEC ? 4 : 1;
+  const int64_t nunits = VEC ? (L >> 2) : L;
+  const int64_t ngroups = (N + Sh::TEAMS - 1) / Sh::TEAMS;
+  for (int64_t g = blockIdx.x; g < ngroups; g += gridDim.x) {
+    const int64_t item = g * Sh::TEAMS + team.team;
+    const bool ok = item < N;
+    const T* irow = in + (ok ? item : 0) * L;
+    T* orow = out + (ok ? item : 0) * L;
+    T carry = T(0);
+    if (init) {  // live-in: the master loads it and broadcasts it
+      T c = T(0);
+      if (team.is_master() && ok) c = init[item];
+      carry = team.read_from_master(c, slot);
+    }
+    if constexpr (DIST == DIST_CYCLIC) {
+      const int64_t nrounds = (nunits + S - 1) / S;
+      for (int64_t rd = 0; rd < nrounds; ++rd) {
+        const int64_t u = rd * S + team.slave;
+        const bool uok = ok && u < nunits;
+        V4<T> v = {T(0), T(0), T(0), T(0)};
+        if (uok) {
+          if constexpr (VEC) v = ldg4(irow + 4 * u);
+          else v.x = ldg1(irow + u);
+        }
+        if constexpr (VEC) {
+          v.y = OpSum::apply(v.x, v.y); v.z = OpSum::apply(v.y, v.z); v.w = OpSum::apply(v.z, v.w);
+        }
+        const T tot = VEC ? v.w : v.x;
+        T all;
+        const T incl = team.inclusive_scan(tot, sm, &all);
+        const T add = OpSum::apply(carry, tsub(incl, tot));  // carry + exclusive prefix
+        if (uok) {
+          if constexpr (VEC)
+            stg4(orow + 4 * u, V4<T>{OpSum::apply(v.x, add), OpSum::apply(v.y, add),
+                                     OpSum::apply(v.z, add), OpSum::apply(v.w, add)});
+          else orow[u] = OpSum::apply(add, v.x);
+        }
+        carry = OpSum::apply(carry, all);
+      }
+    } else {
+      const Range<S, DIST> r(nunits, L, V, team.slave);
+      T csum = T(0);
+      if (ok) {
+        for (int64_t u = r.begin; u < r.end; ++u) {
+          if constexpr (VEC) {
+            const V4<T> v = ldg4(irow + 4 * u);
+            csum = OpSum::apply(csum, OpSum::apply(OpSum::apply(v.x, v.y), OpSum::apply(v.z, v.w)));
+          } else {
+            csum = OpSum::apply(csum, ldg1(irow + u));
+          }
+        }
+      }
+      T all;
+      const T incl = team.inclusive_scan(csum, sm, &all);
+      T run = OpSum::apply(carry, tsub(incl, csum));
+      if (ok) {
+        for (int64_t u = r.begin; u < r.end; ++u) {
+          if constexpr (VEC) {
+            V4<T> v = ldg4(irow + 4 * u);
+            v.x = OpSum::apply(run, v.x); v.y = OpSum::apply(v.x, v.y);
+            v.z = OpSum::apply(v.y, v.z); v.w = OpSum::apply(v.z, v.w);
+            stg4(orow + 4 * u, v);
+            run = v.w;
+          } else {
+            run = OpSum::apply(run, ldg1(irow + u));
+            orow[u] = run;
+          }
+        }
+      }
+    }
+  }
+}
+
+// ---------------------------------------------------------------- dispatch
+#define CUDANP_DISPATCH_BIG_S(S, ...)                        \
+  switch (S) {                                               \
+    case 64: { constexpr int kS = 64; __VA_ARGS__; } break;     \
+    case 128: { constexpr int kS = 128; __VA_ARGS__; } break;   \
+    case 256: { constexpr int kS = 256; __VA_ARGS__; } break;   \
+    case 512: { constexpr int kS = 512; __VA_ARGS__; } break;   \
+    case 1024: { constexpr int kS = 1024; __VA_ARGS__; } break; \
+    default: return fail_invalid("S must be 64, 128, 256, 512 or 1024 for a multi-warp team"); \
+  }
+
+template <class K>
+static int64_t multi_grid(K kern, int cta, int64_t groups) {
+  return persistent_grid(kern, cta, 0, groups);
+}
+
+template <class T, class Op>
+static int reduce_multi_t(const void* in, const void* init, void* out, int64_t N, int64_t L, int S,
+                          int dist, bool vec, cudaStream_t st, LaunchInfo* info) {
+  CUDANP_DISPATCH_BIG_S(S, {
+    using Sh = MultiShape<kS>;
+    auto kern = dist == DIST_CYCLIC
+                    ? (vec ? reduce_multi_kernel<T, Op, kS, DIST_CYCLIC, true> : reduce_multi_kernel<T, Op, kS, DIST_CYCLIC, false>)
+                    : (vec ? reduce_multi_kernel<T, Op, kS, DIST_BLOCK, true> : reduce_multi_kernel<T, Op, kS, DIST_BLOCK, false>);
+    const int64_t grid = multi_grid(kern, Sh::CTA, (N + Sh::TEAMS - 1) / Sh::TEAMS);
+    if (info) {
+      info->block_threads = Sh::CTA; info->grid = grid; info->map = MAP_INTRA;
+      kernel_attrs(kern, &info->regs, &info->smem);
+      return CUDANP_OK;
+    }
+    if (N == 0) return CUDANP_OK;
+    kern<<<(unsigned)grid, Sh::CTA, 0, st>>>((const T*)in, (const T*)init, (T*)out, N, L);
+    return check_launch("batched_loop_reduce (multi-warp team) launch");
+  });
+  return CUDANP_OK;
+}
+
+int reduce_multi(const void* in, const void* init, void* out, int64_t N, int64_t L, int dtype,
+                 int op, int S, int dist, bool vec, cudaStream_t st, LaunchInfo* info) {
+  if (dtype == CUDANP_F32)
+    return op == CUDANP_SUM ? reduce_multi_t<float, OpSum>(in, init, out, N, L, S, dist, vec, st, info)
+                            : reduce_multi_t<float, OpMax>(in, init, out, N, L, S, dist, vec, st, info);
+  return op == CUDANP_SUM ? reduce_multi_t<int32_t, OpSum>(in, init, out, N, L, S, dist, vec, st, info)
+                          : reduce_multi_t<int32_t, OpMax>(in, init, out, N, L, S, dist, vec, st, info);
+}
+
+template <class T>
+static int scan_multi_t(const void* in, const void* init, void* out, int64_t N, int64_t L, int S,
+                        int dist, bool vec, cudaStream_t st, LaunchInfo* info) {
+  CUDANP_DISPATCH_BIG_S(S, {
+    using Sh = MultiShape<kS>;
+    auto kern = dist == DIST_CYCLIC
+                    ? (vec ? scan_multi_kernel<T, kS, DIST_CYCLIC, true> : scan_multi_kernel<T, kS, DIST_CYCLIC, false>)
+                    : (vec ? scan_multi_kernel<T, kS, DIST_BLOCK, true> : scan_multi_kernel<T, kS, DIST_BLOCK, false>);
+    const int64_t grid = multi_grid(kern, Sh::CTA, (N + Sh::TEAMS - 1) / Sh::TEAMS);
+    if (info) {
+      info->block_threads = Sh::CTA; info->grid = grid; info->map = MAP_INTRA;
+      kernel_attrs(kern, &info->regs, &info->smem);
+      return CUDANP_OK;
+    }
+    if (N == 0 || L == 0) return CUDANP_OK;
+    kern<<<(unsigned)grid, Sh::CTA, 0, st>>>((const T*)in, (const T*)init, (T*)out, N, L);
+    return check_launch("batched_loop_scan (multi-warp team) launch");
+  });
+  return CUDANP_OK;
+}
+
+int scan_multi(const void* in, const void* init, void* out, int64_t N, int64_t L, int dtype, int S,
+               int dist, bool vec, cudaStream_t st, LaunchInfo* info) {
+  return dtype == CUDANP_F32 ? scan_multi_t<float>(in, init, out, N, L, S, dist, vec, st, info)
+                             : scan_multi_t<int32_t>(in, init, out, N, L, S, dist, vec, st, info);
+}
+
+int mv_multi(const float* A, int64_t lda, const float* x, float* y, int64_t h, int64_t w, int S,
+             int dist, bool vec, cudaStream_t st, LaunchInfo* info) {
+  CUDANP_DISPATCH_BIG_S(S, {
+    using Sh = MultiShape<kS>;
+    auto kern = dist == DIST_CYCLIC ? (vec ? mv_multi_kernel<kS, DIST_CYCLIC, true> : mv_multi_kernel<kS, DIST_CYCLIC, false>)
+                                    : (vec ? mv_multi_kernel<kS, DIST_BLOCK, true> : mv_multi_kernel<kS, DIST_BLOCK, false>);
+    const int64_t grid = multi_grid(kern, Sh::CTA, (h + Sh::TEAMS - 1) / Sh::TEAMS);
+    if (info) {
+      info->block_threads = Sh::CTA; info->grid = grid; info->map = MAP_INTRA;
+      kernel_attrs(kern, &info->regs, &info->smem);
+      return CUDANP_OK;
+    }
+    if (h == 0) return CUDANP_OK;
+    kern<<<(unsigned)grid, Sh::CTA, 0, st>>>(A, lda, x, y, h, w);
+    return check_launch("mv (multi-warp team) launch");
+  });
+  return CUDANP_OK;
+}
+
+}  // namespace cudanp

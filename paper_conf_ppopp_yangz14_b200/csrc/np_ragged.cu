@@ -63,7 +63,7 @@ struct SegShare {
 template <class T, class Op, int S, int DIST>
 __global__ void __launch_bounds__(kRaggedBlock)
 ragged_intra_kernel(const T* __restrict__ in, const int64_t* __restrict__ off,
-                    const T* __restrict__ init, T* __restrict__ out, int64_t N) {
+                    const T* __restrict__ init, T* __restrict__ out, int64_t N, int keff) {
   constexpr int TPW = 32 / S;
   constexpr int K = kRaggedK;
   const IntraTeam<S> team;
@@ -72,7 +72,7 @@ ragged_intra_kernel(const T* __restrict__ in, const int64_t* __restrict__ off,
   const int64_t ntiles = (N + TPW - 1) / TPW;
   const T id = Op::template identity<T>();
 
-  for (int64_t t0 = warp * K; t0 < ntiles; t0 += nwarps * K) {
+  for (int64_t t0 = warp * keff; t0 < ntiles; t0 += nwarps * keff) {
     int64_t item[K];
     const T* p[K];
     int64_t pstep[K];
@@ -81,7 +81,7 @@ ragged_intra_kernel(const T* __restrict__ in, const int64_t* __restrict__ off,
     int trips = 0;
 #pragma unroll
     for (int k = 0; k < K; ++k) {
-      item[k] = (t0 + k) * TPW + team.team;
+      item[k] = k < keff ? (t0 + k) * TPW + team.team : N;
       // Sequential section (master only): read the loop bounds ...
       int64_t b0 = 0, l0 = 0;
       if (team.is_master() && item[k] < N) {
@@ -197,9 +197,9 @@ static int launch_ragged(const T* in, const int64_t* off, const T* init, T* out,
     auto kern = ragged_intra_kernel<T, Op, S, DIST>;
     constexpr int TPW = 32 / S;
     const int64_t ntiles = (N + TPW - 1) / TPW;
-    const int64_t per_cta = (kRaggedBlock / 32) * kRaggedK;
-    const int64_t grid = persistent_grid(kern, kRaggedBlock, 0, (ntiles + per_cta - 1) / per_cta);
-    kern<<<(unsigned)grid, kRaggedBlock, 0, st>>>(in, off, init, out, N);
+    int keff = 1;
+    const int64_t grid = tiled_grid(kern, kRaggedBlock, ntiles, kRaggedK, &keff);
+    kern<<<(unsigned)grid, kRaggedBlock, 0, st>>>(in, off, init, out, N, keff);
   } else {
     auto kern = ragged_inter_kernel<T, Op, S, DIST>;
     const int64_t grid = persistent_grid(kern, 32 * S, 0, (N + 31) / 32);

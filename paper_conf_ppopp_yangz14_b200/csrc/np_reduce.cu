@@ -51,7 +51,7 @@ __device__ __forceinline__ T redux_op(T v, unsigned mask) {
 template <class T, class Op, int S, int DIST, bool VEC, int RB = RB_SHFL>
 __global__ void __launch_bounds__(kReduceBlock)
 reduce_intra_kernel(const T* __restrict__ in, const T* __restrict__ init, T* __restrict__ out,
-                    int64_t N, int64_t L) {
+                    int64_t N, int64_t L, int keff) {
   __shared__ T slots[RB == RB_SMEM ? kReduceBlock : 1];
   constexpr int TPW = 32 / S;
   constexpr int K = kReduceK;
@@ -64,12 +64,12 @@ reduce_intra_kernel(const T* __restrict__ in, const T* __restrict__ init, T* __r
   const Range<S, DIST> r(nunits, L, VEC ? 4 : 1, team.slave);
   const int64_t ntiles = (N + TPW - 1) / TPW;
 
-  for (int64_t t0 = warp * K; t0 < ntiles; t0 += nwarps * K) {
+  for (int64_t t0 = warp * keff; t0 < ntiles; t0 += nwarps * keff) {
     int64_t item[K];
     const T* row[K];
 #pragma unroll
     for (int k = 0; k < K; ++k) {
-      item[k] = (t0 + k) * TPW + team.team;
+      item[k] = k < keff ? (t0 + k) * TPW + team.team : N;
       row[k] = in + (item[k] < N ? item[k] : 0) * L;
     }
     T part[K];
@@ -193,15 +193,15 @@ static int launch_reduce_map(const T* in, const T* init, T* out, int64_t N, int6
     auto kern = reduce_intra_kernel<T, Op, S, DIST, VEC>;
     constexpr int TPW = 32 / S;
     const int64_t ntiles = (N + TPW - 1) / TPW;
-    const int64_t per_cta = (kReduceBlock / 32) * kReduceK;
-    const int64_t grid = persistent_grid(kern, kReduceBlock, 0, (ntiles + per_cta - 1) / per_cta);
+    int keff = 1;
+    const int64_t grid = tiled_grid(kern, kReduceBlock, ntiles, kReduceK, &keff);
     if (info) {
       info->block_threads = kReduceBlock; info->grid = grid; info->map = MAP_INTRA;
       kernel_attrs(kern, &info->regs, &info->smem);
       return CUDANP_OK;
     }
     if (N == 0) return CUDANP_OK;
-    kern<<<(unsigned)grid, kReduceBlock, 0, st>>>(in, init, out, N, L);
+    kern<<<(unsigned)grid, kReduceBlock, 0, st>>>(in, init, out, N, L, keff);
   } else {
     auto kern = reduce_inter_kernel<T, Op, S, DIST, VEC>;
     const int64_t grid = persistent_grid(kern, 32 * S, 0, (N + 31) / 32);
@@ -234,8 +234,18 @@ static int dispatch_reduce_t(const void* in, const void* init, void* out, int64_
   return CUDANP_OK;
 }
 
+int reduce_multi(const void*, const void*, void*, int64_t, int64_t, int, int, int, int, bool,
+                 cudaStream_t, LaunchInfo*);
+
 int reduce_np(const void* in, const void* init, void* out, int64_t N, int64_t L, int dtype, int op,
               int S, int dist, int map, bool vec, cudaStream_t st, LaunchInfo* info) {
+  if (S > 32) {
+    if (map == MAP_INTER) {
+      set_error("a team of S > 32 is S/32 consecutive warps: intra-warp (consecutive) map only");
+      return CUDANP_ERR_UNSUPPORTED;
+    }
+    return reduce_multi(in, init, out, N, L, dtype, op, S, dist, vec, st, info);
+  }
   if (dtype == CUDANP_F32)
     return op == CUDANP_SUM
                ? dispatch_reduce_t<float, OpSum>(in, init, out, N, L, S, dist, map, vec, st, info)
@@ -253,10 +263,10 @@ static int launch_reduce_backend(const void* in, const void* init, void* out, in
     auto kern = reduce_intra_kernel<T, Op, kS, DIST_CYCLIC, true, RB>;
     constexpr int TPW = 32 / kS;
     const int64_t ntiles = (N + TPW - 1) / TPW;
-    const int64_t per_cta = (kReduceBlock / 32) * kReduceK;
-    const int64_t grid = persistent_grid(kern, kReduceBlock, 0, (ntiles + per_cta - 1) / per_cta);
+    int keff = 1;
+    const int64_t grid = tiled_grid(kern, kReduceBlock, ntiles, kReduceK, &keff);
     if (N == 0) return CUDANP_OK;
-    kern<<<(unsigned)grid, kReduceBlock, 0, st>>>((const T*)in, (const T*)init, (T*)out, N, L);
+    kern<<<(unsigned)grid, kReduceBlock, 0, st>>>((const T*)in, (const T*)init, (T*)out, N, L, keff);
     return check_launch("batched_loop_reduce_backend launch");
   });
   return CUDANP_OK;

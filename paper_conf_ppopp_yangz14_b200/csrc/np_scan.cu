@@ -45,7 +45,7 @@ __device__ __forceinline__ T sum4(V4<T> v) {
 template <class T, int S, int DIST, bool VEC>
 __global__ void __launch_bounds__(kScanBlock)
 scan_intra_kernel(const T* __restrict__ in, const T* __restrict__ init, T* __restrict__ out,
-                  int64_t N, int64_t L) {
+                  int64_t N, int64_t L, int keff) {
   constexpr int TPW = 32 / S;
   constexpr int K = kScanK;
   constexpr int V = VEC ? 4 : 1;
@@ -55,12 +55,12 @@ scan_intra_kernel(const T* __restrict__ in, const T* __restrict__ init, T* __res
   const int64_t nunits = VEC ? (L >> 2) : L;
   const int64_t ntiles = (N + TPW - 1) / TPW;
 
-  for (int64_t t0 = warp * K; t0 < ntiles; t0 += nwarps * K) {
+  for (int64_t t0 = warp * keff; t0 < ntiles; t0 += nwarps * keff) {
     int64_t item[K];
     T carry[K];
 #pragma unroll
     for (int k = 0; k < K; ++k) {
-      item[k] = (t0 + k) * TPW + team.team;
+      item[k] = k < keff ? (t0 + k) * TPW + team.team : N;
       // Sequential section: only the master touches the live-in,
       // then read_from_master hands it to the slaves.
       T c = T(0);
@@ -263,15 +263,15 @@ static int launch_scan_map(const T* in, const T* init, T* out, int64_t N, int64_
     auto kern = scan_intra_kernel<T, S, DIST, VEC>;
     constexpr int TPW = 32 / S;
     const int64_t ntiles = (N + TPW - 1) / TPW;
-    const int64_t per_cta = (kScanBlock / 32) * kScanK;
-    const int64_t grid = persistent_grid(kern, kScanBlock, 0, (ntiles + per_cta - 1) / per_cta);
+    int keff = 1;
+    const int64_t grid = tiled_grid(kern, kScanBlock, ntiles, kScanK, &keff);
     if (info) {
       info->block_threads = kScanBlock; info->grid = grid; info->map = MAP_INTRA;
       kernel_attrs(kern, &info->regs, &info->smem);
       return CUDANP_OK;
     }
     if (N == 0 || L == 0) return CUDANP_OK;
-    kern<<<(unsigned)grid, kScanBlock, 0, st>>>(in, init, out, N, L);
+    kern<<<(unsigned)grid, kScanBlock, 0, st>>>(in, init, out, N, L, keff);
   } else {
     auto kern = scan_inter_kernel<T, S, DIST, VEC>;
     const int64_t grid = persistent_grid(kern, 32 * S, 0, (N + 31) / 32);
@@ -304,8 +304,18 @@ static int dispatch_scan_t(const void* in, const void* init, void* out, int64_t 
   return CUDANP_OK;
 }
 
+int scan_multi(const void*, const void*, void*, int64_t, int64_t, int, int, int, bool, cudaStream_t,
+               LaunchInfo*);
+
 int scan_np(const void* in, const void* init, void* out, int64_t N, int64_t L, int dtype, int S,
             int dist, int map, bool vec, cudaStream_t st, LaunchInfo* info) {
+  if (S > 32) {
+    if (map == MAP_INTER) {
+      set_error("a team of S > 32 is S/32 consecutive warps: intra-warp (consecutive) map only");
+      return CUDANP_ERR_UNSUPPORTED;
+    }
+    return scan_multi(in, init, out, N, L, dtype, S, dist, vec, st, info);
+  }
   if (dtype == CUDANP_F32) return dispatch_scan_t<float>(in, init, out, N, L, S, dist, map, vec, st, info);
   return dispatch_scan_t<int32_t>(in, init, out, N, L, S, dist, map, vec, st, info);
 }

@@ -218,7 +218,7 @@ struct Redux {
 // members (they contain __syncthreads).
 template <int S>
 struct InterTeam {
-  static_assert(S >= 1 && S <= 32, "inter-warp S <= 32 (CTA = 32 x S <= 1024 threads)");
+  static_assert(S >= 1 && S <= 128, "inter-warp S <= 128 (CTA = masters x S <= 1024 threads)");
   int master, slave;
   __device__ __forceinline__ InterTeam() {
     master = threadIdx.x;

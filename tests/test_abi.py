@@ -47,7 +47,7 @@ def test_status_strings(lib):
     assert C.cudanp_version() >= 100
 
 
-@pytest.mark.parametrize("S", [0, 3, 5, 64, -1])
+@pytest.mark.parametrize("S", [0, 3, 5, 48, 2048, -1])
 def test_bad_slave_size_rejected_before_launch(lib, S):
     rc = lib.cudanp_batched_loop_reduce(None, None, None, 10, 10, 0, 0, S, 0, 0, None)
     assert rc == C.ERR_INVALID

@@ -535,3 +535,38 @@ def test_tmv_tma_full_size_C2():
         assert_rel(host(C.cudanp_tmv_tma(A, x, S=S, dist=dist))[cols], ref, n, f"C2 tma S={S} d={dist}")
     del A
     torch.cuda.empty_cache()
+
+
+# ------------------------------------------------------------------ teams larger than a warp
+BIG_S = (64, 128, 256, 512, 1024)
+
+
+def test_big_teams_parity():
+    """S > 32: S/32 consecutive warps, shfl inside each warp + shared memory
+    across them (the north star's "shared-memory fallback when S exceeds 32")."""
+    for N, L in [(1, 1), (3, 0), (7, 1000), (70, 4096), (33, 333), (300, 64)]:
+        x = synth.items(N, L, "i32_full", seed=L)
+        ini = synth.init(N, "i32_full", seed=N)
+        xs = synth.items(N, L, "i32_small", B=1 << 15, seed=L)
+        xd, inid, xsd = dev(x), dev(ini), dev(xs)
+        ref_s, ref_m = O.reduce(x, init=ini), O.reduce(x, op=O.MAX)
+        ref_scan = O.scan(xs, init=ini)
+        xf = synth.items(N, L, "f32_unit", seed=L)
+        ref_f = O.reduce(xf)
+        for S, dist in itertools.product(BIG_S, DISTS):
+            what = f"big S={S} N={N} L={L} dist={dist}"
+            assert_exact(host(C.cudanp_batched_loop_reduce(xd, inid, S=S, dist=dist)), ref_s, what)
+            assert_exact(host(C.cudanp_batched_loop_reduce(xd, op=C.MAX, S=S, dist=dist)), ref_m, what)
+            assert_exact(host(C.cudanp_batched_loop_scan(xsd, inid, S=S, dist=dist)), ref_scan, what)
+            assert_rel(host(C.cudanp_batched_loop_reduce(dev(xf), S=S, dist=dist)), ref_f, L, what)
+            with pytest.raises(C.CudanpError) as ei:
+                C.cudanp_batched_loop_reduce(xd, S=S, dist=dist, map=C.INTER_WARP)
+            assert ei.value.status == C.ERR_UNSUPPORTED
+    for h, w in [(5, 4096), (64, 1000), (300, 260), (2, 65536)]:
+        A = synth.matrix(h, w, "f32_int4", seed=w)
+        xm, xt = synth.vector(w, "f32_int4"), synth.vector(h, "f32_int4")
+        for S, dist in itertools.product(BIG_S, DISTS):
+            assert_exact(host(C.cudanp_mv(dev(A), dev(xm), S=S, dist=dist)), O.mv(A, xm), f"mv big S={S}")
+            if S <= 128:
+                assert_exact(host(C.cudanp_tmv(dev(A), dev(xt), S=S, dist=dist)), O.tmv(A, xt),
+                             f"tmv big S={S} h={h} w={w}")

@@ -343,10 +343,38 @@ def e9(Ls=(32, 64, 128)):
             torch.cuda.empty_cache()
 
 
+def big():
+    """Teams larger than a warp (S = 64..1024) on the shapes that need them:
+    MV with few long rows (the Fig 14 axis: fixed width, growing height) and a
+    batched reduce over few long items."""
+    cases = [("mv", h, 65536) for h in (16, 64, 256, 1024, 4096)] + \
+            [("reduce", N, L) for N, L in ((256, 65536), (2048, 16384), (16384, 4096))]
+    for op, N, L in cases:
+        if op == "mv":
+            A = gen((N, L), "f32_unit")
+            x = gen((L,), "f32_unit", stream_id=2)
+            y = torch.empty(N, device="cuda")
+            nb = 4 * N * L + 4 * N + 4 * L
+            fn = lambda S, d: C.cudanp_mv(A, x, y, S=S, dist=d, map=C.INTRA_WARP)  # noqa: E731
+        else:
+            A = gen((N, L), "f32_unit")
+            y = torch.empty(N, device="cuda")
+            nb = 4 * N * L + 4 * N
+            fn = lambda S, d: C.cudanp_batched_loop_reduce(A, None, y, S=S, dist=d, map=C.INTRA_WARP)  # noqa: E731
+        for S in C.SLAVE_SIZES + (64, 128, 256, 512, 1024):
+            for d in (C.CYCLIC, C.BLOCK):
+                med, mn = time_ms(lambda: fn(S, d))
+                emit({"config": "BIG", "op": op, "dtype": "f32", "N": N, "L": L, "S": S, "dist": DN[d],
+                      "map": "intra", "impl": "np", "t_median_us": round(med * 1e3, 2), "alg_bytes": nb,
+                      "gbs": round(nb / (med * 1e-3) / 1e9, 1)})
+        del A
+        torch.cuda.empty_cache()
+
+
 def main():
     global OUT
     ap = argparse.ArgumentParser()
-    ap.add_argument("--configs", default="C1,C2,C3,C4,C5,R1,F2,F3,E9")
+    ap.add_argument("--configs", default="C1,C2,C3,C4,C5,R1,F2,F3,E9,BIG")
     ap.add_argument("--out", default=os.path.join(ROOT, "gpurun_out", "sweep.jsonl"))
     ap.add_argument("--lib", default=None, help="alternative libcudanp.so (build experiments)")
     a = ap.parse_args()
@@ -356,7 +384,7 @@ def main():
     C.cudanp_dp_set_pending_launch_limit(1 << 17)
     t0 = time.time()
     for c in a.configs.split(","):
-        {"C1": c1, "C2": c2, "C3": c3, "C4": c4, "C5": c5, "R1": r1, "F2": f2, "F3": f3, "E9": e9}[c.strip()]()
+        {"C1": c1, "C2": c2, "C3": c3, "C4": c4, "C5": c5, "R1": r1, "F2": f2, "F3": f3, "E9": e9, "BIG": big}[c.strip()]()
         print(f"# {c} done at {time.time() - t0:.0f}s", file=sys.stderr, flush=True)
     print(f"# dp launch errors: {C.cudanp_dp_error_count(reset=True)}", file=sys.stderr)
 
