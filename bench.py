@@ -224,6 +224,9 @@ def run_cudanp(args):
     sweep = {"tmv": {}, "mv": {}}
     cfgs = [(S, d, m) for S in C.SLAVE_SIZES for d in (C.CYCLIC, C.BLOCK)
             for m in (C.INTRA_WARP, C.INTER_WARP)]
+    # teams larger than a warp: MV with the consecutive-warp team, TMV inter-warp S <= 128
+    big = {"tmv": [(S, d, C.INTER_WARP) for S in (64, 128) for d in (C.CYCLIC, C.BLOCK)],
+           "mv": [(S, d, C.INTRA_WARP) for S in (64, 128, 256, 512, 1024) for d in (C.CYCLIC, C.BLOCK)]}
     if args.no_sweep:
         def parse_cfg(s):
             S, d, m = s.split(",")
@@ -231,7 +234,7 @@ def run_cudanp(args):
                     {"intra": C.INTRA_WARP, "inter": C.INTER_WARP}[m])
         cfg_of = {"tmv": [parse_cfg(args.tmv_cfg)], "mv": [parse_cfg(args.mv_cfg)]}
     else:
-        cfg_of = {"tmv": cfgs, "mv": cfgs}
+        cfg_of = {"tmv": cfgs + big["tmv"], "mv": cfgs + big["mv"]}
     for op, fn_np, nbytes in (("tmv", lambda S, d, m: C.cudanp_tmv(A_t, x_t, y_t, S=S, dist=d, map=m), bytes_t),
                               ("mv", lambda S, d, m: C.cudanp_mv(A_m, x_m, y_m, S=S, dist=d, map=m), bytes_m)):
         for (S, d, m) in cfg_of[op]:
@@ -377,7 +380,7 @@ def run_cudanp(args):
     per_S = {}
     for op, nb in (("tmv", bytes_t), ("mv", bytes_m)):
         s1 = best_s1(op)
-        for S in C.SLAVE_SIZES:
+        for S in C.SLAVE_SIZES + (64, 128, 256, 512, 1024):
             cand = {k: v for k, v in sweep[op].items() if k[0] == S}
             if not cand:
                 continue
