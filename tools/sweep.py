@@ -138,6 +138,12 @@ def c1():
     for impl, name in ((C.DP_BLOCK, "dp_block"), (C.DP_THREAD, "dp_thread")):
         comps.append((name, time_ms(lambda: C.cudanp_tmv_variant(impl, As[0], x, ys[0]), reps=5)[0]))
     sweep_np("C1", "tmv", nb, run, {"dtype": "f32", "N": n, "L": n}, literal=lit, comps=comps)
+    for S in (64, 128):  # teams larger than a warp (inter-warp, 8 masters per CTA)
+        for d in (C.CYCLIC, C.BLOCK):
+            med, mn = run(S, d, C.INTER_WARP)
+            emit({"config": "C1", "op": "tmv_bigS", "dtype": "f32", "N": n, "L": n, "S": S, "dist": DN[d],
+                  "map": "inter", "impl": "np", "t_median_us": round(med * 1e3, 2), "alg_bytes": nb,
+                  "gbs": round(nb / (med * 1e-3) / 1e9, 1)})
 
 
 def c2():
