@@ -49,7 +49,6 @@ void set_error(const char* fmt, ...) {
   vsnprintf(g_err, sizeof(g_err), fmt, ap);
   va_end(ap);
 }
-void clear_error() { g_err[0] = 0; }
 
 int sm_count() {
   static int cache[64] = {0};

@@ -12,7 +12,6 @@ namespace cudanp {
 
 // Thread-local detail for cudanp_last_error().
 void set_error(const char* fmt, ...);
-void clear_error();
 
 inline int fail_invalid(const char* what) {
   set_error("invalid argument: %s", what);

@@ -211,11 +211,12 @@ struct Redux {
 };
 
 // ---------------------------------------------------------------- inter-warp team
-// blockDim = (32, S): master = threadIdx.x (one per lane), slave =
-// threadIdx.y (one per warp).  A master's slaves sit in S
-// different warps, so every exchange goes through shared memory plus a
-// CTA barrier.  All CTA threads must call the collective
-// members (they contain __syncthreads).
+// blockDim = (MX, S): master = threadIdx.x, slave = threadIdx.y.
+// With MX = 32 masters a master's slaves sit in S different warps; the
+// narrow-matrix TMV uses MX = 8 (4 slaves of 8 masters per warp, S <= 128).
+// Every exchange goes through shared memory plus a CTA barrier (P:203,
+// P:209).  All CTA threads must call the collective members (they contain
+// __syncthreads).
 template <int S>
 struct InterTeam {
   static_assert(S >= 1 && S <= 128, "inter-warp S <= 128 (CTA = masters x S <= 1024 threads)");
