@@ -148,8 +148,8 @@ ragged_inter_kernel(const T* __restrict__ in, const int64_t* __restrict__ off,
       l0 = off[item + 1] - b0;
       if (l0 < 0) l0 = 0;
     }
-    const int64_t b = team.read_from_master(b0, slot_b);
-    const int64_t len = team.read_from_master(l0, slot_l);
+    team.read_from_master(b0, l0, slot_b, slot_l);
+    const int64_t b = b0, len = l0;
     const SegShare<T, S, DIST> sh(in, b, len, team.slave);
     T pv = id;
     for (int i = team.slave; i < sh.head; i += S) pv = Op::apply(pv, in[b + i]);
@@ -157,8 +157,15 @@ ragged_inter_kernel(const T* __restrict__ in, const int64_t* __restrict__ off,
     for (int i = team.slave; i < sh.tail; i += S) pv = Op::apply(pv, tl[i]);
     V4<T> acc = {id, id, id, id};
     const T* q = sh.body;
-#pragma unroll 4
-    for (int c = 0; c < sh.cnt; ++c, q += sh.step) acc = op4r<T, Op>(acc, ldg4(q));
+    int c = 0;
+    for (; c + 4 <= sh.cnt; c += 4, q += 4 * sh.step) {  // 4 loads in flight, then fold
+      V4<T> v[4];
+#pragma unroll
+      for (int j = 0; j < 4; ++j) v[j] = ldg4(q + j * sh.step);
+#pragma unroll
+      for (int j = 0; j < 4; ++j) acc = op4r<T, Op>(acc, v[j]);
+    }
+    for (; c < sh.cnt; ++c, q += sh.step) acc = op4r<T, Op>(acc, ldg4(q));
     pv = Op::apply(pv, Op::apply(Op::apply(acc.x, acc.y), Op::apply(acc.z, acc.w)));
     if (S == 1) {
       if (ok) out[item] = init ? Op::apply(init[item], pv) : pv;

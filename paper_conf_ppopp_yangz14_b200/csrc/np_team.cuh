@@ -237,6 +237,16 @@ struct InterTeam {
     __syncthreads();
     return r;
   }
+  // Two live-ins broadcast under one pair of barriers.
+  template <class T>
+  __device__ __forceinline__ void read_from_master(T& a, T& b, T* slot_a, T* slot_b) const {
+    if (S == 1) return;
+    if (slave == 0) { slot_a[master] = a; slot_b[master] = b; }
+    __syncthreads();
+    a = slot_a[master];
+    b = slot_b[master];
+    __syncthreads();
+  }
 };
 
 }  // namespace cudanp

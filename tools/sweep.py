@@ -248,12 +248,13 @@ def c5():
     torch.cuda.empty_cache()
 
 
-def r1(means=(16, 64, 256)):
+def r1(means=(16, 64, 256, 1024)):
     """f1: ragged CSR segments, N = 4M items, uniform and exponential lengths."""
     import synth
     N = 1 << 22
-    for mean in means:
-        for dist in ("uniform", "exp"):
+    cases = [(N, m, d) for m in means for d in ("uniform", "exp")] + [(1 << 15, 8192, "exp")]
+    for N, mean, dist in cases:
+        if True:
             off = torch.from_numpy(synth.offsets_from_lengths(synth.lengths(N, mean, dist))).cuda()
             total = int(off[-1].item())
             x = gen((total,), "f32_unit")
