@@ -144,15 +144,30 @@ reduce_inter_kernel(const T* __restrict__ in, const T* __restrict__ init, T* __r
       const T id = Op::template identity<T>();
       V4<T> acc = {id, id, id, id};
       if (ok) {
-#pragma unroll 4
-        for (int64_t u = r.begin; u < r.end; u += r.step) acc = op4<T, Op>(acc, ldg4(row + 4 * u));
+        // 4 loads in flight before the fold (the same batching as tmv_rows)
+        int64_t u = r.begin;
+        for (; u + 3 * r.step < r.end; u += 4 * r.step) {
+          V4<T> v[4];
+#pragma unroll
+          for (int j = 0; j < 4; ++j) v[j] = ldg4(row + 4 * (u + j * r.step));
+#pragma unroll
+          for (int j = 0; j < 4; ++j) acc = op4<T, Op>(acc, v[j]);
+        }
+        for (; u < r.end; u += r.step) acc = op4<T, Op>(acc, ldg4(row + 4 * u));
       }
       part = fold4<T, Op>(acc);
     } else {
       part = Op::template identity<T>();
       if (ok) {
-#pragma unroll 4
-        for (int64_t u = r.begin; u < r.end; u += r.step) part = Op::apply(part, ldg1(row + u));
+        int64_t u = r.begin;
+        for (; u + 3 * r.step < r.end; u += 4 * r.step) {
+          T v[4];
+#pragma unroll
+          for (int j = 0; j < 4; ++j) v[j] = ldg1(row + u + j * r.step);
+#pragma unroll
+          for (int j = 0; j < 4; ++j) part = Op::apply(part, v[j]);
+        }
+        for (; u < r.end; u += r.step) part = Op::apply(part, ldg1(row + u));
       }
     }
     if (S == 1) {
