@@ -174,6 +174,15 @@ def tma_sweep(cfg, A, x, y, n):
                   "alg_bytes": nb, "gbs": round(nb / (med * 1e-3) / 1e9, 1)})
 
 
+def dp_thread_time(full, prefix, N, Np=65536):
+    """DP with one child launch per item, timed on a 65,536-item prefix and
+    scaled (SURVEY §8(d) DP budget rule).  A full-size attempt (2M-4M device
+    launches) did not finish within 20 minutes on B200, so it is not tried."""
+    C.cudanp_dp_error_count(reset=True)
+    tp = time_ms(prefix, reps=3, warm=1)[0]
+    return f"dp_thread_prefix{Np}_scaled", tp * N / Np
+
+
 def c3(Ls=(32, 64, 128, 256, 80, 150)):
     N = 1 << 22
     for L in Ls:
@@ -187,11 +196,12 @@ def c3(Ls=(32, 64, 128, 256, 80, 150)):
             lit = time_ms(lambda: C.cudanp_batched_loop_reduce_variant(C.S1_LITERAL, x, None, out, op=op))[0]
             comps = [("s1_literal", lit),
                      ("dp_block", time_ms(lambda: C.cudanp_batched_loop_reduce_variant(C.DP_BLOCK, x, None, out, op=op), reps=3, warm=1)[0])]
-            # DP per thread: one device launch per item -> measured on a 65,536-item prefix
+            # DP per thread: one device launch per item (full size if the runtime takes it)
             Np = 65536
             xp, op_ = x[:Np], out[:Np]
-            tp = time_ms(lambda: C.cudanp_batched_loop_reduce_variant(C.DP_THREAD, xp, None, op_, op=op), reps=3, warm=1)[0]
-            comps.append(("dp_thread_prefix65536_scaled", tp * N / Np))
+            comps.append(dp_thread_time(
+                lambda: C.cudanp_batched_loop_reduce_variant(C.DP_THREAD, x, None, out, op=op),
+                lambda: C.cudanp_batched_loop_reduce_variant(C.DP_THREAD, xp, None, op_, op=op), N, Np))
             sweep_np("C3", "reduce", nb,
                      lambda S, d, m: time_ms(lambda: C.cudanp_batched_loop_reduce(x, None, out, op=op, S=S, dist=d, map=m)),
                      {"dtype": "f32" if dtype == C.F32 else "i32", "opname": "sum" if op == C.SUM else "max",
@@ -212,8 +222,9 @@ def c4(Ls=(64, 128, 256, 512, 1024)):
                      ("dp_block", time_ms(lambda: C.cudanp_batched_loop_scan_variant(C.DP_BLOCK, x, None, out), reps=3, warm=1)[0])]
             Np = 65536
             xp, op_ = x[:Np], out[:Np]
-            tp = time_ms(lambda: C.cudanp_batched_loop_scan_variant(C.DP_THREAD, xp, None, op_), reps=3, warm=1)[0]
-            comps.append(("dp_thread_prefix65536_scaled", tp * N / Np))
+            comps.append(dp_thread_time(
+                lambda: C.cudanp_batched_loop_scan_variant(C.DP_THREAD, x, None, out),
+                lambda: C.cudanp_batched_loop_scan_variant(C.DP_THREAD, xp, None, op_), N, Np))
             sweep_np("C4", "scan", nb,
                      lambda S, d, m: time_ms(lambda: C.cudanp_batched_loop_scan(x, None, out, S=S, dist=d, map=m), reps=3),
                      {"dtype": "f32" if dtype == C.F32 else "i32", "N": N, "L": L}, literal=lit, comps=comps)
