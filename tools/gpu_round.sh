@@ -14,6 +14,9 @@ timeout 1500 python tools/sweep.py --out $O/sweep_$TAG.jsonl > $O/sweep_$TAG.log
 TCFG=$(python -c "import json;d=json.load(open('$O/bench_$TAG.json'));c=d['config']['tmv'];print(f\"{c['S']},{c['dist']},{c['map']}\")" 2>/dev/null || echo 32,block,inter)
 MCFG=$(python -c "import json;d=json.load(open('$O/bench_$TAG.json'));c=d['config']['mv'];print(f\"{c['S']},{c['dist']},{c['map']}\")" 2>/dev/null || echo 32,cyclic,intra)
 echo "TCFG=$TCFG MCFG=$MCFG" > $O/cfg_$TAG.txt
+# the launch list of the driver's own command (default `python bench.py`), and of the timed
+# step alone (--no-sweep: the two kernels of the step and the input generator)
+timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $O/launches_full_$TAG.csv python bench.py > $O/bench_ncu_full_$TAG.log 2>&1
 timeout 300 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $O/launches_$TAG.csv python bench.py --steps 5 --warmup 2 --no-cpu-baseline --e2e-steps 0 --no-sweep --tmv-cfg $TCFG --mv-cfg $MCFG > $O/bench_ncu_$TAG.log 2>&1
 IFS=, read TS TD TM <<< "$TCFG"
 IFS=, read MS MD MM <<< "$MCFG"

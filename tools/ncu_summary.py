@@ -118,6 +118,21 @@ def main():
                                "dram_read": rb, "dram_write": wb, "source": os.path.basename(rep)}
                 md.append(f"| DRAM read+write per launch | {rb + wb:.4g} B |")
             md.append("")
+    fpath = os.path.join(a.dir, f"launches_full_{a.tag}.csv")
+    if os.path.exists(fpath):
+        ls = launches(fpath)
+        tot = sum(t for _, t in ls) or 1
+        agg = {}
+        for k, t in ls:
+            short = k.split("(")[0]
+            c, s_ = agg.get(short, (0, 0.0))
+            agg[short] = (c + 1, s_ + t)
+        md += ["## Launch list of the driver's command `python bench.py` (ncu gpu__time_duration, "
+               "--clock-control none; includes the autotune sweep, comparison kernels and e2e steps)", "",
+               "| kernel | launches | total µs | share |", "|---|---|---|---|"]
+        for k, (c, s_) in sorted(agg.items(), key=lambda kv: -kv[1][1])[:25]:
+            md.append(f"| `{k}` | {c} | {s_ / 1e3:.1f} | {100 * s_ / tot:.1f} % |")
+        md.append("")
     lpath = os.path.join(a.dir, f"launches_{a.tag}.csv")
     if os.path.exists(lpath):
         ls = launches(lpath)
