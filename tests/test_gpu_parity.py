@@ -570,3 +570,22 @@ def test_big_teams_parity():
             if S <= 128:
                 assert_exact(host(C.cudanp_tmv(dev(A), dev(xt), S=S, dist=dist)), O.tmv(A, xt),
                              f"tmv big S={S} h={h} w={w}")
+
+
+def test_launch_info_and_auto_map():
+    """cudanp_launch_info reports the instantiation a call would launch; MAP_AUTO
+    resolves per P:340-342 (TMV -> inter-warp, MV/reduce/scan -> intra-warp)."""
+    for op, auto in (("tmv", "inter_warp"), ("mv", "intra_warp"), ("reduce", "intra_warp"),
+                     ("scan", "intra_warp")):
+        for S in SS:
+            i = C.cudanp_launch_info(op, 1 << 14, 1 << 10, dtype=C.F32 if op != "scan" else C.I32, S=S)
+            assert i["map"] == auto, (op, S, i)
+            assert i["block_threads"] > 0 and i["grid_ctas"] > 0 and i["regs_per_thread"] > 0
+            assert i["block_threads"] <= 1024
+        for m in (C.INTRA_WARP, C.INTER_WARP):
+            i = C.cudanp_launch_info(op, 1000, 64, S=8, map=m)
+            assert i["map"] == {C.INTRA_WARP: "intra_warp", C.INTER_WARP: "inter_warp"}[m]
+    # inter-warp CTA = masters x S (P:178-180); big teams are S/32 warps of one CTA
+    assert C.cudanp_launch_info("reduce", 1000, 64, S=8, map=C.INTER_WARP)["block_threads"] == 32 * 8
+    assert C.cudanp_launch_info("reduce", 1000, 64, S=512)["block_threads"] == 512
+    assert C.cudanp_launch_info("mv", 1000, 4096, S=1024)["block_threads"] == 1024
