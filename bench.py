@@ -171,6 +171,17 @@ def max_over_ranks(v: float, world: int) -> float:
     return float(t.item())
 
 
+def max_over_ranks_list(vals, world: int):
+    if world == 1:
+        return list(vals)
+    import torch
+    import torch.distributed as dist
+    dev = "cuda" if dist.get_backend() == "nccl" else "cpu"
+    t = torch.tensor(vals, dtype=torch.float64, device=dev)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return t.tolist()
+
+
 # ------------------------------------------------------------------ cudanp arm
 def alg_bytes_matvec(h, w):
     # A once, x once, y once
@@ -220,27 +231,26 @@ def run_cudanp(args):
     bytes_t = alg_bytes_matvec(n, wt)
     bytes_m = alg_bytes_matvec(hm, n)
 
-    # ---- autotune sweep: every S x dist x map, per op
+    # ---- autotune: every (S, dist, map) version timed on the resident operands --
+    # the paper's exhaustive version selection, run by the
+    # library's native cudanp_autotune; max over ranks so every rank picks the same.
     sweep = {"tmv": {}, "mv": {}}
-    cfgs = [(S, d, m) for S in C.SLAVE_SIZES for d in (C.CYCLIC, C.BLOCK)
-            for m in (C.INTRA_WARP, C.INTER_WARP)]
-    # teams larger than a warp: MV with the consecutive-warp team, TMV inter-warp S <= 128
-    big = {"tmv": [(S, d, C.INTER_WARP) for S in (64, 128) for d in (C.CYCLIC, C.BLOCK)],
-           "mv": [(S, d, C.INTRA_WARP) for S in (64, 128, 256, 512, 1024) for d in (C.CYCLIC, C.BLOCK)]}
     if args.no_sweep:
         def parse_cfg(s):
             S, d, m = s.split(",")
             return (int(S), {"cyclic": C.CYCLIC, "block": C.BLOCK}[d],
                     {"intra": C.INTRA_WARP, "inter": C.INTER_WARP}[m])
-        cfg_of = {"tmv": [parse_cfg(args.tmv_cfg)], "mv": [parse_cfg(args.mv_cfg)]}
+        sweep["tmv"][parse_cfg(args.tmv_cfg)] = 1.0
+        sweep["mv"][parse_cfg(args.mv_cfg)] = 1.0
     else:
-        cfg_of = {"tmv": cfgs + big["tmv"], "mv": cfgs + big["mv"]}
-    for op, fn_np, nbytes in (("tmv", lambda S, d, m: C.cudanp_tmv(A_t, x_t, y_t, S=S, dist=d, map=m), bytes_t),
-                              ("mv", lambda S, d, m: C.cudanp_mv(A_m, x_m, y_m, S=S, dist=d, map=m), bytes_m)):
-        for (S, d, m) in cfg_of[op]:
-            ms = time_op(lambda: fn_np(S, d, m))
-            ms = max_over_ranks(ms, world)
-            sweep[op][(S, d, m)] = ms
+        for op, A_, x_, y_, h_, w_ in (("tmv", A_t, x_t, y_t, wt, n), ("mv", A_m, x_m, y_m, hm, n)):
+            _, table = C.cudanp_autotune(op, A_, x_, y_, lda=A_.shape[1], n_outer=h_, n_inner=w_,
+                                         reps=5)
+            cands = list(table)
+            vals = max_over_ranks_list([min(table[c], 1e30) for c in cands], world)
+            for cand, ms in zip(cands, vals):
+                if ms < 1e29:  # not supported for this shape
+                    sweep[op][cand] = ms
     best = {op: min(sweep[op], key=sweep[op].get) for op in sweep}
     # literal S=1 (Fig 2) and DP (per-CTA / per-thread) comparison, once each
     comp = {}

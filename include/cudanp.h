@@ -203,6 +203,24 @@ int cudanp_dp_memcopy(const float* in, float* out, int64_t total, int64_t m, int
                       void* stream);
 
 /* ------------------------------------------------------------------------
+ * Version selection (the paper's exhaustive autotune, P:384, P:413,
+ * P:484-486): op_kind 0 tmv, 1 mv, 2 reduce, 3 scan.  The candidates are the
+ * library's (S, dist, map) instantiations (S = 1..32 x cyclic/block x
+ * intra/inter, plus multi-warp teams); cudanp_autotune_count/_candidate list
+ * them.  cudanp_autotune runs each candidate once as warm-up and `reps` times
+ * under CUDA events on `stream` with the caller's operands (a = A or in,
+ * b = x or init, out = y or out; lda for tmv/mv; dtype/op for reduce, dtype
+ * for scan), writes the mean ms per launch to ms_table[i] (INFINITY for a
+ * combination this shape does not support; ms_table may be NULL) and the
+ * fastest candidate's index to *best_index.  Synchronizes `stream`.  `out` is
+ * overwritten by every candidate (the last run's result is valid). */
+int cudanp_autotune_count(int op_kind);
+int cudanp_autotune_candidate(int op_kind, int index, int* S, int* dist, int* map);
+int cudanp_autotune(int op_kind, const void* a, const void* b, void* out, int64_t lda,
+                    int64_t n_outer, int64_t n_inner, int dtype, int op, int reps,
+                    float* ms_table, int* best_index, void* stream);
+
+/* ------------------------------------------------------------------------
  * Launch shape actually used (the paper's resource analysis, Table 1 P:96,
  * and autotune space P:384): for an NP call with these arguments,
  * report the kernel's block size, grid size, registers per thread, static

@@ -52,6 +52,11 @@ _SIGS = {
     "cudanp_dp_set_pending_launch_limit": [_sz],
     "cudanp_dp_error_count": [_int, ctypes.POINTER(_i64)],
     "cudanp_dp_memcopy": [_vp, _vp, _i64, _i64, _int, _vp],
+    "cudanp_autotune_count": [_int],
+    "cudanp_autotune_candidate": [_int, _int, ctypes.POINTER(_int), ctypes.POINTER(_int),
+                                  ctypes.POINTER(_int)],
+    "cudanp_autotune": [_int, _vp, _vp, _vp, _i64, _i64, _i64, _int, _int, _int,
+                        ctypes.POINTER(ctypes.c_float), ctypes.POINTER(_int), _vp],
     "cudanp_launch_info": [_int, _i64, _i64, _int, _int, _int, _int, _int, _int,
                            ctypes.POINTER(_int), ctypes.POINTER(_i64), ctypes.POINTER(_int),
                            ctypes.POINTER(_int), ctypes.POINTER(_int)],
@@ -327,6 +332,34 @@ def cudanp_dp_memcopy(x, out=None, *, m=1, variant=2, stream=None):
     _check(load().cudanp_dp_memcopy(_ptr(x), _ptr(out), x.numel(), m, variant, _stream(stream)),
            "cudanp_dp_memcopy")
     return out
+
+
+OP_KINDS = {"tmv": 0, "mv": 1, "reduce": 2, "scan": 3}
+
+
+def cudanp_autotune_candidates(op_kind: str) -> list[tuple[int, int, int]]:
+    L = load()
+    k = OP_KINDS[op_kind]
+    out = []
+    for i in range(L.cudanp_autotune_count(k)):
+        S, d, m = _int(), _int(), _int()
+        _check(L.cudanp_autotune_candidate(k, i, ctypes.byref(S), ctypes.byref(d), ctypes.byref(m)),
+               "cudanp_autotune_candidate")
+        out.append((S.value, d.value, m.value))
+    return out
+
+
+def cudanp_autotune(op_kind: str, a, b, out, *, lda=0, n_outer, n_inner, dtype=F32, op=SUM,
+                    reps=5, stream=None):
+    """Time every (S, dist, map) candidate on these operands.
+    Returns (best (S, dist, map), {candidate: ms})."""
+    k = OP_KINDS[op_kind]
+    cands = cudanp_autotune_candidates(op_kind)
+    table = (ctypes.c_float * len(cands))()
+    best = _int()
+    _check(load().cudanp_autotune(k, _ptr(a), _ptr(b), _ptr(out), lda, n_outer, n_inner, dtype, op,
+                                  reps, table, ctypes.byref(best), _stream(stream)), "cudanp_autotune")
+    return cands[best.value], {c: table[i] for i, c in enumerate(cands)}
 
 
 # ---------------------------------------------------------------- support

@@ -589,3 +589,32 @@ def test_launch_info_and_auto_map():
     assert C.cudanp_launch_info("reduce", 1000, 64, S=8, map=C.INTER_WARP)["block_threads"] == 32 * 8
     assert C.cudanp_launch_info("reduce", 1000, 64, S=512)["block_threads"] == 512
     assert C.cudanp_launch_info("mv", 1000, 4096, S=1024)["block_threads"] == 1024
+
+
+def test_autotune_picks_a_valid_fastest_version():
+    # the paper's exhaustive version selection, run by the library
+    A = torch.empty(2048, 2048, device="cuda")
+    C.cudanp_generate(A, "f32_int4")
+    x = torch.empty(2048, device="cuda")
+    C.cudanp_generate(x, "f32_int4", stream_id=2)
+    y = torch.empty(2048, device="cuda")
+    tables = {}
+    for op in ("tmv", "mv"):
+        best, table = C.cudanp_autotune(op, A, x, y, lda=2048, n_outer=2048, n_inner=2048, reps=2)
+        tables[op] = table
+        finite = {k: v for k, v in table.items() if v != float("inf")}
+        assert best in finite and finite[best] == min(finite.values())
+        assert len(finite) >= 24
+        S, d, m = best
+        fn = C.cudanp_tmv if op == "tmv" else C.cudanp_mv
+        ref = (O.tmv if op == "tmv" else O.mv)(host(A), host(x))
+        assert_exact(host(fn(A, x, S=S, dist=d, map=m)), ref, f"autotuned {op} {best}")
+    X = torch.empty(4096, 96, dtype=torch.int32, device="cuda")
+    C.cudanp_generate(X, "i32_full")
+    out = torch.empty(4096, dtype=torch.int32, device="cuda")
+    best, table = C.cudanp_autotune("reduce", X, None, out, n_outer=4096, n_inner=96, dtype=C.I32, reps=2)
+    assert_exact(host(out), O.reduce(host(X)), "autotune reduce: last run result")
+    assert table[(64, C.CYCLIC, C.INTRA_WARP)] != float("inf")  # multi-warp reduce team
+    # TMV's candidate list only holds the built combinations (inter-warp for S > 32)
+    assert (64, C.CYCLIC, C.INTRA_WARP) not in tables["tmv"]
+    assert tables["tmv"][(64, C.CYCLIC, C.INTER_WARP)] != float("inf")
