@@ -57,20 +57,15 @@ inline int64_t persistent_grid(K kernel, int block_threads, size_t dyn_smem, int
   return work_ctas < cap ? work_ctas : cap;
 }
 
-// Persistent intra-warp launch where each warp takes K consecutive warp tiles
-// per step: returns the grid and the effective tiles per step `keff` -- K
-// for large problems, fewer when there are not enough tiles to give every
-// resident warp K of them (so few-item launches still use every SM).
+// Persistent intra-warp launches take K consecutive warp tiles per warp step
+// (K tiles of loads in flight).  When there are too few tiles to give every
+// resident warp K of them, the K = 1 instantiation is launched instead so a
+// few-item launch still spreads over every SM (a compile-time K keeps the
+// register count, and so the occupancy, of the common case).
 template <class Kn>
-inline int64_t tiled_grid(Kn kernel, int block_threads, int64_t ntiles, int K, int* keff) {
-  const int64_t cap_ctas = persistent_grid(kernel, block_threads, 0, INT64_MAX / 4);
-  const int64_t warps = cap_ctas * (block_threads / 32);
-  int64_t k = (ntiles + warps - 1) / warps;
-  if (k < 1) k = 1;
-  if (k > K) k = K;
-  *keff = (int)k;
-  const int64_t per_cta = (block_threads / 32) * k;
-  return persistent_grid(kernel, block_threads, 0, (ntiles + per_cta - 1) / per_cta);
+inline bool few_tiles(Kn kernel_k, int block_threads, int64_t ntiles, int K) {
+  const int64_t cap_ctas = persistent_grid(kernel_k, block_threads, 0, INT64_MAX / 4);
+  return 2 * ntiles < cap_ctas * (block_threads / 32) * K;
 }
 
 template <class K>

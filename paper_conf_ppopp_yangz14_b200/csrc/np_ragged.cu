@@ -60,19 +60,19 @@ struct SegShare {
 };
 
 // ---------------------------------------------------------------- intra-warp
-template <class T, class Op, int S, int DIST>
+template <class T, class Op, int S, int DIST, int KT = kRaggedK>
 __global__ void __launch_bounds__(kRaggedBlock)
 ragged_intra_kernel(const T* __restrict__ in, const int64_t* __restrict__ off,
-                    const T* __restrict__ init, T* __restrict__ out, int64_t N, int keff) {
+                    const T* __restrict__ init, T* __restrict__ out, int64_t N) {
   constexpr int TPW = 32 / S;
-  constexpr int K = kRaggedK;
+  constexpr int K = KT;
   const IntraTeam<S> team;
   const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
   const int64_t ntiles = (N + TPW - 1) / TPW;
   const T id = Op::template identity<T>();
 
-  for (int64_t t0 = warp * keff; t0 < ntiles; t0 += nwarps * keff) {
+  for (int64_t t0 = warp * K; t0 < ntiles; t0 += nwarps * K) {
     int64_t item[K];
     const T* p[K];
     int64_t pstep[K];
@@ -81,7 +81,7 @@ ragged_intra_kernel(const T* __restrict__ in, const int64_t* __restrict__ off,
     int trips = 0;
 #pragma unroll
     for (int k = 0; k < K; ++k) {
-      item[k] = k < keff ? (t0 + k) * TPW + team.team : N;
+      item[k] = (t0 + k) * TPW + team.team;
       // Sequential section (master only): read the loop bounds ...
       int64_t b0 = 0, l0 = 0;
       if (team.is_master() && item[k] < N) {
@@ -201,12 +201,13 @@ static int launch_ragged(const T* in, const int64_t* off, const T* init, T* out,
                          cudaStream_t st) {
   if (N == 0) return CUDANP_OK;
   if (map == MAP_INTRA) {
-    auto kern = ragged_intra_kernel<T, Op, S, DIST>;
     constexpr int TPW = 32 / S;
     const int64_t ntiles = (N + TPW - 1) / TPW;
-    int keff = 1;
-    const int64_t grid = tiled_grid(kern, kRaggedBlock, ntiles, kRaggedK, &keff);
-    kern<<<(unsigned)grid, kRaggedBlock, 0, st>>>(in, off, init, out, N, keff);
+    const bool few = few_tiles(ragged_intra_kernel<T, Op, S, DIST>, kRaggedBlock, ntiles, kRaggedK);
+    auto kern = few ? ragged_intra_kernel<T, Op, S, DIST, 1> : ragged_intra_kernel<T, Op, S, DIST, kRaggedK>;
+    const int64_t per_cta = (kRaggedBlock / 32) * (few ? 1 : kRaggedK);
+    const int64_t grid = persistent_grid(kern, kRaggedBlock, 0, (ntiles + per_cta - 1) / per_cta);
+    kern<<<(unsigned)grid, kRaggedBlock, 0, st>>>(in, off, init, out, N);
   } else {
     auto kern = ragged_inter_kernel<T, Op, S, DIST>;
     const int64_t grid = persistent_grid(kern, 32 * S, 0, (N + 31) / 32);

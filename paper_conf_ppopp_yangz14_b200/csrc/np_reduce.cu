@@ -48,13 +48,13 @@ __device__ __forceinline__ T redux_op(T v, unsigned mask) {
 // Team = S lanes; a warp holds TPW = 32/S teams = TPW items ("warp tile").
 // Each warp processes K consecutive warp tiles per step of a grid-stride
 // loop, so a lane has K independent rows in flight.
-template <class T, class Op, int S, int DIST, bool VEC, int RB = RB_SHFL>
+template <class T, class Op, int S, int DIST, bool VEC, int RB = RB_SHFL, int KT = kReduceK>
 __global__ void __launch_bounds__(kReduceBlock)
 reduce_intra_kernel(const T* __restrict__ in, const T* __restrict__ init, T* __restrict__ out,
-                    int64_t N, int64_t L, int keff) {
+                    int64_t N, int64_t L) {
   __shared__ T slots[RB == RB_SMEM ? kReduceBlock : 1];
   constexpr int TPW = 32 / S;
-  constexpr int K = kReduceK;
+  constexpr int K = KT;
   const IntraTeam<S> team;
   const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
@@ -64,12 +64,12 @@ reduce_intra_kernel(const T* __restrict__ in, const T* __restrict__ init, T* __r
   const Range<S, DIST> r(nunits, L, VEC ? 4 : 1, team.slave);
   const int64_t ntiles = (N + TPW - 1) / TPW;
 
-  for (int64_t t0 = warp * keff; t0 < ntiles; t0 += nwarps * keff) {
+  for (int64_t t0 = warp * K; t0 < ntiles; t0 += nwarps * K) {
     int64_t item[K];
     const T* row[K];
 #pragma unroll
     for (int k = 0; k < K; ++k) {
-      item[k] = k < keff ? (t0 + k) * TPW + team.team : N;
+      item[k] = (t0 + k) * TPW + team.team;
       row[k] = in + (item[k] < N ? item[k] : 0) * L;
     }
     T part[K];
@@ -205,18 +205,20 @@ template <class T, class Op, int S, int DIST, bool VEC>
 static int launch_reduce_map(const T* in, const T* init, T* out, int64_t N, int64_t L, int map,
                              cudaStream_t st, LaunchInfo* info) {
   if (map == MAP_INTRA) {
-    auto kern = reduce_intra_kernel<T, Op, S, DIST, VEC>;
     constexpr int TPW = 32 / S;
     const int64_t ntiles = (N + TPW - 1) / TPW;
-    int keff = 1;
-    const int64_t grid = tiled_grid(kern, kReduceBlock, ntiles, kReduceK, &keff);
+    const bool few = few_tiles(reduce_intra_kernel<T, Op, S, DIST, VEC>, kReduceBlock, ntiles, kReduceK);
+    auto kern = few ? reduce_intra_kernel<T, Op, S, DIST, VEC, RB_SHFL, 1>
+                    : reduce_intra_kernel<T, Op, S, DIST, VEC, RB_SHFL, kReduceK>;
+    const int64_t per_cta = (kReduceBlock / 32) * (few ? 1 : kReduceK);
+    const int64_t grid = persistent_grid(kern, kReduceBlock, 0, (ntiles + per_cta - 1) / per_cta);
     if (info) {
       info->block_threads = kReduceBlock; info->grid = grid; info->map = MAP_INTRA;
       kernel_attrs(kern, &info->regs, &info->smem);
       return CUDANP_OK;
     }
     if (N == 0) return CUDANP_OK;
-    kern<<<(unsigned)grid, kReduceBlock, 0, st>>>(in, init, out, N, L, keff);
+    kern<<<(unsigned)grid, kReduceBlock, 0, st>>>(in, init, out, N, L);
   } else {
     auto kern = reduce_inter_kernel<T, Op, S, DIST, VEC>;
     const int64_t grid = persistent_grid(kern, 32 * S, 0, (N + 31) / 32);
@@ -278,10 +280,10 @@ static int launch_reduce_backend(const void* in, const void* init, void* out, in
     auto kern = reduce_intra_kernel<T, Op, kS, DIST_CYCLIC, true, RB>;
     constexpr int TPW = 32 / kS;
     const int64_t ntiles = (N + TPW - 1) / TPW;
-    int keff = 1;
-    const int64_t grid = tiled_grid(kern, kReduceBlock, ntiles, kReduceK, &keff);
+    const int64_t per_cta = (kReduceBlock / 32) * kReduceK;
+    const int64_t grid = persistent_grid(kern, kReduceBlock, 0, (ntiles + per_cta - 1) / per_cta);
     if (N == 0) return CUDANP_OK;
-    kern<<<(unsigned)grid, kReduceBlock, 0, st>>>((const T*)in, (const T*)init, (T*)out, N, L, keff);
+    kern<<<(unsigned)grid, kReduceBlock, 0, st>>>((const T*)in, (const T*)init, (T*)out, N, L);
     return check_launch("batched_loop_reduce_backend launch");
   });
   return CUDANP_OK;

@@ -42,12 +42,12 @@ __device__ __forceinline__ T sum4(V4<T> v) {
 }
 
 // ---------------------------------------------------------------- intra-warp
-template <class T, int S, int DIST, bool VEC>
+template <class T, int S, int DIST, bool VEC, int KT = kScanK>
 __global__ void __launch_bounds__(kScanBlock)
 scan_intra_kernel(const T* __restrict__ in, const T* __restrict__ init, T* __restrict__ out,
-                  int64_t N, int64_t L, int keff) {
+                  int64_t N, int64_t L) {
   constexpr int TPW = 32 / S;
-  constexpr int K = kScanK;
+  constexpr int K = KT;
   constexpr int V = VEC ? 4 : 1;
   const IntraTeam<S> team;
   const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
@@ -55,12 +55,12 @@ scan_intra_kernel(const T* __restrict__ in, const T* __restrict__ init, T* __res
   const int64_t nunits = VEC ? (L >> 2) : L;
   const int64_t ntiles = (N + TPW - 1) / TPW;
 
-  for (int64_t t0 = warp * keff; t0 < ntiles; t0 += nwarps * keff) {
+  for (int64_t t0 = warp * K; t0 < ntiles; t0 += nwarps * K) {
     int64_t item[K];
     T carry[K];
 #pragma unroll
     for (int k = 0; k < K; ++k) {
-      item[k] = k < keff ? (t0 + k) * TPW + team.team : N;
+      item[k] = (t0 + k) * TPW + team.team;
       // Sequential section: only the master touches the live-in,
       // then read_from_master hands it to the slaves.
       T c = T(0);
@@ -260,18 +260,19 @@ template <class T, int S, int DIST, bool VEC>
 static int launch_scan_map(const T* in, const T* init, T* out, int64_t N, int64_t L, int map,
                            cudaStream_t st, LaunchInfo* info) {
   if (map == MAP_INTRA) {
-    auto kern = scan_intra_kernel<T, S, DIST, VEC>;
     constexpr int TPW = 32 / S;
     const int64_t ntiles = (N + TPW - 1) / TPW;
-    int keff = 1;
-    const int64_t grid = tiled_grid(kern, kScanBlock, ntiles, kScanK, &keff);
+    const bool few = few_tiles(scan_intra_kernel<T, S, DIST, VEC>, kScanBlock, ntiles, kScanK);
+    auto kern = few ? scan_intra_kernel<T, S, DIST, VEC, 1> : scan_intra_kernel<T, S, DIST, VEC, kScanK>;
+    const int64_t per_cta = (kScanBlock / 32) * (few ? 1 : kScanK);
+    const int64_t grid = persistent_grid(kern, kScanBlock, 0, (ntiles + per_cta - 1) / per_cta);
     if (info) {
       info->block_threads = kScanBlock; info->grid = grid; info->map = MAP_INTRA;
       kernel_attrs(kern, &info->regs, &info->smem);
       return CUDANP_OK;
     }
     if (N == 0 || L == 0) return CUDANP_OK;
-    kern<<<(unsigned)grid, kScanBlock, 0, st>>>(in, init, out, N, L, keff);
+    kern<<<(unsigned)grid, kScanBlock, 0, st>>>(in, init, out, N, L);
   } else {
     auto kern = scan_inter_kernel<T, S, DIST, VEC>;
     const int64_t grid = persistent_grid(kern, 32 * S, 0, (N + 31) / 32);
