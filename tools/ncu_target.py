@@ -20,7 +20,7 @@ def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--op", required=True, choices=["tmv", "mv", "reduce", "scan", "tmv_literal",
                                                     "mv_literal", "reduce_literal", "scan_literal",
-                                                    "ragged", "le"])
+                                                    "ragged", "le", "tmv_tma"])
     ap.add_argument("--lens", default="uniform", help="ragged: length distribution")
     ap.add_argument("--layout", type=int, default=0, help="le: 0 item-major, 1 point-major")
     ap.add_argument("--S", type=int, default=8)
@@ -53,6 +53,7 @@ def main():
         C.cudanp_generate(x, "f32_unit", stream_id=2)
         y = torch.empty(a.n, device="cuda")
         fns = {"tmv": lambda: C.cudanp_tmv(A, x, y, S=a.S, dist=d, map=m),
+               "tmv_tma": lambda: C.cudanp_tmv_tma(A, x, y, S=a.S, dist=d),
                "mv": lambda: C.cudanp_mv(A, x, y, S=a.S, dist=d, map=m),
                "tmv_literal": lambda: C.cudanp_tmv_variant(C.S1_LITERAL, A, x, y),
                "mv_literal": lambda: C.cudanp_mv_variant(C.S1_LITERAL, A, x, y)}
