@@ -12,7 +12,7 @@
 // slaves read their rows from shared memory.  Memory-level parallelism then
 // comes from the stages in flight, not from the number of resident threads.
 //
-//  cyclic: one box of R = kRows rows per stage; slave s owns the box rows
+//  cyclic: one box of R rows per stage (TmaShape); slave s owns the box rows
 //          k*S + s, i.e. global rows i = s (mod S) exactly as P:166.
 //  block : S boxes of R/S rows per stage, one from each slave's contiguous
 //          chunk [s*c, (s+1)*c) (c = ceil(h/S)).
@@ -24,8 +24,14 @@
 
 namespace cudanp {
 
-constexpr int kTmaRows = 32;    // rows per stage
-constexpr int kTmaStages = 8;   // ring depth per CTA
+// Rows per stage and ring depth per S.  Every consumer warp spins on the
+// stage's mbarrier, so stages must carry enough rows per slave to amortise
+// the waits (measured on C2: 32 rows x 8 stages is best for S <= 2, 128 x 4
+// for S = 4, 256 x 4 for S >= 8; box height <= 256).
+template <int S> struct TmaShape {
+  static constexpr int ROWS = S <= 2 ? 32 : (S == 4 ? 128 : 256);
+  static constexpr int STAGES = S <= 2 ? 8 : 4;
+};
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
   return (uint32_t)__cvta_generic_to_shared(p);
@@ -66,7 +72,8 @@ tmv_tma_kernel(const __grid_constant__ CUtensorMap mapA, const float* __restrict
                float* __restrict__ y, int64_t w, int64_t h) {
   constexpr int kTmaCols = COLS;
   constexpr int V = COLS / 32;
-  constexpr int R = kTmaRows;
+  constexpr int R = TmaShape<S>::ROWS;
+  constexpr int kTmaStages = TmaShape<S>::STAGES;
   constexpr int RK = R / S;  // rows per slave per stage
   static_assert(R % S == 0, "S must divide the rows per stage");
   extern __shared__ __align__(128) unsigned char smem_raw[];
@@ -202,6 +209,7 @@ static int launch_tmv_tma_s(const float* A, int64_t lda, const float* x, float* 
   CUtensorMap map;
   const cuuint64_t dims[2] = {(cuuint64_t)w, (cuuint64_t)h};
   const cuuint64_t strides[1] = {(cuuint64_t)lda * 4};
+  constexpr int kTmaRows = TmaShape<S>::ROWS, kTmaStages = TmaShape<S>::STAGES;
   const cuuint32_t box[2] = {kTmaCols, DIST == DIST_CYCLIC ? (cuuint32_t)kTmaRows : (cuuint32_t)(kTmaRows / S)};
   const cuuint32_t estr[2] = {1, 1};
   CUresult r = enc(&map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, (void*)A, dims, strides, box, estr,
