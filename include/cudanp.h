@@ -18,9 +18,9 @@
  * S = 1 means no nesting: the tuned one-thread-per-item kernel.
  * S in {64, 128, 256, 512, 1024} ("shared-memory fallback when S exceeds
  * 32"): a team of S/32 consecutive warps, shfl inside each warp and shared
- * memory across them; supported by the reduce, scan and MV calls with
- * CUDANP_MAP_AUTO / CUDANP_MAP_INTRA_WARP, and by TMV with the inter-warp
- * map for S <= 128 (CUDANP_ERR_UNSUPPORTED otherwise).
+ * memory across them; supported by the reduce, scan, MV and ragged-reduce
+ * calls with CUDANP_MAP_AUTO / CUDANP_MAP_INTRA_WARP, and by TMV with the
+ * inter-warp map for S <= 128 (CUDANP_ERR_UNSUPPORTED otherwise).
  *
  * Conventions for every call:
  *  - Data pointers are DEVICE pointers owned by the caller; the library never

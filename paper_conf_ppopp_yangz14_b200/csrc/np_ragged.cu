@@ -183,6 +183,72 @@ ragged_inter_kernel(const T* __restrict__ in, const int64_t* __restrict__ off,
   }
 }
 
+// ---------------------------------------------------------------- multi-warp team (S > 32)
+// Few, long segments: a team of S/32 consecutive warps per segment (shfl per
+// warp + shared memory across them); bounds broadcast through a shared slot.
+template <class T, class Op, int S, int DIST>
+__global__ void __launch_bounds__(MultiShape<S>::CTA, MultiShape<S>::MINB)
+ragged_multi_kernel(const T* __restrict__ in, const int64_t* __restrict__ off,
+                    const T* __restrict__ init, T* __restrict__ out, int64_t N) {
+  using Sh = MultiShape<S>;
+  __shared__ T sm[Sh::TEAMS * MultiTeam<S>::W];
+  __shared__ int64_t slot_b[Sh::TEAMS], slot_l[Sh::TEAMS];
+  const MultiTeam<S> team;
+  const int64_t ngroups = (N + Sh::TEAMS - 1) / Sh::TEAMS;
+  const T id = Op::template identity<T>();
+  for (int64_t g = blockIdx.x; g < ngroups; g += gridDim.x) {
+    const int64_t item = g * Sh::TEAMS + team.team;
+    const bool ok = item < N;
+    int64_t b0 = 0, l0 = 0;
+    if (team.is_master() && ok) {  // sequential section: the master reads the bounds
+      b0 = off[item];
+      l0 = off[item + 1] - b0;
+      if (l0 < 0) l0 = 0;
+    }
+    const int64_t b = team.read_from_master(b0, slot_b);
+    const int64_t len = team.read_from_master(l0, slot_l);
+    const SegShare<T, S, DIST> sh(in, b, len, team.slave);
+    T pv = id;
+    for (int i = team.slave; i < sh.head; i += S) pv = Op::apply(pv, in[b + i]);
+    const T* tl = in + b + sh.head + 4 * ((len - sh.head) >> 2);
+    for (int i = team.slave; i < sh.tail; i += S) pv = Op::apply(pv, tl[i]);
+    V4<T> acc = {id, id, id, id};
+    const T* q = sh.body;
+    int c = 0;
+    for (; c + 4 <= sh.cnt; c += 4, q += 4 * sh.step) {
+      V4<T> v[4];
+#pragma unroll
+      for (int j = 0; j < 4; ++j) v[j] = ldg4(q + j * sh.step);
+#pragma unroll
+      for (int j = 0; j < 4; ++j) acc = op4r<T, Op>(acc, v[j]);
+    }
+    for (; c < sh.cnt; ++c, q += sh.step) acc = op4r<T, Op>(acc, ldg4(q));
+    pv = Op::apply(pv, Op::apply(Op::apply(acc.x, acc.y), Op::apply(acc.z, acc.w)));
+    const T res = team.template reduce<Op>(pv, sm);
+    if (team.is_master() && ok) out[item] = init ? Op::apply(init[item], res) : res;
+  }
+}
+
+template <class T, class Op>
+static int launch_ragged_multi(const T* in, const int64_t* off, const T* init, T* out, int64_t N,
+                               int S, int dist, cudaStream_t st) {
+#define CUDANP_RAGGED_BIG(SV)                                                                     \
+  case SV: {                                                                                      \
+    auto kern = dist == DIST_CYCLIC ? ragged_multi_kernel<T, Op, SV, DIST_CYCLIC>                 \
+                                    : ragged_multi_kernel<T, Op, SV, DIST_BLOCK>;                 \
+    using Sh = MultiShape<SV>;                                                                    \
+    const int64_t grid = persistent_grid(kern, Sh::CTA, 0, (N + Sh::TEAMS - 1) / Sh::TEAMS);      \
+    kern<<<(unsigned)grid, Sh::CTA, 0, st>>>(in, off, init, out, N);                              \
+    return check_launch("ragged_loop_reduce (multi-warp team) launch");                          \
+  }
+  switch (S) {
+    CUDANP_RAGGED_BIG(64) CUDANP_RAGGED_BIG(128) CUDANP_RAGGED_BIG(256) CUDANP_RAGGED_BIG(512)
+    CUDANP_RAGGED_BIG(1024)
+    default: return fail_invalid("S");
+  }
+#undef CUDANP_RAGGED_BIG
+}
+
 // ---------------------------------------------------------------- S=1 literal
 template <class T, class Op>
 __global__ void __launch_bounds__(256)
@@ -222,6 +288,14 @@ static int dispatch_ragged_t(const void* in, const int64_t* off, const void* ini
   const T* i = (const T*)in;
   const T* ini = (const T*)init;
   T* o = (T*)out;
+  if (S > 32) {
+    if (map == MAP_INTER) {
+      set_error("a team of S > 32 is S/32 consecutive warps: intra-warp (consecutive) map only");
+      return CUDANP_ERR_UNSUPPORTED;
+    }
+    if (N == 0) return CUDANP_OK;
+    return launch_ragged_multi<T, Op>(i, off, ini, o, N, S, dist, st);
+  }
   CUDANP_DISPATCH_S(S, {
     return dist == DIST_CYCLIC ? launch_ragged<T, Op, kS, DIST_CYCLIC>(i, off, ini, o, N, map, st)
                                : launch_ragged<T, Op, kS, DIST_BLOCK>(i, off, ini, o, N, map, st);

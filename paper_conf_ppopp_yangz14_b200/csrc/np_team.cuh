@@ -249,4 +249,74 @@ struct InterTeam {
   }
 };
 
+// ---------------------------------------------------------------- multi-warp team
+// S > 32 ("shared-memory fallback when S exceeds 32", north star): S/32
+// consecutive warps of one CTA; shfl trees inside each warp and the
+// warp results combined through shared memory.
+template <int S>
+struct MultiTeam {
+  static_assert(S % 32 == 0 && S >= 64 && S <= 1024, "multi-warp teams: S = 64..1024");
+  static constexpr int W = S / 32;  // warps per team
+  int slave, team, lane, wit;       // wit: warp index inside the team
+  __device__ __forceinline__ MultiTeam() {
+    slave = threadIdx.x % S;
+    team = threadIdx.x / S;
+    lane = threadIdx.x & 31;
+    wit = slave >> 5;
+  }
+  __device__ __forceinline__ bool is_master() const { return slave == 0; }
+
+  // Reduction: shfl butterfly per warp, then the team's W warp results through
+  // shared memory.  Every CTA thread must call it (it holds CTA barriers);
+  // every team member returns the team's result.
+  template <class Op, class T>
+  __device__ __forceinline__ T reduce(T v, T* sm /*[teams*W]*/) const {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v = Op::apply(v, __shfl_xor_sync(kFull, v, o));
+    if (lane == 0) sm[team * W + wit] = v;
+    __syncthreads();
+    T r = sm[team * W];
+#pragma unroll 4
+    for (int k = 1; k < W; ++k) r = Op::apply(r, sm[team * W + k]);
+    __syncthreads();
+    return r;
+  }
+  // Inclusive scan over the S team threads; *total = the team's sum.
+  template <class T>
+  __device__ __forceinline__ T inclusive_scan(T v, T* sm /*[teams*W]*/, T* total) const {
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const T t = __shfl_up_sync(kFull, v, o);
+      if (lane >= o) v = OpSum::apply(v, t);
+    }
+    if (lane == 31) sm[team * W + wit] = v;
+    __syncthreads();
+    T off = T(0), tot = T(0);
+#pragma unroll 4
+    for (int k = 0; k < W; ++k) {
+      const T p = sm[team * W + k];
+      if (k < wit) off = OpSum::apply(off, p);
+      tot = OpSum::apply(tot, p);
+    }
+    __syncthreads();
+    *total = tot;
+    return OpSum::apply(off, v);
+  }
+  // read_from_master through a per-team shared slot.
+  template <class T>
+  __device__ __forceinline__ T read_from_master(T v, T* slot /*[teams]*/) const {
+    if (slave == 0) slot[team] = v;
+    __syncthreads();
+    const T r = slot[team];
+    __syncthreads();
+    return r;
+  }
+};
+
+template <int S> struct MultiShape {
+  static constexpr int CTA = S < 256 ? 256 : S;  // threads per CTA
+  static constexpr int TEAMS = CTA / S;          // teams (items) per CTA
+  static constexpr int MINB = 1024 / CTA;        // CTAs per SM -> 64 registers/thread
+};
+
 }  // namespace cudanp

@@ -82,3 +82,20 @@ def test_ragged_full_size_sampled():
     for S, d in itertools.product(SS, (C.CYCLIC, C.BLOCK)):
         got = host(C.cudanp_ragged_loop_reduce(x, od, S=S, dist=d, map=C.INTRA_WARP))
         assert_exact(got[items], ref, f"full ragged S={S} d={d}")
+
+
+def test_ragged_big_teams():
+    """S > 32 multi-warp teams on few, long segments."""
+    for N, mean in [(1, 5000), (37, 3000), (300, 700)]:
+        lens = synth.lengths(N, mean, "exp", seed=N)
+        for shift in (0, 2):
+            off = synth.offsets_from_lengths(lens) + shift
+            x = synth.gen(1, "i32_full", 0, int(off[-1]) + 1, seed=N)
+            ref = O.ragged_reduce(x, off)
+            refm = O.ragged_reduce(x, off, op=C.MAX)
+            for S in (64, 128, 256, 512, 1024):
+                for d in (C.CYCLIC, C.BLOCK):
+                    what = f"ragged big N={N} S={S} d={d} shift={shift}"
+                    assert_exact(host(C.cudanp_ragged_loop_reduce(dev(x), dev(off), S=S, dist=d)), ref, what)
+                    assert_exact(host(C.cudanp_ragged_loop_reduce(dev(x), dev(off), op=C.MAX, S=S, dist=d)),
+                                 refm, what)

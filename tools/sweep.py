@@ -272,6 +272,14 @@ def r1(means=(16, 64, 256, 1024)):
             out = torch.empty(N, device="cuda")
             nb = 4 * total + 8 * (N + 1) + 4 * N
             lit = time_ms(lambda: C.cudanp_ragged_loop_reduce_literal(x, off, None, out))[0]
+            if N < (1 << 20):  # few, long segments: multi-warp teams too
+                for S in (64, 128, 256, 512, 1024):
+                    for d in (C.CYCLIC, C.BLOCK):
+                        med, _ = time_ms(lambda: C.cudanp_ragged_loop_reduce(x, off, None, out, S=S, dist=d))
+                        emit({"config": "R1", "op": "ragged_reduce_bigS", "dtype": "f32", "N": N,
+                              "L": f"{dist}{mean}", "S": S, "dist": DN[d], "map": "intra", "impl": "np",
+                              "t_median_us": round(med * 1e3, 2), "alg_bytes": nb,
+                              "gbs": round(nb / (med * 1e-3) / 1e9, 1)})
             sweep_np("R1", "ragged_reduce", nb,
                      lambda S, d, m: time_ms(lambda: C.cudanp_ragged_loop_reduce(x, off, None, out, S=S, dist=d, map=m)),
                      {"dtype": "f32", "N": N, "L": f"{dist}{mean}"}, literal=lit, comps=[("s1_literal", lit)])
