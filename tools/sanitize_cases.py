@@ -56,6 +56,18 @@ def main():
                 C.cudanp_le_gicov(le, 0.01, S=S, dist=d, map=m)
         for be in (C.SHFL, C.SMEM, C.REDUX):
             C.cudanp_batched_loop_reduce_backend(Xi4, inii, S=S, backend=be)
+    for S in (64, 256, 1024):  # multi-warp teams
+        for d in (C.CYCLIC, C.BLOCK):
+            for X, ini in ((Xf, inif), (Xi, inii)):
+                C.cudanp_batched_loop_reduce(X, ini, S=S, dist=d)
+                C.cudanp_batched_loop_scan(X, ini, S=S, dist=d)
+            C.cudanp_mv(A, xm, S=S, dist=d)
+            C.cudanp_ragged_loop_reduce(xr, off, S=S, dist=d)
+            if S == 64:
+                C.cudanp_tmv(A, xt, S=S, dist=d, map=C.INTER_WARP, n_outer=70)
+    for S in (1, 4, 8, 32):  # TMA-staged TMV
+        for d in (C.CYCLIC, C.BLOCK):
+            C.cudanp_tmv_tma(A4, xt, S=S, dist=d)
     for S in (3, 5, 10, 15):
         C.cudanp_le_gicov(le, 0.01, S=S, map=C.INTER_WARP, layout=0)
     if not quick:
