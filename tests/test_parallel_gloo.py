@@ -56,6 +56,8 @@ def _worker(rank, world, port, q):
 def test_sharded_gather_matches_unsharded(world):
     import oracle as O
     import synth
+    from paper_conf_ppopp_yangz14_b200 import build as B
+    B.build()  # the shard ranges come from the library (host logic, no GPU needed)
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
