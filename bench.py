@@ -257,6 +257,7 @@ def run_cudanp(args):
     C.cudanp_dp_set_pending_launch_limit(1 << 16)
     for op, fn in () if args.no_sweep else (("tmv_s1_literal", lambda: C.cudanp_tmv_variant(C.S1_LITERAL, A_t, x_t, y_t)),
                    ("mv_s1_literal", lambda: C.cudanp_mv_variant(C.S1_LITERAL, A_m, x_m, y_m)),
+                   ("tmv_s1_tma", lambda: C.cudanp_tmv_tma(A_t, x_t, y_t, S=1)),
                    ("tmv_dp_block", lambda: C.cudanp_tmv_variant(C.DP_BLOCK, A_t, x_t, y_t)),
                    ("mv_dp_block", lambda: C.cudanp_mv_variant(C.DP_BLOCK, A_m, x_m, y_m)),
                    ("tmv_dp_thread", lambda: C.cudanp_tmv_variant(C.DP_THREAD, A_t, x_t, y_t)),
@@ -380,11 +381,13 @@ def run_cudanp(args):
     def gbs(nb, t):
         return round(nb / (t * 1e-3) / 1e9, 1)
 
-    # "tuned S=1" = the best no-NP kernel: the S=1 instantiations and the literal
+    # "tuned S=1" = the best no-NP kernel: the S=1 instantiations, the literal and
+    # (TMV) the TMA-staged S=1 kernel
     def best_s1(op):
         c = [v for (S, d, m), v in sweep[op].items() if S == 1]
-        if f"{op}_s1_literal" in comp:
-            c.append(comp[f"{op}_s1_literal"])
+        for extra in (f"{op}_s1_literal", f"{op}_s1_tma"):  # every no-NP kernel we have
+            if extra in comp:
+                c.append(comp[extra])
         return min(c or [float("nan")])
 
     per_S = {}
