@@ -40,6 +40,7 @@ sys.path.insert(0, ROOT)
 METRIC = "HBM GB/s and speedup vs S=1 no-NP kernel per slave count, at 1/2/4/8 B200"
 H = W = 16384
 SEED = 20140215
+MAPN = {1: "intra", 2: "inter", 3: "inter_tma"}   # cudanp_map
 
 
 def parse():
@@ -239,7 +240,7 @@ def run_cudanp(args):
         def parse_cfg(s):
             S, d, m = s.split(",")
             return (int(S), {"cyclic": C.CYCLIC, "block": C.BLOCK}[d],
-                    {"intra": C.INTRA_WARP, "inter": C.INTER_WARP}[m])
+                    {"intra": C.INTRA_WARP, "inter": C.INTER_WARP, "inter_tma": C.INTER_WARP_TMA}[m])
         sweep["tmv"][parse_cfg(args.tmv_cfg)] = 1.0
         sweep["mv"][parse_cfg(args.mv_cfg)] = 1.0
     else:
@@ -402,8 +403,8 @@ def run_cudanp(args):
                 "gbs": gbs(nb, cand[k]), "ms": round(cand[k], 4),
                 "speedup_vs_s1": round(s1 / cand[k], 3),
                 "dist": "cyclic" if k[1] == C.CYCLIC else "block",
-                "map": "intra" if k[2] == C.INTRA_WARP else "inter",
-                "all": {f"{'cyc' if d == C.CYCLIC else 'blk'}/{'intra' if m == C.INTRA_WARP else 'inter'}":
+                "map": MAPN[k[2]],
+                "all": {f"{'cyc' if d == C.CYCLIC else 'blk'}/{MAPN[m]}":
                         gbs(nb, v) for (SS, d, m), v in cand.items()}}
     s1_tmv, s1_mv = best_s1("tmv"), best_s1("mv")
 
@@ -415,10 +416,8 @@ def run_cudanp(args):
         "config": {
             "workload": f"C2: TMV y=A^T x + MV y=A x, {n}x{n} fp32 per rank (BASELINE configs[1])",
             "h": n, "w": n, "outer_items_per_rank": {"tmv": wt, "mv": hm}, "inner_count": n,
-            "tmv": {"S": St, "dist": "cyclic" if dt == 0 else "block",
-                    "map": "intra" if mt == 1 else "inter"},
-            "mv": {"S": Sm, "dist": "cyclic" if dm == 0 else "block",
-                   "map": "intra" if mm == 1 else "inter"},
+            "tmv": {"S": St, "dist": "cyclic" if dt == 0 else "block", "map": MAPN[mt]},
+            "mv": {"S": Sm, "dist": "cyclic" if dm == 0 else "block", "map": MAPN[mm]},
             "parallelism": (f"dp{world}: contiguous outer-item shards + "
                             + ("gather fused into the master stores (CUDA IPC over NVLink)"
                                if fused else "NCCL send/recv gather to rank 0"))

@@ -58,7 +58,12 @@ typedef enum {
 } cudanp_status;
 
 typedef enum { CUDANP_DIST_CYCLIC = 0, CUDANP_DIST_BLOCK = 1 } cudanp_dist;
-typedef enum { CUDANP_MAP_AUTO = 0, CUDANP_MAP_INTRA_WARP = 1, CUDANP_MAP_INTER_WARP = 2 } cudanp_map;
+typedef enum {
+  CUDANP_MAP_AUTO = 0,
+  CUDANP_MAP_INTRA_WARP = 1,
+  CUDANP_MAP_INTER_WARP = 2,
+  CUDANP_MAP_INTER_WARP_TMA = 3  /* cudanp_tmv only: inter-warp, A staged by TMA (= cudanp_tmv_tma) */
+} cudanp_map;
 typedef enum { CUDANP_F32 = 0, CUDANP_I32 = 1 } cudanp_dtype;
 typedef enum { CUDANP_SUM = 0, CUDANP_MAX = 1 } cudanp_op;
 
@@ -70,19 +75,32 @@ typedef enum { CUDANP_SUM = 0, CUDANP_MAX = 1 } cudanp_op;
  * j < n_outer.  Master = column j (one output per master); the inner loop
  * runs over the h = n_inner rows.  A: n_inner x lda fp32 (lda >= n_outer),
  * x: n_inner fp32, y: n_outer fp32.  fp32 FMA accumulation; the S partial
- * sums are combined by the team reduction. */
+ * sums are combined by the team reduction.  map = CUDANP_MAP_INTER_WARP_TMA
+ * runs cudanp_tmv_tma (S <= 32; its alignment preconditions apply). */
 int cudanp_tmv(const float* A, int64_t lda, const float* x, float* y,
                int64_t n_outer, int64_t n_inner, int S, int dist, int map, void* stream);
 
 /* TMV with TMA-staged tiles (north star: "TMA or cp.async staging where the
  * access pattern is strided (as in y=A^T x)"): the inter-warp map of
- * cudanp_tmv, with one elected thread streaming [32 rows x 128 columns]
- * tiles of A into an 8-stage shared-memory ring (cp.async.bulk.tensor, an
- * mbarrier per stage) that the S slave warps consume; cyclic or block rows.
- * Needs A and y 16-byte aligned, lda % 4 == 0, n_outer % 4 == 0 and both
- * sizes < 2^31, else CUDANP_ERR_UNSUPPORTED (cudanp_tmv handles any case). */
+ * cudanp_tmv (Fig 2).  A CTA owns a strip of COLS
+ * columns (32 column-masters x V) and S slave warps; a dedicated producer
+ * warp (S <= 16; thread 0 for S = 32) streams [R rows x COLS] boxes of A
+ * into a ring of shared-memory stages with cp.async.bulk.tensor (one
+ * full/empty mbarrier pair per stage) and the slaves consume their rows,
+ * cyclic or block (R5).  The shape makes the whole grid resident
+ * at once.  Same result contract as cudanp_tmv (the S partial
+ * sums meet in slave order).  Needs A and y 16-byte aligned, lda % 4 == 0,
+ * n_outer % 4 == 0 and both sizes < 2^31, else CUDANP_ERR_UNSUPPORTED
+ * (cudanp_tmv handles any case). */
 int cudanp_tmv_tma(const float* A, int64_t lda, const float* x, float* y,
                    int64_t n_outer, int64_t n_inner, int S, int dist, void* stream);
+/* Same with the launch shape pinned (tuning / the sweep): cols in {0 = auto,
+ * 32, 64, 128} columns per CTA; rows_sel in {-1 = auto, 0, 1, 2} picks one
+ * of three rows-per-slave-per-stage sizes for this S (each twice the last); stages 0 = auto,
+ * else 2..64 ring stages (CUDANP_ERR_INVALID if the ring exceeds 227 KB). */
+int cudanp_tmv_tma_ex(const float* A, int64_t lda, const float* x, float* y,
+                      int64_t n_outer, int64_t n_inner, int S, int dist,
+                      int cols, int rows_sel, int stages, void* stream);
 
 /* MV (Table 1 "MV"): y[i] = sum_{j<n_inner} A[i*lda + j] * x[j],
  * for i < n_outer.  Master = row i; inner loop over the w = n_inner columns.
@@ -225,7 +243,8 @@ int cudanp_autotune(int op_kind, const void* a, const void* b, void* out, int64_
  * and autotune space P:384): for an NP call with these arguments,
  * report the kernel's block size, grid size, registers per thread, static
  * shared memory bytes and the resolved map.  `op_kind`: 0 tmv, 1 mv,
- * 2 reduce, 3 scan.  Any out pointer may be NULL.
+ * 2 reduce, 3 scan, 4 TMA-staged tmv (dynamic shared memory of its ring in
+ * smem_bytes).  Any out pointer may be NULL.
  * ---------------------------------------------------------------------- */
 int cudanp_launch_info(int op_kind, int64_t n_outer, int64_t n_inner, int dtype, int op,
                        int S, int dist, int map, int vec4,

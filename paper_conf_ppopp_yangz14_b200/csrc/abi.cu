@@ -32,7 +32,8 @@ int dp_reduce(bool, const void*, const void*, void*, int64_t, int64_t, int, int,
 int dp_scan(bool, const void*, const void*, void*, int64_t, int64_t, int, cudaStream_t);
 int dp_error_count(int, int64_t*);
 int dp_memcopy(const float*, float*, int64_t, int64_t, int, cudaStream_t);
-int tmv_tma(const float*, int64_t, const float*, float*, int64_t, int64_t, int, int, cudaStream_t);
+int tmv_tma(const float*, int64_t, const float*, float*, int64_t, int64_t, int, int, int, int, int,
+            cudaStream_t, LaunchInfo*);
 int ragged_np(const void*, const int64_t*, const void*, void*, int64_t, int, int, int, int, int,
               cudaStream_t);
 int ragged_literal(const void*, const int64_t*, const void*, void*, int64_t, int, int, cudaStream_t);
@@ -244,14 +245,17 @@ const char* cudanp_last_error(void) { return g_err; }
 
 int cudanp_tmv(const float* A, int64_t lda, const float* x, float* y, int64_t n_outer,
                int64_t n_inner, int S, int dist, int map, void* stream) {
+  if (map == CUDANP_MAP_INTER_WARP_TMA)
+    return cudanp_tmv_tma_ex(A, lda, x, y, n_outer, n_inner, S, dist, 0, -1, 0, stream);
   int rc = check_tmv_args(A, lda, x, y, n_outer, n_inner, S, dist, map);
   if (rc) return rc;
   return tmv_np(A, lda, x, y, n_outer, n_inner, S, dist, resolve_map(map, true),
                 tmv_vec(A, lda, y, n_outer), as_stream(stream), nullptr);
 }
 
-int cudanp_tmv_tma(const float* A, int64_t lda, const float* x, float* y, int64_t n_outer,
-                   int64_t n_inner, int S, int dist, void* stream) {
+int cudanp_tmv_tma_ex(const float* A, int64_t lda, const float* x, float* y, int64_t n_outer,
+                      int64_t n_inner, int S, int dist, int cols, int rows_sel, int stages,
+                      void* stream) {
   int rc = check_tmv_args(A, lda, x, y, n_outer, n_inner, S, dist, CUDANP_MAP_INTER_WARP);
   if (rc) return rc;
   if (n_outer == 0) return CUDANP_OK;
@@ -262,7 +266,13 @@ int cudanp_tmv_tma(const float* A, int64_t lda, const float* x, float* y, int64_
     set_error("TMA path needs 16-byte aligned A and y, lda %% 4 == 0, n_outer %% 4 == 0, sizes < 2^31");
     return CUDANP_ERR_UNSUPPORTED;
   }
-  return tmv_tma(A, lda, x, y, n_outer, n_inner, S, dist, as_stream(stream));
+  return tmv_tma(A, lda, x, y, n_outer, n_inner, S, dist, cols, rows_sel, stages, as_stream(stream),
+                 nullptr);
+}
+
+int cudanp_tmv_tma(const float* A, int64_t lda, const float* x, float* y, int64_t n_outer,
+                   int64_t n_inner, int S, int dist, void* stream) {
+  return cudanp_tmv_tma_ex(A, lda, x, y, n_outer, n_inner, S, dist, 0, -1, 0, stream);
 }
 
 int cudanp_mv(const float* A, int64_t lda, const float* x, float* y, int64_t n_outer,
@@ -467,6 +477,10 @@ int cudanp_launch_info(int op_kind, int64_t n_outer, int64_t n_inner, int dtype,
     case 3:
       rc = check_dtype_op(dtype, CUDANP_SUM);
       if (!rc) rc = scan_np(nullptr, nullptr, nullptr, n_outer, n_inner, dtype, S, dist, m, v, 0, &info);
+      break;
+    case 4:  // TMA-staged TMV (auto shape), inter-warp
+      if (n_outer == 0 || n_inner == 0) return fail_invalid("tma launch shape needs n_outer, n_inner > 0");
+      rc = tmv_tma(nullptr, 0, nullptr, nullptr, n_outer, n_inner, S, dist, 0, -1, 0, 0, &info);
       break;
     default: return fail_invalid("op_kind");
   }

@@ -5,7 +5,8 @@
 // the fastest by running them, since "CUDA-NP only generates a small number of
 // versions, the optimal version can be found by testing these versions
 // exhaustively".  Here the versions are the
-// library's (S, dist, map) instantiations; cudanp_autotune times each one on
+// library's (S, dist, map) instantiations (for TMV also the TMA-staged
+// inter-warp kernel, map CUDANP_MAP_INTER_WARP_TMA); cudanp_autotune times each one on
 // the caller's operands with CUDA events on the caller's stream and reports
 // the fastest.  Host code only: it calls the public entry points.
 #include <cmath>
@@ -23,7 +24,9 @@ static std::vector<Candidate> candidates(int op_kind) {
   for (int S : small)
     for (int d = 0; d < 2; ++d)
       for (int m = CUDANP_MAP_INTRA_WARP; m <= CUDANP_MAP_INTER_WARP; ++m) c.push_back({S, d, m});
-  if (op_kind == 0) {  // TMV: inter-warp teams up to 128
+  if (op_kind == 0) {  // TMV: TMA-staged inter-warp, and inter-warp teams up to 128
+    for (int S : small)
+      for (int d = 0; d < 2; ++d) c.push_back({S, d, CUDANP_MAP_INTER_WARP_TMA});
     for (int S : {64, 128})
       for (int d = 0; d < 2; ++d) c.push_back({S, d, CUDANP_MAP_INTER_WARP});
   } else {             // MV / reduce / scan: multi-warp teams
@@ -93,7 +96,7 @@ int cudanp_autotune(int op_kind, const void* a, const void* b, void* out, int64_
         cudaEventElapsedTime(&ms, e0, e1);
         ms /= reps;
       }
-    } else if (r == CUDANP_ERR_CUDA) {
+    } else if (r == CUDANP_ERR_CUDA && c[i].map != CUDANP_MAP_INTER_WARP_TMA) {
       rc = r;
       break;
     }

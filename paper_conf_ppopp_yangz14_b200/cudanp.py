@@ -22,7 +22,7 @@ LIB_PATH = os.path.join(_PKG, "libcudanp.so")
 
 OK, ERR_INVALID, ERR_UNSUPPORTED, ERR_CUDA, ERR_NCCL = 0, 1, 2, 3, 4
 CYCLIC, BLOCK = 0, 1
-AUTO, INTRA_WARP, INTER_WARP = 0, 1, 2
+AUTO, INTRA_WARP, INTER_WARP, INTER_WARP_TMA = 0, 1, 2, 3
 F32, I32 = 0, 1
 SUM, MAX = 0, 1
 S1_LITERAL, DP_THREAD, DP_BLOCK = 1, 2, 3
@@ -37,6 +37,7 @@ _SIGS = {
     "cudanp_tmv": [_vp, _i64, _vp, _vp, _i64, _i64, _int, _int, _int, _vp],
     "cudanp_mv": [_vp, _i64, _vp, _vp, _i64, _i64, _int, _int, _int, _vp],
     "cudanp_tmv_tma": [_vp, _i64, _vp, _vp, _i64, _i64, _int, _int, _vp],
+    "cudanp_tmv_tma_ex": [_vp, _i64, _vp, _vp, _i64, _i64, _int, _int, _int, _int, _int, _vp],
     "cudanp_batched_loop_reduce": [_vp, _vp, _vp, _i64, _i64, _int, _int, _int, _int, _int, _vp],
     "cudanp_batched_loop_scan": [_vp, _vp, _vp, _i64, _i64, _int, _int, _int, _int, _vp],
     "cudanp_batched_loop_reduce_backend": [_vp, _vp, _vp, _i64, _i64, _int, _int, _int, _int, _vp],
@@ -153,15 +154,21 @@ def cudanp_tmv(A, x, y=None, *, S=32, dist=CYCLIC, map=AUTO, n_outer=None, strea
     return y
 
 
-def cudanp_tmv_tma(A, x, y=None, *, S=8, dist=CYCLIC, n_outer=None, stream=None):
-    """TMV with TMA-staged tiles (inter-warp map); same result contract as cudanp_tmv."""
+def cudanp_tmv_tma(A, x, y=None, *, S=8, dist=CYCLIC, n_outer=None, stream=None,
+                   cols=0, rows_sel=-1, stages=0):
+    """TMV with TMA-staged tiles (inter-warp map); same result contract as cudanp_tmv.
+    cols / rows_sel / stages pin the launch shape (cudanp_tmv_tma_ex); defaults = auto."""
     import torch
     h, lda = A.shape
     w = lda if n_outer is None else n_outer
     if y is None:
         y = torch.empty(w, dtype=torch.float32, device=A.device)
-    _check(load().cudanp_tmv_tma(_ptr(A), lda, _ptr(x), _ptr(y), w, h, S, dist, _stream(stream)),
-           "cudanp_tmv_tma")
+    if cols == 0 and rows_sel == -1 and stages == 0:
+        rc = load().cudanp_tmv_tma(_ptr(A), lda, _ptr(x), _ptr(y), w, h, S, dist, _stream(stream))
+    else:
+        rc = load().cudanp_tmv_tma_ex(_ptr(A), lda, _ptr(x), _ptr(y), w, h, S, dist, cols,
+                                      rows_sel, stages, _stream(stream))
+    _check(rc, "cudanp_tmv_tma")
     return y
 
 
@@ -365,13 +372,13 @@ def cudanp_autotune(op_kind: str, a, b, out, *, lda=0, n_outer, n_inner, dtype=F
 # ---------------------------------------------------------------- support
 def cudanp_launch_info(op_kind: str, n_outer: int, n_inner: int, *, dtype=F32, op=SUM, S=8,
                        dist=CYCLIC, map=AUTO, vec4=True) -> dict:
-    kinds = {"tmv": 0, "mv": 1, "reduce": 2, "scan": 3}
+    kinds = {"tmv": 0, "mv": 1, "reduce": 2, "scan": 3, "tmv_tma": 4}
     b, g, r, s, m = _int(), _i64(), _int(), _int(), _int()
     _check(load().cudanp_launch_info(kinds[op_kind], n_outer, n_inner, dtype, op, S, dist, map,
                                      int(vec4), ctypes.byref(b), ctypes.byref(g), ctypes.byref(r),
                                      ctypes.byref(s), ctypes.byref(m)), "cudanp_launch_info")
     return {"block_threads": b.value, "grid_ctas": g.value, "regs_per_thread": r.value,
-            "smem_bytes": s.value, "map": {1: "intra_warp", 2: "inter_warp"}.get(m.value, "?")}
+            "smem_bytes": s.value, "map": {1: "intra_warp", 2: "inter_warp", 3: "inter_warp_tma"}.get(m.value, "?")}
 
 
 def cudanp_ipc_get_handle(t) -> tuple[bytes, int]:

@@ -511,6 +511,8 @@ def test_tmv_tma_parity():
             for S, dist in itertools.product(SS, DISTS):
                 got = host(C.cudanp_tmv_tma(Ad, xd, S=S, dist=dist))
                 what = f"tma h={h} w={w} {kind} S={S} dist={dist}"
+                # the same kernel through cudanp_tmv's map argument
+                assert_exact(host(C.cudanp_tmv(Ad, xd, S=S, dist=dist, map=C.INTER_WARP_TMA)), got, what)
                 if kind == "f32_int4":
                     assert_exact(got, ref, what)
                 else:
@@ -523,6 +525,33 @@ def test_tmv_tma_parity():
     with pytest.raises(C.CudanpError) as ei:
         C.cudanp_tmv_tma(dev(synth.matrix(5, 6, "f32_int4")), dev(synth.vector(5, "f32_int4")))
     assert ei.value.status == C.ERR_UNSUPPORTED
+
+
+def test_tmv_tma_pinned_shapes_parity():
+    # every strip width x rows-per-slave x ring depth, with rings that wrap
+    # many times, ragged last strips and rows past h (zero-filled by TMA)
+    for h, w in [(1000, 516), (2049, 1028)]:
+        A = synth.matrix(h, w, "f32_int4")
+        x = synth.vector(h, "f32_int4")
+        ref = O.tmv(A, x)
+        Ad, xd = dev(A), dev(x)
+        ran = 0
+        for S, dist, cols, rs, st in itertools.product(SS, DISTS, (32, 64, 128), (0, 1, 2), (2, 3)):
+            try:
+                got = host(C.cudanp_tmv_tma(Ad, xd, S=S, dist=dist, cols=cols, rows_sel=rs, stages=st))
+            except C.CudanpError as e:   # this ring does not fit 227 KB
+                assert e.status == C.ERR_INVALID
+                continue
+            ran += 1
+            assert_exact(got, ref, f"tma h={h} w={w} S={S} dist={dist} cols={cols} rs={rs} st={st}")
+        assert ran >= 180
+    with pytest.raises(C.CudanpError) as ei:   # a ring larger than shared memory
+        C.cudanp_tmv_tma(Ad, xd, S=32, cols=128, rows_sel=1, stages=64)
+    assert ei.value.status == C.ERR_INVALID
+    info = C.cudanp_launch_info("tmv_tma", 16384, 16384, S=8)
+    # a producer warp beside the 8 slave warps; one CTA per strip of 32/64/128 columns
+    assert info["block_threads"] == 32 * 8 + 32 and info["grid_ctas"] in (128, 256, 512)
+    assert 0 < info["smem_bytes"] <= 227 * 1024
 
 
 def test_tmv_tma_full_size_C2():

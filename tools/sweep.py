@@ -33,7 +33,7 @@ from paper_conf_ppopp_yangz14_b200 import cudanp as C  # noqa: E402
 PEAK = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json"))).get("hbm_gbs", 6537.0) \
     if os.path.exists(os.path.join(ROOT, "MEASURED_PEAKS.json")) else 6537.0
 DN = {C.CYCLIC: "cyclic", C.BLOCK: "block"}
-MN = {C.INTRA_WARP: "intra", C.INTER_WARP: "inter"}
+MN = {C.INTRA_WARP: "intra", C.INTER_WARP: "inter", C.INTER_WARP_TMA: "inter_tma"}
 OUT = None
 
 
@@ -87,11 +87,13 @@ def graph_time_ms(fns, reps=5):
     return statistics.median(ts), min(ts)
 
 
-def sweep_np(cfg, op, nbytes, run, extra, s1_ref=None, literal=None, comps=()):
+def sweep_np(cfg, op, nbytes, run, extra, s1_ref=None, literal=None, comps=(), maps=None):
     """run(S, dist, map) -> (median_ms, min_ms).  s1_ref: extra no-NP kernel
     times (e.g. the TMA-staged S=1 TMV) that count toward "tuned S=1"."""
     res = {}
-    for S, d, m in itertools.product(C.SLAVE_SIZES, (C.CYCLIC, C.BLOCK), (C.INTRA_WARP, C.INTER_WARP)):
+    if maps is None:  # TMV also has the TMA-staged inter-warp kernel
+        maps = (C.INTRA_WARP, C.INTER_WARP) + ((C.INTER_WARP_TMA,) if op == "tmv" else ())
+    for S, d, m in itertools.product(C.SLAVE_SIZES, (C.CYCLIC, C.BLOCK), maps):
         res[(S, d, m)] = run(S, d, m)
     # "tuned S=1" = the best no-NP kernel: the S=1 NP-path instantiations and the
     # Fig 2 literal, whichever is faster.
