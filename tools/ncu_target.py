@@ -33,7 +33,7 @@ def main():
     ap.add_argument("--reps", type=int, default=3)
     a = ap.parse_args()
     d = {"cyclic": C.CYCLIC, "block": C.BLOCK}[a.dist]
-    m = {"auto": C.AUTO, "intra": C.INTRA_WARP, "inter": C.INTER_WARP}[a.map]
+    m = {"auto": C.AUTO, "intra": C.INTRA_WARP, "inter": C.INTER_WARP, "inter_tma": C.INTER_WARP_TMA}[a.map]
     C.load()
     if a.op == "ragged":
         import synth

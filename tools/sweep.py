@@ -166,6 +166,10 @@ def c2():
             s1_ref.append(t_tma1)
         for impl, name in ((C.DP_BLOCK, "dp_block"), (C.DP_THREAD, "dp_thread")):
             comps.append((name, time_ms(lambda: fv(impl, A, x, y), reps=3, warm=1)[0]))
+        # vendor-library context (the paper's CUBLAS comparison, Figs 13/14; not
+        # part of the product path): torch.mv on the same operands = cuBLAS sgemv
+        At = A.t() if op == "tmv" else A
+        comps.append(("cublas_sgemv", time_ms(lambda: torch.mv(At, x, out=y))[0]))
         sweep_np("C2", op, nb, lambda S, d, m: time_ms(lambda: fnp(A, x, y, S=S, dist=d, map=m)),
                  {"dtype": "f32", "N": n, "L": n}, s1_ref=s1_ref, literal=lit, comps=comps)
     tma_sweep("C2", A, x, y, n)
