@@ -67,6 +67,14 @@ int sm_count() {
   return cache[dev];
 }
 
+bool pdl_enabled() {
+  static const bool on = [] {
+    const char* e = getenv("CUDANP_PDL");
+    return !(e && e[0] == '0');
+  }();
+  return on;
+}
+
 // ---------------------------------------------------------------- validation
 static bool size_ok(int64_t a, int64_t b) {  // a*b*4 bytes addressable
   if (a < 0 || b < 0) return false;

@@ -40,6 +40,28 @@ inline bool aligned16(const void* p) { return ((uintptr_t)p & 15u) == 0; }
 // SM count of the current device (cached per device ordinal).
 int sm_count();
 
+// Programmatic dependent launch on/off for the hot-path kernels (default on;
+// CUDANP_PDL=0 in the environment turns it off, for A/B measurements).
+bool pdl_enabled();
+
+// Launch `kern` with programmatic stream serialization allowed (when enabled):
+// the kernel must begin with pdl_entry() (np_team.cuh).
+template <typename... KArgs, typename... Args>
+inline cudaError_t launch_pdl(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem,
+                              cudaStream_t st, Args... args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = pdl_enabled() ? 1 : 0;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, kern, static_cast<KArgs>(args)...);
+}
+
 // Grid for a persistent grid-stride kernel: enough CTAs to cover `work_ctas`
 // units of CTA work, capped at (resident CTAs per SM) x (SM count), so the
 // grid is a whole number of waves.

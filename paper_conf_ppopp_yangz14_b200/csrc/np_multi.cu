@@ -28,6 +28,7 @@ template <class T, class Op, int S, int DIST, bool VEC>
 __global__ void __launch_bounds__(MultiShape<S>::CTA, MultiShape<S>::MINB)
 reduce_multi_kernel(const T* __restrict__ in, const T* __restrict__ init, T* __restrict__ out,
                     int64_t N, int64_t L) {
+  pdl_entry();
   using Sh = MultiShape<S>;
   __shared__ T sm[Sh::TEAMS * MultiTeam<S>::W];
   const MultiTeam<S> team;
@@ -69,6 +70,7 @@ template <int S, int DIST, bool VEC>
 __global__ void __launch_bounds__(MultiShape<S>::CTA, MultiShape<S>::MINB)
 mv_multi_kernel(const float* __restrict__ A, int64_t lda, const float* __restrict__ x,
                 float* __restrict__ y, int64_t h, int64_t w) {
+  pdl_entry();
   using Sh = MultiShape<S>;
   __shared__ float sm[Sh::TEAMS * MultiTeam<S>::W];
   const MultiTeam<S> team;
@@ -122,6 +124,7 @@ template <class T, int S, int DIST, bool VEC>
 __global__ void __launch_bounds__(MultiShape<S>::CTA, MultiShape<S>::MINB)
 scan_multi_kernel(const T* __restrict__ in, const T* __restrict__ init, T* __restrict__ out,
                   int64_t N, int64_t L) {
+  pdl_entry();
   using Sh = MultiShape<S>;
   __shared__ T sm[Sh::TEAMS * MultiTeam<S>::W];
   __shared__ T slot[Sh::TEAMS];
@@ -230,7 +233,7 @@ static int reduce_multi_t(const void* in, const void* init, void* out, int64_t N
       return CUDANP_OK;
     }
     if (N == 0) return CUDANP_OK;
-    kern<<<(unsigned)grid, Sh::CTA, 0, st>>>((const T*)in, (const T*)init, (T*)out, N, L);
+    launch_pdl(kern, dim3((unsigned)grid), dim3(Sh::CTA), 0, st, (const T*)in, (const T*)init, (T*)out, N, L);
     return check_launch("batched_loop_reduce (multi-warp team) launch");
   });
   return CUDANP_OK;
@@ -260,7 +263,7 @@ static int scan_multi_t(const void* in, const void* init, void* out, int64_t N, 
       return CUDANP_OK;
     }
     if (N == 0 || L == 0) return CUDANP_OK;
-    kern<<<(unsigned)grid, Sh::CTA, 0, st>>>((const T*)in, (const T*)init, (T*)out, N, L);
+    launch_pdl(kern, dim3((unsigned)grid), dim3(Sh::CTA), 0, st, (const T*)in, (const T*)init, (T*)out, N, L);
     return check_launch("batched_loop_scan (multi-warp team) launch");
   });
   return CUDANP_OK;
@@ -285,7 +288,7 @@ int mv_multi(const float* A, int64_t lda, const float* x, float* y, int64_t h, i
       return CUDANP_OK;
     }
     if (h == 0) return CUDANP_OK;
-    kern<<<(unsigned)grid, Sh::CTA, 0, st>>>(A, lda, x, y, h, w);
+    launch_pdl(kern, dim3((unsigned)grid), dim3(Sh::CTA), 0, st, A, lda, x, y, h, w);
     return check_launch("mv (multi-warp team) launch");
   });
   return CUDANP_OK;

@@ -52,6 +52,7 @@ template <class T, class Op, int S, int DIST, bool VEC, int RB = RB_SHFL, int KT
 __global__ void __launch_bounds__(kReduceBlock)
 reduce_intra_kernel(const T* __restrict__ in, const T* __restrict__ init, T* __restrict__ out,
                     int64_t N, int64_t L) {
+  pdl_entry();
   __shared__ T slots[RB == RB_SMEM ? kReduceBlock : 1];
   constexpr int TPW = 32 / S;
   constexpr int K = KT;
@@ -129,6 +130,7 @@ template <class T, class Op, int S, int DIST, bool VEC>
 __global__ void __launch_bounds__(32 * S)
 reduce_inter_kernel(const T* __restrict__ in, const T* __restrict__ init, T* __restrict__ out,
                     int64_t N, int64_t L) {
+  pdl_entry();
   __shared__ T red[S][33];
   const InterTeam<S> team;
   const int64_t nunits = VEC ? (L >> 2) : L;
@@ -218,7 +220,7 @@ static int launch_reduce_map(const T* in, const T* init, T* out, int64_t N, int6
       return CUDANP_OK;
     }
     if (N == 0) return CUDANP_OK;
-    kern<<<(unsigned)grid, kReduceBlock, 0, st>>>(in, init, out, N, L);
+    launch_pdl(kern, dim3((unsigned)grid), dim3(kReduceBlock), 0, st, in, init, out, N, L);
   } else {
     auto kern = reduce_inter_kernel<T, Op, S, DIST, VEC>;
     const int64_t grid = persistent_grid(kern, 32 * S, 0, (N + 31) / 32);
@@ -228,7 +230,7 @@ static int launch_reduce_map(const T* in, const T* init, T* out, int64_t N, int6
       return CUDANP_OK;
     }
     if (N == 0) return CUDANP_OK;
-    kern<<<(unsigned)grid, dim3(32, S), 0, st>>>(in, init, out, N, L);
+    launch_pdl(kern, dim3((unsigned)grid), dim3(32, S), 0, st, in, init, out, N, L);
   }
   return check_launch("batched_loop_reduce launch");
 }
@@ -283,7 +285,7 @@ static int launch_reduce_backend(const void* in, const void* init, void* out, in
     const int64_t per_cta = (kReduceBlock / 32) * kReduceK;
     const int64_t grid = persistent_grid(kern, kReduceBlock, 0, (ntiles + per_cta - 1) / per_cta);
     if (N == 0) return CUDANP_OK;
-    kern<<<(unsigned)grid, kReduceBlock, 0, st>>>((const T*)in, (const T*)init, (T*)out, N, L);
+    launch_pdl(kern, dim3((unsigned)grid), dim3(kReduceBlock), 0, st, (const T*)in, (const T*)init, (T*)out, N, L);
     return check_launch("batched_loop_reduce_backend launch");
   });
   return CUDANP_OK;

@@ -46,6 +46,7 @@ template <class T, int S, int DIST, bool VEC, int KT = kScanK>
 __global__ void __launch_bounds__(kScanBlock)
 scan_intra_kernel(const T* __restrict__ in, const T* __restrict__ init, T* __restrict__ out,
                   int64_t N, int64_t L) {
+  pdl_entry();
   constexpr int TPW = 32 / S;
   constexpr int K = KT;
   constexpr int V = VEC ? 4 : 1;
@@ -156,6 +157,7 @@ template <class T, int S, int DIST, bool VEC>
 __global__ void __launch_bounds__(32 * S)
 scan_inter_kernel(const T* __restrict__ in, const T* __restrict__ init, T* __restrict__ out,
                   int64_t N, int64_t L) {
+  pdl_entry();
   __shared__ T part[S][33];
   __shared__ T slot[32];
   constexpr int V = VEC ? 4 : 1;
@@ -272,7 +274,7 @@ static int launch_scan_map(const T* in, const T* init, T* out, int64_t N, int64_
       return CUDANP_OK;
     }
     if (N == 0 || L == 0) return CUDANP_OK;
-    kern<<<(unsigned)grid, kScanBlock, 0, st>>>(in, init, out, N, L);
+    launch_pdl(kern, dim3((unsigned)grid), dim3(kScanBlock), 0, st, in, init, out, N, L);
   } else {
     auto kern = scan_inter_kernel<T, S, DIST, VEC>;
     const int64_t grid = persistent_grid(kern, 32 * S, 0, (N + 31) / 32);
@@ -282,7 +284,7 @@ static int launch_scan_map(const T* in, const T* init, T* out, int64_t N, int64_
       return CUDANP_OK;
     }
     if (N == 0 || L == 0) return CUDANP_OK;
-    kern<<<(unsigned)grid, dim3(32, S), 0, st>>>(in, init, out, N, L);
+    launch_pdl(kern, dim3((unsigned)grid), dim3(32, S), 0, st, in, init, out, N, L);
   }
   return check_launch("batched_loop_scan launch");
 }

@@ -25,6 +25,20 @@ namespace cudanp {
 constexpr unsigned kFull = 0xffffffffu;
 
 enum Map : int { MAP_AUTO = 0, MAP_INTRA = 1, MAP_INTER = 2 };
+
+// ---------------------------------------------------------------- launch overlap
+// Programmatic dependent launch (sm_90+): the hot-path kernels are launched
+// with programmatic stream serialization (launch_pdl in common.cuh), so the
+// next kernel on the stream is scheduled while this one drains.  Every such
+// kernel therefore waits for its predecessors' completion and memory
+// (griddepcontrol.wait) before touching global memory -- reads and writes
+// alike, so neither RAW nor WAR hazards can cross kernels -- and only then
+// lets its own dependent launch (one kernel ahead at most).  Launched
+// without the attribute both instructions are no-ops.
+__device__ __forceinline__ void pdl_entry() {
+  asm volatile("griddepcontrol.wait;" ::: "memory");
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+}
 enum Dist : int { DIST_CYCLIC = 0, DIST_BLOCK = 1 };
 
 // ---------------------------------------------------------------- operators

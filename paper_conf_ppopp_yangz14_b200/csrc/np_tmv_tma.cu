@@ -85,6 +85,7 @@ template <int S, int DIST, int COLS, int RK>
 __global__ void __launch_bounds__(TmaThreads<S>::value, TmaMinBlocks<S>::value)
 tmv_tma_kernel(const __grid_constant__ CUtensorMap mapA, const float* __restrict__ x,
                float* __restrict__ y, int64_t w, int64_t h, int stages) {
+  pdl_entry();
   constexpr bool PW = TmaPW<S>::value;
   constexpr int V = COLS / 32;
   constexpr int R = RK * S;  // rows per stage
@@ -263,7 +264,7 @@ static int launch_tmv_tma_s(const float* A, int64_t lda, const float* x, float* 
   }
   if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess)
     return check_launch("tmv_tma smem attribute");
-  kern<<<grid, TmaThreads<S>::value, smem, st>>>(map, x, y, w, h, stages);
+  launch_pdl(kern, dim3(grid), dim3(TmaThreads<S>::value), smem, st, map, x, y, w, h, stages);
   return check_launch("tmv_tma launch");
 }
 

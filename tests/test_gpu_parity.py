@@ -647,3 +647,32 @@ def test_autotune_picks_a_valid_fastest_version():
     # TMV's candidate list only holds the built combinations (inter-warp for S > 32)
     assert (64, C.CYCLIC, C.INTRA_WARP) not in tables["tmv"]
     assert tables["tmv"][(64, C.CYCLIC, C.INTER_WARP)] != float("inf")
+
+
+# ------------------------------------------------------------------ launch overlap (PDL)
+def test_chained_calls_without_sync_see_their_predecessors():
+    # The hot-path kernels are launched with programmatic dependent launch, so
+    # each must wait for the previous kernel before reading its output (RAW)
+    # or overwriting what it still reads (WAR).  Chain calls through shared
+    # buffers with no host synchronisation in between and compare with the
+    # oracle applied to the same chain.
+    h = w = 1024
+    A = synth.matrix(h, w, "f32_int4")
+    x = synth.vector(h, "f32_int4")
+    it = synth.items(3000, 96, "i32_small")
+    Ad, xd, itd = dev(A), dev(x), dev(it)
+    y1 = torch.empty(w, device="cuda")
+    y2 = torch.empty(h, device="cuda")
+    sc = torch.empty_like(itd)
+    red = torch.empty(3000, dtype=torch.int32, device="cuda")
+    for rep in range(20):
+        S = (8, 16, 32, 64)[rep % 4]
+        C.cudanp_tmv(Ad, xd, y1, S=min(S, 32), map=C.INTER_WARP_TMA if rep % 2 else C.INTER_WARP)
+        C.cudanp_mv(Ad, y1, y2, S=S, map=C.INTRA_WARP)          # reads y1 (RAW)
+        C.cudanp_tmv(Ad, y2, y1, S=S if S <= 32 else 64, map=C.INTER_WARP)  # overwrites y1 (WAR)
+        C.cudanp_batched_loop_scan(itd, None, sc, S=S, map=C.INTRA_WARP)
+        C.cudanp_batched_loop_reduce(sc, None, red, dtype=C.I32, S=S, map=C.INTRA_WARP)
+    ref_y2 = O.mv(A, O.tmv(A, x))           # integers < 2^24: exact in any order
+    assert_exact(host(y2), ref_y2, "tmv -> mv chain")
+    assert_rel(host(y1), O.tmv(A, ref_y2), h, "tmv -> mv -> tmv chain")
+    assert_exact(host(red), O.reduce(O.scan(it)), "scan -> reduce chain")
