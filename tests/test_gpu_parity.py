@@ -671,7 +671,7 @@ def test_chained_calls_without_sync_see_their_predecessors():
         C.cudanp_mv(Ad, y1, y2, S=S, map=C.INTRA_WARP)          # reads y1 (RAW)
         C.cudanp_tmv(Ad, y2, y1, S=S if S <= 32 else 64, map=C.INTER_WARP)  # overwrites y1 (WAR)
         C.cudanp_batched_loop_scan(itd, None, sc, S=S, map=C.INTRA_WARP)
-        C.cudanp_batched_loop_reduce(sc, None, red, dtype=C.I32, S=S, map=C.INTRA_WARP)
+        C.cudanp_batched_loop_reduce(sc, None, red, S=S, map=C.INTRA_WARP)
     ref_y2 = O.mv(A, O.tmv(A, x))           # integers < 2^24: exact in any order
     assert_exact(host(y2), ref_y2, "tmv -> mv chain")
     assert_rel(host(y1), O.tmv(A, ref_y2), h, "tmv -> mv -> tmv chain")
