@@ -65,9 +65,17 @@ def main():
             C.cudanp_ragged_loop_reduce(xr, off, S=S, dist=d)
             if S == 64:
                 C.cudanp_tmv(A, xt, S=S, dist=d, map=C.INTER_WARP, n_outer=70)
-    for S in (1, 4, 8, 32):  # TMA-staged TMV
+    At = dev(synth.matrix(600, 132, "f32_unit"))   # tall: the rings wrap several times
+    xtt = dev(synth.vector(600))
+    for S in (1, 2, 4, 8, 16, 32):  # TMA-staged TMV, auto and pinned shapes
         for d in (C.CYCLIC, C.BLOCK):
             C.cudanp_tmv_tma(A4, xt, S=S, dist=d)
+            C.cudanp_tmv(At, xtt, S=S, dist=d, map=C.INTER_WARP_TMA)
+            for cols, rs in ((32, 0), (64, 1), (128, 2)):
+                try:
+                    C.cudanp_tmv_tma(At, xtt, S=S, dist=d, cols=cols, rows_sel=rs, stages=2)
+                except C.CudanpError:
+                    pass  # ring larger than shared memory for this S
     for S in (3, 5, 10, 15):
         C.cudanp_le_gicov(le, 0.01, S=S, map=C.INTER_WARP, layout=0)
     if not quick:
