@@ -62,7 +62,9 @@ typedef enum {
   CUDANP_MAP_AUTO = 0,
   CUDANP_MAP_INTRA_WARP = 1,
   CUDANP_MAP_INTER_WARP = 2,
-  CUDANP_MAP_INTER_WARP_TMA = 3  /* cudanp_tmv only: inter-warp, A staged by TMA (= cudanp_tmv_tma) */
+  CUDANP_MAP_INTER_WARP_TMA = 3, /* cudanp_tmv only: inter-warp, A staged by TMA (= cudanp_tmv_tma) */
+  CUDANP_MAP_INTRA_WARP_TMA = 4  /* cudanp_batched_loop_reduce only: intra-warp teams fed from a
+                                    TMA bulk-copy ring (= cudanp_batched_loop_reduce_tma) */
 } cudanp_map;
 typedef enum { CUDANP_F32 = 0, CUDANP_I32 = 1 } cudanp_dtype;
 typedef enum { CUDANP_SUM = 0, CUDANP_MAX = 1 } cudanp_op;
@@ -130,6 +132,18 @@ int cudanp_batched_loop_reduce(const void* in, const void* init, void* out,
 int cudanp_batched_loop_reduce_backend(const void* in, const void* init, void* out,
                                        int64_t n_outer, int64_t n_inner, int dtype, int op,
                                        int S, int backend, void* stream);
+
+/* Batched loop-reduce with the loop body staged by TMA (same contract and
+ * bit-identical results as cudanp_batched_loop_reduce with the intra-warp
+ * map; map = CUDANP_MAP_INTRA_WARP_TMA there selects it): a producer warp
+ * streams runs of consecutive items -- one contiguous block each -- into a
+ * ring of shared-memory stages with cp.async.bulk, eight consumer warps run
+ * the S-lane teams (S <= 32) out of shared memory.  stage_bytes (0 = 64 KB)
+ * and stages (0 = as many as fit, <= 6) shape the ring.  Needs `in` 16-byte
+ * aligned and n_inner % 4 == 0, else CUDANP_ERR_UNSUPPORTED. */
+int cudanp_batched_loop_reduce_tma(const void* in, const void* init, void* out,
+                                   int64_t n_outer, int64_t n_inner, int dtype, int op,
+                                   int S, int dist, int stage_bytes, int stages, void* stream);
 
 /* Batched inclusive scan (scan clause; inclusive per R1):
  * out[n*L + k] = init[n] + sum_{i<=k} in[n*L + i].  init may be NULL (0);
@@ -243,8 +257,8 @@ int cudanp_autotune(int op_kind, const void* a, const void* b, void* out, int64_
  * and autotune space P:384): for an NP call with these arguments,
  * report the kernel's block size, grid size, registers per thread, static
  * shared memory bytes and the resolved map.  `op_kind`: 0 tmv, 1 mv,
- * 2 reduce, 3 scan, 4 TMA-staged tmv (dynamic shared memory of its ring in
- * smem_bytes).  Any out pointer may be NULL.
+ * 2 reduce, 3 scan, 4 TMA-staged tmv, 5 TMA-staged reduce (dynamic shared
+ * memory of their rings in smem_bytes).  Any out pointer may be NULL.
  * ---------------------------------------------------------------------- */
 int cudanp_launch_info(int op_kind, int64_t n_outer, int64_t n_inner, int dtype, int op,
                        int S, int dist, int map, int vec4,

@@ -34,6 +34,8 @@ int dp_error_count(int, int64_t*);
 int dp_memcopy(const float*, float*, int64_t, int64_t, int, cudaStream_t);
 int tmv_tma(const float*, int64_t, const float*, float*, int64_t, int64_t, int, int, int, int, int,
             cudaStream_t, LaunchInfo*);
+int reduce_tma(const void*, const void*, void*, int64_t, int64_t, int, int, int, int, int, int,
+               cudaStream_t, LaunchInfo*);
 int ragged_np(const void*, const int64_t*, const void*, void*, int64_t, int, int, int, int, int,
               cudaStream_t);
 int ragged_literal(const void*, const int64_t*, const void*, void*, int64_t, int, int, cudaStream_t);
@@ -304,9 +306,31 @@ static int check_batched(const void* in, void* out, int64_t N, int64_t L, int S,
   return CUDANP_OK;
 }
 
+int cudanp_batched_loop_reduce_tma(const void* in, const void* init, void* out, int64_t n_outer,
+                                   int64_t n_inner, int dtype, int op, int S, int dist,
+                                   int stage_bytes, int stages, void* stream) {
+  int rc = check_batched(in, out, n_outer, n_inner, S, dist, CUDANP_MAP_INTRA_WARP, dtype, op, true);
+  if (rc) return rc;
+  if (!valid_S(S)) return fail_invalid("TMA-staged reduce: S must be one of 1,2,4,8,16,32");
+  if (stage_bytes < 0 || stages < 0 || stages > 64) return fail_invalid("stage_bytes / stages");
+  if (n_outer == 0) return CUDANP_OK;
+  if (n_inner == 0)  // nothing to stream: the plain kernel writes init / the identity
+    return reduce_np(in, init, out, n_outer, n_inner, dtype, op, S, dist, MAP_INTRA, false,
+                     as_stream(stream), nullptr);
+  if (!((n_inner % 4 == 0) && aligned16(in))) {
+    set_error("TMA-staged reduce needs 16-byte aligned input and n_inner %% 4 == 0");
+    return CUDANP_ERR_UNSUPPORTED;
+  }
+  return reduce_tma(in, init, out, n_outer, n_inner, dtype, op, S, dist, stage_bytes, stages,
+                    as_stream(stream), nullptr);
+}
+
 int cudanp_batched_loop_reduce(const void* in, const void* init, void* out, int64_t n_outer,
                                int64_t n_inner, int dtype, int op, int S, int dist, int map,
                                void* stream) {
+  if (map == CUDANP_MAP_INTRA_WARP_TMA)
+    return cudanp_batched_loop_reduce_tma(in, init, out, n_outer, n_inner, dtype, op, S, dist, 0, 0,
+                                          stream);
   int rc = check_batched(in, out, n_outer, n_inner, S, dist, map, dtype, op, true);
   if (rc) return rc;
   const bool vec = (n_inner % 4 == 0) && aligned16(in);
@@ -489,6 +513,11 @@ int cudanp_launch_info(int op_kind, int64_t n_outer, int64_t n_inner, int dtype,
     case 4:  // TMA-staged TMV (auto shape), inter-warp
       if (n_outer == 0 || n_inner == 0) return fail_invalid("tma launch shape needs n_outer, n_inner > 0");
       rc = tmv_tma(nullptr, 0, nullptr, nullptr, n_outer, n_inner, S, dist, 0, -1, 0, 0, &info);
+      break;
+    case 5:  // TMA-staged reduce (auto shape), intra-warp
+      if (n_outer == 0 || n_inner == 0 || n_inner % 4) return fail_invalid("tma reduce shape needs N, L > 0, L % 4 == 0");
+      rc = check_dtype_op(dtype, op);
+      if (!rc) rc = reduce_tma(nullptr, nullptr, nullptr, n_outer, n_inner, dtype, op, S, dist, 0, 0, 0, &info);
       break;
     default: return fail_invalid("op_kind");
   }

@@ -6,7 +6,8 @@
 // versions, the optimal version can be found by testing these versions
 // exhaustively".  Here the versions are the
 // library's (S, dist, map) instantiations (for TMV also the TMA-staged
-// inter-warp kernel, map CUDANP_MAP_INTER_WARP_TMA); cudanp_autotune times each one on
+// inter-warp kernel, map CUDANP_MAP_INTER_WARP_TMA, and for reduce the
+// TMA-staged intra-warp kernel, CUDANP_MAP_INTRA_WARP_TMA); cudanp_autotune times each one on
 // the caller's operands with CUDA events on the caller's stream and reports
 // the fastest.  Host code only: it calls the public entry points.
 #include <cmath>
@@ -29,7 +30,10 @@ static std::vector<Candidate> candidates(int op_kind) {
       for (int d = 0; d < 2; ++d) c.push_back({S, d, CUDANP_MAP_INTER_WARP_TMA});
     for (int S : {64, 128})
       for (int d = 0; d < 2; ++d) c.push_back({S, d, CUDANP_MAP_INTER_WARP});
-  } else {             // MV / reduce / scan: multi-warp teams
+  } else {             // MV / reduce / scan: multi-warp teams (+ the TMA-staged reduce)
+    if (op_kind == 2)
+      for (int S : small)
+        for (int d = 0; d < 2; ++d) c.push_back({S, d, CUDANP_MAP_INTRA_WARP_TMA});
     for (int S : {64, 128, 256, 512, 1024})
       for (int d = 0; d < 2; ++d) c.push_back({S, d, CUDANP_MAP_INTRA_WARP});
   }
@@ -96,7 +100,7 @@ int cudanp_autotune(int op_kind, const void* a, const void* b, void* out, int64_
         cudaEventElapsedTime(&ms, e0, e1);
         ms /= reps;
       }
-    } else if (r == CUDANP_ERR_CUDA && c[i].map != CUDANP_MAP_INTER_WARP_TMA) {
+    } else if (r == CUDANP_ERR_CUDA && c[i].map < CUDANP_MAP_INTER_WARP_TMA) {
       rc = r;
       break;
     }

@@ -22,7 +22,7 @@ LIB_PATH = os.path.join(_PKG, "libcudanp.so")
 
 OK, ERR_INVALID, ERR_UNSUPPORTED, ERR_CUDA, ERR_NCCL = 0, 1, 2, 3, 4
 CYCLIC, BLOCK = 0, 1
-AUTO, INTRA_WARP, INTER_WARP, INTER_WARP_TMA = 0, 1, 2, 3
+AUTO, INTRA_WARP, INTER_WARP, INTER_WARP_TMA, INTRA_WARP_TMA = 0, 1, 2, 3, 4
 F32, I32 = 0, 1
 SUM, MAX = 0, 1
 S1_LITERAL, DP_THREAD, DP_BLOCK = 1, 2, 3
@@ -39,6 +39,8 @@ _SIGS = {
     "cudanp_tmv_tma": [_vp, _i64, _vp, _vp, _i64, _i64, _int, _int, _vp],
     "cudanp_tmv_tma_ex": [_vp, _i64, _vp, _vp, _i64, _i64, _int, _int, _int, _int, _int, _vp],
     "cudanp_batched_loop_reduce": [_vp, _vp, _vp, _i64, _i64, _int, _int, _int, _int, _int, _vp],
+    "cudanp_batched_loop_reduce_tma": [_vp, _vp, _vp, _i64, _i64, _int, _int, _int, _int, _int, _int,
+                                       _vp],
     "cudanp_batched_loop_scan": [_vp, _vp, _vp, _i64, _i64, _int, _int, _int, _int, _vp],
     "cudanp_batched_loop_reduce_backend": [_vp, _vp, _vp, _i64, _i64, _int, _int, _int, _int, _vp],
     "cudanp_ragged_loop_reduce": [_vp, _vp, _vp, _vp, _i64, _int, _int, _int, _int, _int, _vp],
@@ -215,6 +217,19 @@ def cudanp_batched_loop_reduce_backend(x, init=None, out=None, *, op=SUM, S=8, b
     return out
 
 
+def cudanp_batched_loop_reduce_tma(x, init=None, out=None, *, op=SUM, S=8, dist=CYCLIC,
+                                   stage_bytes=0, stages=0, stream=None):
+    """cudanp_batched_loop_reduce with the rows staged by TMA bulk copies (same result)."""
+    import torch
+    N, L = x.shape
+    if out is None:
+        out = torch.empty(N, dtype=x.dtype, device=x.device)
+    _check(load().cudanp_batched_loop_reduce_tma(_ptr(x), _ptr(init), _ptr(out), N, L, _dtype_code(x),
+                                                 op, S, dist, stage_bytes, stages, _stream(stream)),
+           "cudanp_batched_loop_reduce_tma")
+    return out
+
+
 def cudanp_batched_loop_scan(x, init=None, out=None, *, S=8, dist=CYCLIC, map=AUTO, stream=None):
     """Inclusive scan out[n, k] = init[n] + sum_{i<=k} x[n, i]."""
     import torch
@@ -372,13 +387,13 @@ def cudanp_autotune(op_kind: str, a, b, out, *, lda=0, n_outer, n_inner, dtype=F
 # ---------------------------------------------------------------- support
 def cudanp_launch_info(op_kind: str, n_outer: int, n_inner: int, *, dtype=F32, op=SUM, S=8,
                        dist=CYCLIC, map=AUTO, vec4=True) -> dict:
-    kinds = {"tmv": 0, "mv": 1, "reduce": 2, "scan": 3, "tmv_tma": 4}
+    kinds = {"tmv": 0, "mv": 1, "reduce": 2, "scan": 3, "tmv_tma": 4, "reduce_tma": 5}
     b, g, r, s, m = _int(), _i64(), _int(), _int(), _int()
     _check(load().cudanp_launch_info(kinds[op_kind], n_outer, n_inner, dtype, op, S, dist, map,
                                      int(vec4), ctypes.byref(b), ctypes.byref(g), ctypes.byref(r),
                                      ctypes.byref(s), ctypes.byref(m)), "cudanp_launch_info")
     return {"block_threads": b.value, "grid_ctas": g.value, "regs_per_thread": r.value,
-            "smem_bytes": s.value, "map": {1: "intra_warp", 2: "inter_warp", 3: "inter_warp_tma"}.get(m.value, "?")}
+            "smem_bytes": s.value, "map": {1: "intra_warp", 2: "inter_warp", 3: "inter_warp_tma", 4: "intra_warp_tma"}.get(m.value, "?")}
 
 
 def cudanp_ipc_get_handle(t) -> tuple[bytes, int]:

@@ -676,3 +676,56 @@ def test_chained_calls_without_sync_see_their_predecessors():
     assert_exact(host(y2), ref_y2, "tmv -> mv chain")
     assert_rel(host(y1), O.tmv(A, ref_y2), h, "tmv -> mv -> tmv chain")
     assert_exact(host(red), O.reduce(O.scan(it)), "scan -> reduce chain")
+
+
+# ------------------------------------------------------------------ TMA-staged reduce
+def test_reduce_tma_parity_and_identity_with_ldg():
+    # same per-lane order as the LDG intra-warp kernel -> bit-identical even on
+    # fp32 data; and against the oracle (exact for int32 / max, tol for fp32 sums)
+    for N, L in [(1, 4), (70, 36), (1000, 32), (3001, 64), (777, 256), (50, 1024), (9, 8192)]:
+        for kind, dt in (("f32_unit", C.F32), ("i32_full", C.I32)):
+            X = synth.items(N, L, kind)
+            ini = synth.init(N, "f32_unit" if dt == C.F32 else "i32_small")
+            Xd, inid = dev(X), dev(ini)
+            for op in (C.SUM, C.MAX):
+                ref = O.reduce(X, op=O.SUM if op == C.SUM else O.MAX, init=ini)
+                for S, dist in itertools.product(SS, DISTS):
+                    got = host(C.cudanp_batched_loop_reduce(Xd, inid, op=op, S=S, dist=dist,
+                                                            map=C.INTRA_WARP_TMA))
+                    ldg = host(C.cudanp_batched_loop_reduce(Xd, inid, op=op, S=S, dist=dist,
+                                                            map=C.INTRA_WARP))
+                    what = f"reduce_tma N={N} L={L} {kind} op={op} S={S} dist={dist}"
+                    assert_exact(got, ldg, what + " vs LDG kernel")
+                    if dt == C.I32 or op == C.MAX:
+                        assert_exact(got, ref, what)
+                    else:
+                        assert_rel(got, ref, L, what)
+    # ring shapes: tiny stages (one item per stage, many wraps) and 2-stage rings
+    X = synth.items(513, 64, "i32_small")
+    Xd = dev(X)
+    for sb, st in ((256, 2), (256, 3), (4096, 2), (65536, 3)):
+        got = host(C.cudanp_batched_loop_reduce_tma(Xd, S=8, stage_bytes=sb, stages=st))
+        assert_exact(got, O.reduce(X), f"reduce_tma stage_bytes={sb} stages={st}")
+    # L = 0 writes init; misaligned / L % 4 != 0 are unsupported (the plain call handles them)
+    ini = synth.init(10, "i32_small")
+    got = host(C.cudanp_batched_loop_reduce_tma(dev(np.zeros((10, 0), np.int32)), dev(ini)))
+    assert_exact(got, ini, "reduce_tma L=0")
+    with pytest.raises(C.CudanpError) as ei:
+        C.cudanp_batched_loop_reduce_tma(dev(synth.items(10, 6, "i32_small")))
+    assert ei.value.status == C.ERR_UNSUPPORTED
+    info = C.cudanp_launch_info("reduce_tma", 1 << 22, 32, S=4)
+    assert info["block_threads"] % 32 == 0 and info["grid_ctas"] <= 148
+    assert 0 < info["smem_bytes"] <= 227 * 1024
+
+
+def test_reduce_tma_full_size_C3_sampled():
+    N, L = 1 << 22, 32
+    X = torch.empty(N, L, dtype=torch.int32, device="cuda")
+    C.cudanp_generate(X, "i32_small", stream_id=1, B=1 << 20)
+    items = np.concatenate([np.arange(0, N, 9973), [N - 1]])
+    ref = O.reduce_gen(L, items, O.I32, "i32_small")
+    for S, dist in itertools.product((2, 4, 8), DISTS):
+        got = host(C.cudanp_batched_loop_reduce(X, S=S, dist=dist, map=C.INTRA_WARP_TMA))
+        assert_exact(got[items], ref, f"C3 reduce_tma S={S} dist={dist}")
+    del X
+    torch.cuda.empty_cache()

@@ -33,7 +33,7 @@ from paper_conf_ppopp_yangz14_b200 import cudanp as C  # noqa: E402
 PEAK = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json"))).get("hbm_gbs", 6537.0) \
     if os.path.exists(os.path.join(ROOT, "MEASURED_PEAKS.json")) else 6537.0
 DN = {C.CYCLIC: "cyclic", C.BLOCK: "block"}
-MN = {C.INTRA_WARP: "intra", C.INTER_WARP: "inter", C.INTER_WARP_TMA: "inter_tma"}
+MN = {C.INTRA_WARP: "intra", C.INTER_WARP: "inter", C.INTER_WARP_TMA: "inter_tma", C.INTRA_WARP_TMA: "intra_tma"}
 OUT = None
 
 
@@ -91,10 +91,16 @@ def sweep_np(cfg, op, nbytes, run, extra, s1_ref=None, literal=None, comps=(), m
     """run(S, dist, map) -> (median_ms, min_ms).  s1_ref: extra no-NP kernel
     times (e.g. the TMA-staged S=1 TMV) that count toward "tuned S=1"."""
     res = {}
-    if maps is None:  # TMV also has the TMA-staged inter-warp kernel
-        maps = (C.INTRA_WARP, C.INTER_WARP) + ((C.INTER_WARP_TMA,) if op == "tmv" else ())
+    if maps is None:  # TMV and reduce also have TMA-staged kernels
+        maps = (C.INTRA_WARP, C.INTER_WARP) + {"tmv": (C.INTER_WARP_TMA,),
+                                               "reduce": (C.INTRA_WARP_TMA,)}.get(op, ())
     for S, d, m in itertools.product(C.SLAVE_SIZES, (C.CYCLIC, C.BLOCK), maps):
-        res[(S, d, m)] = run(S, d, m)
+        try:
+            res[(S, d, m)] = run(S, d, m)
+        except C.CudanpError:
+            if m in (C.INTER_WARP_TMA, C.INTRA_WARP_TMA):
+                continue  # e.g. the TMA reduce needs L % 4 == 0
+            raise
     # "tuned S=1" = the best no-NP kernel: the S=1 NP-path instantiations and the
     # Fig 2 literal, whichever is faster.
     s1 = min([v[0] for k, v in res.items() if k[0] == 1] + ([literal] if literal else [])
