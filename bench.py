@@ -55,9 +55,11 @@ def parse():
     ap.add_argument("--no-sweep", action="store_true",
                     help="skip the autotune sweep and comparisons (for ncu launch lists); "
                          "use --tmv-cfg / --mv-cfg")
-    ap.add_argument("--gather", choices=["nccl", "fused"], default="nccl",
-                    help="N > 1: gather outputs to rank 0 with NCCL send/recv, or fused into the "
-                         "kernels' master stores through CUDA IPC over NVLink (SURVEY f4)")
+    ap.add_argument("--gather", choices=["nccl", "fused", "native"], default="nccl",
+                    help="N > 1: gather outputs to rank 0 with NCCL send/recv through "
+                         "torch.distributed, fused into the kernels' master stores through CUDA IPC "
+                         "over NVLink (SURVEY f4), or with the library's own NCCL group "
+                         "(cudanp_group_gather)")
     ap.add_argument("--tmv-cfg", default="32,block,inter")
     ap.add_argument("--mv-cfg", default="16,cyclic,intra")
     return ap.parse_args()
@@ -253,6 +255,16 @@ def run_cudanp(args):
                 if ms < 1e29:  # not supported for this shape
                     sweep[op][cand] = ms
     best = {op: min(sweep[op], key=sweep[op].get) for op in sweep}
+    if not args.no_sweep:
+        # refine: the three fastest versions of each op re-timed with 30 launches
+        # each (the 5-launch sweep is noisy at the 1-2 % level), max over ranks
+        for op, A_, x_, y_, w_ in (("tmv", A_t, x_t, y_t, wt), ("mv", A_m, x_m, y_m, None)):
+            top = sorted(sweep[op], key=sweep[op].get)[:3]
+            fn = C.cudanp_tmv if op == "tmv" else C.cudanp_mv
+            kw = {"n_outer": w_} if op == "tmv" else {}
+            ref = [max_over_ranks(time_op(lambda c=c: fn(A_, x_, y_, S=c[0], dist=c[1], map=c[2], **kw),
+                                          reps=30, warm=3), world) for c in top]
+            best[op] = top[min(range(len(top)), key=ref.__getitem__)]
     # literal S=1 (Fig 2) and DP (per-CTA / per-thread) comparison, once each
     comp = {}
     C.cudanp_dp_set_pending_launch_limit(1 << 16)
@@ -272,6 +284,7 @@ def run_cudanp(args):
     ym_root = torch.empty(n * world, dtype=torch.float32, device="cuda") if rank == 0 else None
 
     fused = world > 1 and args.gather == "fused"
+    native = P.NativeGroup(rank, world) if world > 1 and args.gather == "native" else None
     if fused:
         fg_t = P.FusedGather(y_root, n * world, rank, world)
         fg_m = P.FusedGather(ym_root, n * world, rank, world)
@@ -288,7 +301,10 @@ def run_cudanp(args):
         C.cudanp_mv(A_m, x_m, out_m, S=Sm, dist=dm, map=mm)
         if evs:
             evs[2].record(st)
-        if world > 1 and not fused:
+        if native is not None:
+            native.gather(y_t, y_root, n * world)
+            native.gather(y_m, ym_root, n * world)
+        elif world > 1 and not fused:
             P.gather_to_root(y_t, y_root, n * world, rank, world)
             P.gather_to_root(y_m, ym_root, n * world, rank, world)
 
@@ -420,7 +436,8 @@ def run_cudanp(args):
             "mv": {"S": Sm, "dist": "cyclic" if dm == 0 else "block", "map": MAPN[mm]},
             "parallelism": (f"dp{world}: contiguous outer-item shards + "
                             + ("gather fused into the master stores (CUDA IPC over NVLink)"
-                               if fused else "NCCL send/recv gather to rank 0"))
+                               if fused else "NCCL send/recv gather to rank 0"
+                               + (" (library group, cudanp_group_gather)" if native else "")))
                            if world > 1 else "single GPU",
             "l2": "no flush: each matrix is 1 GiB > 126 MB L2",
             "step": "cudanp_tmv + cudanp_mv (+ gather when n_gpus > 1)",

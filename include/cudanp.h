@@ -272,6 +272,38 @@ int cudanp_launch_info(int op_kind, int64_t n_outer, int64_t n_inner, int dtype,
  * ---------------------------------------------------------------------- */
 int cudanp_shard_range(int64_t n_outer, int nranks, int rank, int64_t* begin, int64_t* end);
 
+/* Native multi-GPU group, one process per GPU: a group is
+ * this process's rank of an NCCL communicator on the current device.
+ * cudanp_group_unique_id: rank 0 writes 128 opaque bytes to id_out, which the
+ *   caller hands to every rank (any channel).
+ * cudanp_group_create: every rank, with the same id, nranks and its rank
+ *   (collective: blocks until all ranks joined).  *out is owned by the caller
+ *   and released with cudanp_group_destroy.
+ * cudanp_group_gather: the contiguous shard [begin_g, end_g) of n_total items
+ *   (cudanp_shard_range) of every rank lands in root_buf on rank 0 (root_buf
+ *   may be NULL elsewhere); NCCL send/recv enqueued on `stream`.
+ * cudanp_sharded_tmv / cudanp_sharded_batched_loop_reduce: this rank's shard
+ *   of the outer items (A_shard = the h x (end-begin) column block, lda its row
+ *   stride, x all h rows; in_shard = items [begin, end)) through the NP call,
+ *   then the gather to y_root / out_root on rank 0.  Same argument rules as
+ *   the single-GPU calls.
+ * NCCL is loaded at run time (libnccl.so.2); CUDANP_ERR_NCCL if it cannot be,
+ * or on any NCCL failure (text in cudanp_last_error()). */
+typedef struct cudanp_group cudanp_group;
+int cudanp_group_unique_id(void* id_out);
+int cudanp_group_create(const void* id, int nranks, int rank, cudanp_group** out);
+int cudanp_group_destroy(cudanp_group* group);
+int cudanp_group_rank(const cudanp_group* group, int* rank, int* nranks);
+int cudanp_group_gather(cudanp_group* group, const void* local, void* root_buf, int64_t n_total,
+                        int dtype, void* stream);
+int cudanp_sharded_tmv(cudanp_group* group, const float* A_shard, int64_t lda, const float* x,
+                       float* y_shard, float* y_root, int64_t n_outer_total, int64_t n_inner,
+                       int S, int dist, int map, void* stream);
+int cudanp_sharded_batched_loop_reduce(cudanp_group* group, const void* in_shard,
+                                       const void* init_shard, void* out_shard, void* out_root,
+                                       int64_t n_outer_total, int64_t n_inner, int dtype, int op,
+                                       int S, int dist, int map, void* stream);
+
 /* Fused gather over NVLink: CUDA IPC lets rank g's kernel
  * epilogue store its outputs straight into rank 0's result buffer, so the
  * master's store *is* the gather -- pass the opened pointer (plus the

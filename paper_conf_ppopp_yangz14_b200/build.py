@@ -27,7 +27,7 @@ LIB = os.path.join(PKG, "libcudanp.so")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 NVFLAGS = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC", "--expt-relaxed-constexpr",
            "-Xptxas", "-warn-spills", "-I" + os.path.join(ROOT, "include")]
-SOURCES = ["abi.cu", "np_reduce.cu", "np_scan.cu", "np_matvec.cu", "np_ragged.cu", "np_le.cu", "np_tmv_tma.cu", "np_reduce_tma.cu", "np_multi.cu", "autotune.cu"]
+SOURCES = ["abi.cu", "np_reduce.cu", "np_scan.cu", "np_matvec.cu", "np_ragged.cu", "np_le.cu", "np_tmv_tma.cu", "np_reduce_tma.cu", "np_multi.cu", "autotune.cu", "group.cu"]
 RDC_SOURCES = ["np_dp.cu"]
 
 
@@ -88,7 +88,7 @@ def build(force: bool = False, jobs: int | None = None, verbose: bool = False,
     _run([cc, *ARCH, "-Xcompiler", "-fPIC", "-dlink", *rdc_objs, "-o", dlink, "-lcudadevrt"])
     tmp = lib + f".tmp{os.getpid()}"
     _run([cc, *ARCH, "-shared", "-Xcompiler", "-fPIC", "-o", tmp, *objs, *rdc_objs, dlink,
-          "-lcudadevrt", "-cudart", "static"])
+          "-lcudadevrt", "-cudart", "static", "-ldl"])
     os.replace(tmp, lib)
     if verbose:
         print("built", lib)

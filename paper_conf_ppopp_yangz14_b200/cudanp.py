@@ -63,6 +63,14 @@ _SIGS = {
     "cudanp_launch_info": [_int, _i64, _i64, _int, _int, _int, _int, _int, _int,
                            ctypes.POINTER(_int), ctypes.POINTER(_i64), ctypes.POINTER(_int),
                            ctypes.POINTER(_int), ctypes.POINTER(_int)],
+    "cudanp_group_unique_id": [_vp],
+    "cudanp_group_create": [_vp, _int, _int, ctypes.POINTER(_vp)],
+    "cudanp_group_destroy": [_vp],
+    "cudanp_group_rank": [_vp, ctypes.POINTER(_int), ctypes.POINTER(_int)],
+    "cudanp_group_gather": [_vp, _vp, _vp, _i64, _int, _vp],
+    "cudanp_sharded_tmv": [_vp, _vp, _i64, _vp, _vp, _vp, _i64, _i64, _int, _int, _int, _vp],
+    "cudanp_sharded_batched_loop_reduce": [_vp, _vp, _vp, _vp, _vp, _i64, _i64, _int, _int, _int, _int,
+                                           _int, _vp],
     "cudanp_shard_range": [_i64, _int, _int, ctypes.POINTER(_i64), ctypes.POINTER(_i64)],
     "cudanp_ipc_get_handle": [_vp, _vp, ctypes.POINTER(_i64)],
     "cudanp_ipc_open": [_vp, _i64, ctypes.POINTER(_vp)],
@@ -412,6 +420,50 @@ def cudanp_ipc_open(handle: bytes, offset: int) -> int:
 
 def cudanp_ipc_close(ptr: int, offset: int) -> None:
     _check(load().cudanp_ipc_close(ptr, offset), "cudanp_ipc_close")
+
+
+# ---------------------------------------------------------------- native multi-GPU group
+def cudanp_group_unique_id() -> bytes:
+    """128-byte NCCL unique id (rank 0 creates it; every rank needs the same bytes)."""
+    buf = ctypes.create_string_buffer(128)
+    _check(load().cudanp_group_unique_id(buf), "cudanp_group_unique_id")
+    return buf.raw
+
+
+def cudanp_group_create(uid: bytes, nranks: int, rank: int) -> int:
+    """This process's rank of the group, on the current CUDA device (collective)."""
+    h = _vp()
+    _check(load().cudanp_group_create(ctypes.create_string_buffer(uid, 128), nranks, rank,
+                                      ctypes.byref(h)), "cudanp_group_create")
+    return h.value
+
+
+def cudanp_group_destroy(group: int) -> None:
+    _check(load().cudanp_group_destroy(group), "cudanp_group_destroy")
+
+
+def cudanp_group_gather(group: int, local, root_buf, n_total: int, stream=None) -> None:
+    _check(load().cudanp_group_gather(group, _ptr(local), _ptr(root_buf), n_total, _dtype_code(local),
+                                      _stream(stream)), "cudanp_group_gather")
+
+
+def cudanp_sharded_tmv(group: int, A_shard, x, y_shard, y_root, n_outer_total: int, *, S=32,
+                       dist=CYCLIC, map=AUTO, stream=None) -> None:
+    h, lda = A_shard.shape
+    _check(load().cudanp_sharded_tmv(group, _ptr(A_shard), lda, _ptr(x), _ptr(y_shard), _ptr(y_root),
+                                     n_outer_total, h, S, dist, map, _stream(stream)),
+           "cudanp_sharded_tmv")
+
+
+def cudanp_sharded_batched_loop_reduce(group: int, in_shard, init_shard, out_shard, out_root,
+                                       n_outer_total: int, *, op=SUM, S=8, dist=CYCLIC, map=AUTO,
+                                       stream=None) -> None:
+    L = in_shard.shape[1]
+    _check(load().cudanp_sharded_batched_loop_reduce(group, _ptr(in_shard), _ptr(init_shard),
+                                                     _ptr(out_shard), _ptr(out_root), n_outer_total, L,
+                                                     _dtype_code(in_shard), op, S, dist, map,
+                                                     _stream(stream)),
+           "cudanp_sharded_batched_loop_reduce")
 
 
 def cudanp_shard_range(n_outer: int, nranks: int, rank: int) -> tuple[int, int]:

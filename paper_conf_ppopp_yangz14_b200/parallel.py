@@ -85,3 +85,36 @@ class FusedGather:
         if self.mapped is not None:
             C.cudanp_ipc_close(self.mapped, self.offset)
             self.mapped = None
+
+
+class NativeGroup:
+    """The library's own multi-GPU group (cudanp_group_*, include/cudanp.h):
+    an NCCL communicator rank created natively from a unique id that rank 0
+    makes and torch.distributed broadcasts once.  ``gather`` enqueues the
+    shard gather to rank 0 on the current stream (NCCL send/recv in the
+    library); ``sharded_tmv`` / ``sharded_reduce`` run this rank's shard and
+    the gather in one C call."""
+
+    def __init__(self, rank: int, world: int):
+        import torch.distributed as dist
+        self.rank, self.world = rank, world
+        obj = [C.cudanp_group_unique_id() if rank == 0 else None]
+        if world > 1:
+            dist.broadcast_object_list(obj, src=0)
+        self.handle = C.cudanp_group_create(obj[0], world, rank)
+
+    def gather(self, local, root_buf, n_total: int):
+        C.cudanp_group_gather(self.handle, local, root_buf, n_total)
+        return root_buf if self.rank == 0 else None
+
+    def sharded_tmv(self, A_shard, x, y_shard, y_root, n_total: int, **kw):
+        C.cudanp_sharded_tmv(self.handle, A_shard, x, y_shard, y_root, n_total, **kw)
+
+    def sharded_reduce(self, in_shard, init_shard, out_shard, out_root, n_total: int, **kw):
+        C.cudanp_sharded_batched_loop_reduce(self.handle, in_shard, init_shard, out_shard, out_root,
+                                             n_total, **kw)
+
+    def close(self):
+        if self.handle:
+            C.cudanp_group_destroy(self.handle)
+            self.handle = None

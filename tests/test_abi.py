@@ -99,3 +99,17 @@ def test_binding_fails_loudly_without_library(tmp_path):
             mod.load(str(tmp_path / "missing.so"))
     finally:
         mod._lib = saved
+
+
+def test_native_group_host_side(lib):
+    # the NCCL unique id needs no GPU; bad arguments are rejected before NCCL
+    uid = C.cudanp_group_unique_id()
+    assert len(uid) == 128 and any(uid)
+    h = ctypes.c_void_p()
+    buf = ctypes.create_string_buffer(uid, 128)
+    assert lib.cudanp_group_create(buf, 0, 0, ctypes.byref(h)) == C.ERR_INVALID
+    assert lib.cudanp_group_create(buf, 2, 2, ctypes.byref(h)) == C.ERR_INVALID
+    assert lib.cudanp_group_create(None, 1, 0, ctypes.byref(h)) == C.ERR_INVALID
+    assert lib.cudanp_group_gather(None, None, None, 10, 0, None) == C.ERR_INVALID
+    assert lib.cudanp_sharded_tmv(None, None, 4, None, None, None, 4, 4, 8, 0, 0, None) == C.ERR_INVALID
+    assert lib.cudanp_group_destroy(None) == C.OK

@@ -2,9 +2,10 @@
 """C5 (BASELINE configs[4]) at G GPUs: TMV 65536^2 fp32 sharded by column
 blocks and a 64M-item x 64 loop-reduce sharded by item blocks (contiguous
 outer ranges), outputs gathered to rank 0 -- NCCL send/recv, or
-fused into the kernels' master stores through CUDA IPC (--gather fused).
+fused into the kernels' master stores through CUDA IPC (--gather fused), or
+the library's own NCCL group (--gather native, cudanp_group_gather).
 
-    torchrun --nproc-per-node G --master-addr 127.0.0.1 tools/c5_scale.py [--gather nccl|fused]
+    torchrun --nproc-per-node G --master-addr 127.0.0.1 tools/c5_scale.py [--gather nccl|fused|native]
 
 Strong scaling: the problem is fixed, each rank owns 1/G of it, generated on
 its device from global indices.  Per op, rank 0 prints one JSON record with
@@ -40,7 +41,7 @@ def ev():
 
 def main():
     ap = argparse.ArgumentParser()
-    ap.add_argument("--gather", choices=["nccl", "fused"], default="nccl")
+    ap.add_argument("--gather", choices=["nccl", "fused", "native"], default="nccl")
     ap.add_argument("--scale", type=int, default=1, help="divide n (TMV) and N (reduce) by this")
     ap.add_argument("--reps", type=int, default=10)
     ap.add_argument("--tmv-cfg", default="16,cyclic,inter")
@@ -59,6 +60,7 @@ def main():
             dist.init_process_group(backend)
     C.load()
     fused = world > 1 and a.gather == "fused"
+    native = P.NativeGroup(rank, world) if world > 1 and a.gather == "native" else None
     maps = {"intra": C.INTRA_WARP, "inter": C.INTER_WARP, "inter_tma": C.INTER_WARP_TMA}
     dists = {"cyclic": C.CYCLIC, "block": C.BLOCK}
 
@@ -75,7 +77,6 @@ def main():
 
     n = 65536 // a.scale
     N, L = (1 << 26) // a.scale, 64
-    results = []
     for op in ("tmv", "reduce"):
         total = n if op == "tmv" else N
         b, e = P.shard(total, world, rank)
@@ -103,7 +104,9 @@ def main():
                 C.cudanp_batched_loop_reduce(A, None, out, S=S, dist=d, map=m)
 
         def gather():
-            if world > 1 and not fused:
+            if native is not None:
+                native.gather(y, root, total)
+            elif world > 1 and not fused:
                 P.gather_to_root(y, root, total, rank, world)
             elif world == 1:
                 root.copy_(y)
@@ -141,7 +144,7 @@ def main():
         if rank == 0:
             import oracle as O  # test infrastructure: the sampled parity check only
             idx = np.unique(np.concatenate([np.linspace(0, total - 1, 257).astype(np.int64),
-                                            [b for g in range(world) for b in P.shard(total, world, g)[:1]]]))
+                                            [P.shard(total, world, g)[0] for g in range(world)]]))
             got = root.cpu().numpy()[idx]
             ref = O.tmv_gen(n, n, idx) if op == "tmv" else O.reduce_gen(L, idx, O.F32, "f32_unit")
             L_ = n if op == "tmv" else L
@@ -153,6 +156,8 @@ def main():
             fg.close()
         del A, y, root
         torch.cuda.empty_cache()
+    if native is not None:
+        native.close()
     if world > 1:
         dist.barrier()
         dist.destroy_process_group()
