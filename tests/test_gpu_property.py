@@ -78,3 +78,28 @@ def test_ragged_random(N, mean, S, dist, map_, op, shift, seed):
     x = synth.gen(1, "i32_full", 0, int(off[-1]) + 1, seed=seed)
     got = host(C.cudanp_ragged_loop_reduce(dev(x), dev(off), op=op, S=S, dist=dist, map=map_))
     assert_exact(got, O.ragged_reduce(x, off, op=op), f"N={N} mean={mean} S={S} d={dist} m={map_}")
+
+
+@CFG
+@given(N=st.integers(0, 700), L4=st.integers(0, 80), S=S_, dist=D_, op=st.sampled_from([C.SUM, C.MAX]),
+       use_init=st.booleans(), sb=st.sampled_from([0, 512, 8192]), seed=st.integers(0, 10**6))
+def test_reduce_tma_random(N, L4, S, dist, op, use_init, sb, seed):
+    L = 4 * L4
+    x = synth.gen(1, "i32_full", 0, N * L, seed=seed).reshape(N, L)
+    ini = synth.init(N, "i32_full", seed=seed)
+    ref = O.reduce(x, op=op, init=ini if use_init else None)
+    got = host(C.cudanp_batched_loop_reduce_tma(dev(x), dev(ini) if use_init and N else None, op=op,
+                                                S=S, dist=dist, stage_bytes=sb))
+    assert_exact(got, ref, f"TMA N={N} L={L} S={S} dist={dist} op={op} stage_bytes={sb}")
+
+
+@CFG
+@given(h=st.integers(0, 400), w4=st.integers(1, 80), pad4=st.integers(0, 2), S=S_, dist=D_,
+       seed=st.integers(0, 10**6))
+def test_tmv_tma_random(h, w4, pad4, S, dist, seed):
+    w, lda = 4 * w4, 4 * (w4 + pad4)
+    A = synth.matrix(h, lda, "f32_int4", seed=seed)
+    x = synth.vector(h, "f32_int4", seed=seed)
+    ref = O.tmv(A, x, w) if h else np.zeros(w, np.float32)
+    got = host(C.cudanp_tmv(dev(A), dev(x), S=S, dist=dist, map=C.INTER_WARP_TMA, n_outer=w))
+    assert_exact(got, ref, f"TMA h={h} w={w} lda={lda} S={S} dist={dist}")

@@ -76,6 +76,17 @@ def main():
                     C.cudanp_tmv_tma(At, xtt, S=S, dist=d, cols=cols, rows_sel=rs, stages=2)
                 except C.CudanpError:
                     pass  # ring larger than shared memory for this S
+    Xt4 = dev(synth.items(300, 36, "i32_small"))   # TMA-staged reduce: rings that wrap
+    for S in (1, 4, 8, 32):
+        for d in (C.CYCLIC, C.BLOCK):
+            C.cudanp_batched_loop_reduce(Xi4, inii, S=S, dist=d, map=C.INTRA_WARP_TMA)
+            C.cudanp_batched_loop_reduce_tma(Xt4, None, op=C.MAX, S=S, dist=d, stage_bytes=1024, stages=2)
+    if not quick:  # native group, world 1
+        g = C.cudanp_group_create(C.cudanp_group_unique_id(), 1, 0)
+        yr = torch.empty(68, device="cuda")
+        C.cudanp_sharded_tmv(g, A4, xt, torch.empty(68, device="cuda"), yr, 68, S=8)
+        torch.cuda.synchronize()
+        C.cudanp_group_destroy(g)
     for S in (3, 5, 10, 15):
         C.cudanp_le_gicov(le, 0.01, S=S, map=C.INTER_WARP, layout=0)
     if not quick:
