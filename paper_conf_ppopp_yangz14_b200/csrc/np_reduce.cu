@@ -48,7 +48,8 @@ __device__ __forceinline__ T redux_op(T v, unsigned mask) {
 // Team = S lanes; a warp holds TPW = 32/S teams = TPW items ("warp tile").
 // Each warp processes K consecutive warp tiles per step of a grid-stride
 // loop, so a lane has K independent rows in flight.
-template <class T, class Op, int S, int DIST, bool VEC, int RB = RB_SHFL, int KT = kReduceK>
+template <class T, class Op, int S, int DIST, bool VEC, int RB = RB_SHFL, int KT = kReduceK,
+          bool W8 = false>
 __global__ void __launch_bounds__(kReduceBlock)
 reduce_intra_kernel(const T* __restrict__ in, const T* __restrict__ init, T* __restrict__ out,
                     int64_t N, int64_t L) {
@@ -56,13 +57,14 @@ reduce_intra_kernel(const T* __restrict__ in, const T* __restrict__ init, T* __r
   __shared__ T slots[RB == RB_SMEM ? kReduceBlock : 1];
   constexpr int TPW = 32 / S;
   constexpr int K = KT;
+  constexpr int V = W8 ? 8 : (VEC ? 4 : 1);  // elements per unit (one load)
   const IntraTeam<S> team;
   const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
-  const int64_t nunits = VEC ? (L >> 2) : L;
+  const int64_t nunits = L / V;
   // Iteration share of this slave: uniform index math, recomputed by every
   // slave instead of broadcast.
-  const Range<S, DIST> r(nunits, L, VEC ? 4 : 1, team.slave);
+  const Range<S, DIST> r(nunits, L, V, team.slave);
   const int64_t ntiles = (N + TPW - 1) / TPW;
 
   for (int64_t t0 = warp * K; t0 < ntiles; t0 += nwarps * K) {
@@ -74,7 +76,32 @@ reduce_intra_kernel(const T* __restrict__ in, const T* __restrict__ init, T* __r
       row[k] = in + (item[k] < N ? item[k] : 0) * L;
     }
     T part[K];
-    if constexpr (VEC) {
+    if constexpr (W8) {
+      // 256-bit units (rows 32-byte aligned, L % 8 == 0): 8 accumulators per lane
+      V8<T> acc[K];
+#pragma unroll
+      for (int k = 0; k < K; ++k)
+#pragma unroll
+        for (int j = 0; j < 8; ++j) acc[k].v[j] = Op::template identity<T>();
+#pragma unroll 2
+      for (int64_t u = r.begin; u < r.end; u += r.step) {
+        V8<T> v[K];
+#pragma unroll
+        for (int k = 0; k < K; ++k)
+          if (item[k] < N) v[k] = ldg8(row[k] + 8 * u);
+#pragma unroll
+        for (int k = 0; k < K; ++k)
+          if (item[k] < N)
+#pragma unroll
+            for (int j = 0; j < 8; ++j) acc[k].v[j] = Op::apply(acc[k].v[j], v[k].v[j]);
+      }
+#pragma unroll
+      for (int k = 0; k < K; ++k) {
+        const V8<T>& a = acc[k];
+        part[k] = Op::apply(Op::apply(Op::apply(a.v[0], a.v[1]), Op::apply(a.v[2], a.v[3])),
+                            Op::apply(Op::apply(a.v[4], a.v[5]), Op::apply(a.v[6], a.v[7])));
+      }
+    } else if constexpr (VEC) {
       V4<T> acc[K];
 #pragma unroll
       for (int k = 0; k < K; ++k) {
@@ -212,6 +239,13 @@ static int launch_reduce_map(const T* in, const T* init, T* out, int64_t N, int6
     const bool few = few_tiles(reduce_intra_kernel<T, Op, S, DIST, VEC>, kReduceBlock, ntiles, kReduceK);
     auto kern = few ? reduce_intra_kernel<T, Op, S, DIST, VEC, RB_SHFL, 1>
                     : reduce_intra_kernel<T, Op, S, DIST, VEC, RB_SHFL, kReduceK>;
+#if defined(CUDANP_LDG256)
+    if constexpr (VEC) {  // 256-bit units when rows are 32-byte aligned
+      if (L % 8 == 0 && ((uintptr_t)in & 31) == 0)
+        kern = few ? reduce_intra_kernel<T, Op, S, DIST, true, RB_SHFL, 1, true>
+                   : reduce_intra_kernel<T, Op, S, DIST, true, RB_SHFL, kReduceK, true>;
+    }
+#endif
     const int64_t per_cta = (kReduceBlock / 32) * (few ? 1 : kReduceK);
     const int64_t grid = persistent_grid(kern, kReduceBlock, 0, (ntiles + per_cta - 1) / per_cta);
     if (info) {

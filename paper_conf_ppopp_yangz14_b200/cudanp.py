@@ -18,7 +18,8 @@ import threading
 import numpy as np
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_PKG, "libcudanp.so")
+# CUDANP_LIB selects a build-variant library (experiments, e.g. -DCUDANP_LDG256)
+LIB_PATH = os.environ.get("CUDANP_LIB") or os.path.join(_PKG, "libcudanp.so")
 
 OK, ERR_INVALID, ERR_UNSUPPORTED, ERR_CUDA, ERR_NCCL = 0, 1, 2, 3, 4
 CYCLIC, BLOCK = 0, 1
