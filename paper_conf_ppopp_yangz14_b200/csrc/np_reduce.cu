@@ -68,6 +68,18 @@ reduce_intra_kernel(const T* __restrict__ in, const T* __restrict__ init, T* __r
   const int64_t ntiles = (N + TPW - 1) / TPW;
 
   for (int64_t t0 = warp * K; t0 < ntiles; t0 += nwarps * K) {
+#if defined(CUDANP_L2PF)
+    if constexpr (VEC) {
+      // The warp's K tiles CUDANP_L2PF steps ahead are one contiguous block of
+      // items: prefetch it into L2 so more bytes are in flight than the
+      // registers of the resident warps hold.
+      const int64_t tp = t0 + (int64_t)CUDANP_L2PF * nwarps * K;
+      if (tp < ntiles && team.lane == 0) {
+        const int64_t i0 = tp * TPW, i1 = (tp + K) * TPW < N ? (tp + K) * TPW : N;
+        prefetch_l2(in + i0 * L, (uint32_t)((i1 - i0) * L * (int64_t)sizeof(T)));
+      }
+    }
+#endif
     int64_t item[K];
     const T* row[K];
 #pragma unroll

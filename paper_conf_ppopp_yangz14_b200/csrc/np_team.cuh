@@ -99,6 +99,12 @@ __device__ __forceinline__ V4<T> ldg4_stream(const T* p) {
 template <class T>
 __device__ __forceinline__ T ldg1(const T* p) { return __ldg(p); }
 
+// Bulk L2 prefetch through the TMA unit (cp.async.bulk.prefetch.L2, SASS
+// UBLKPF.L2): fire-and-forget, no registers; 16-byte aligned, bytes % 16 == 0.
+__device__ __forceinline__ void prefetch_l2(const void* p, uint32_t bytes) {
+  asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(p), "r"(bytes) : "memory");
+}
+
 // 256-bit load (sm_100: LDG.E.ENL2.256.CONSTANT), 32-byte aligned: one
 // request per lane covers a whole 32-byte sector, half the load instructions
 // of 128-bit units for the same bytes in flight.
