@@ -48,9 +48,12 @@ __device__ __forceinline__ T redux_op(T v, unsigned mask) {
 // Team = S lanes; a warp holds TPW = 32/S teams = TPW items ("warp tile").
 // Each warp processes K consecutive warp tiles per step of a grid-stride
 // loop, so a lane has K independent rows in flight.
+#ifndef CUDANP_REDUCE_MINB
+#define CUDANP_REDUCE_MINB 1
+#endif
 template <class T, class Op, int S, int DIST, bool VEC, int RB = RB_SHFL, int KT = kReduceK,
           bool W8 = false>
-__global__ void __launch_bounds__(kReduceBlock)
+__global__ void __launch_bounds__(kReduceBlock, CUDANP_REDUCE_MINB)
 reduce_intra_kernel(const T* __restrict__ in, const T* __restrict__ init, T* __restrict__ out,
                     int64_t N, int64_t L) {
   pdl_entry();
