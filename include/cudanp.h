@@ -184,6 +184,19 @@ int cudanp_ragged_loop_reduce_literal(const void* in, const int64_t* offsets, co
 int cudanp_le_gicov(const float* in, float* gicov, float* ave, float* var, float* ep,
                     int64_t n_outer, int64_t n_inner, float threshold, int layout, int S,
                     int dist, int map, void* stream);
+/* The same with the home of Grad chosen (Fig 6a-c; Fig 15):
+ * CUDANP_GRAD_REGISTERS = cudanp_le_gicov (6c, per-slave register partition);
+ * CUDANP_GRAD_GLOBAL (6a: no private copy, loop 3 re-reads the input through
+ * L1/L2); CUDANP_GRAD_SHARED (6b: runs of whole items are staged in a
+ * shared-memory ring by TMA bulk copies and both loops read it there; built
+ * for layout 0, the intra-warp map, S = 2^k <= 32 and a 16-byte aligned
+ * input, else CUDANP_ERR_UNSUPPORTED; the < 4 items past the last whole
+ * 16-byte run take the register kernel).  All three give
+ * bit-identical results (each slave visits its elements in the same order). */
+typedef enum { CUDANP_GRAD_REGISTERS = 0, CUDANP_GRAD_SHARED = 1, CUDANP_GRAD_GLOBAL = 2 } cudanp_grad_placement;
+int cudanp_le_gicov_placement(const float* in, float* gicov, float* ave, float* var, float* ep,
+                              int64_t n_outer, int64_t n_inner, float threshold, int layout,
+                              int S, int dist, int map, int placement, void* stream);
 /* Comparison: Fig 5 as written, one thread per item, Grad in a per-thread
  * local-memory array when L <= 256. */
 int cudanp_le_gicov_literal(const float* in, float* gicov, float* ave, float* var, float* ep,

@@ -40,7 +40,9 @@ int ragged_np(const void*, const int64_t*, const void*, void*, int64_t, int, int
               cudaStream_t);
 int ragged_literal(const void*, const int64_t*, const void*, void*, int64_t, int, int, cudaStream_t);
 int le_np(const float*, float*, float*, float*, float*, int64_t, int64_t, float, int, int, int, int,
-          cudaStream_t);
+          bool, cudaStream_t);
+int le_tma(const float*, float*, float*, float*, float*, int64_t, int64_t, float, int, int,
+           cudaStream_t);
 int le_literal(const float*, float*, float*, float*, float*, int64_t, int64_t, float, int,
                cudaStream_t);
 
@@ -409,8 +411,29 @@ int cudanp_le_gicov(const float* in, float* gicov, float* ave, float* var, float
   // MAP_AUTO: keep the masters' accesses coalesced: point-major
   // data -> inter-warp (the paper's LE choice); item-major -> intra.
   const int m = map != CUDANP_MAP_AUTO ? map : (layout ? MAP_INTER : MAP_INTRA);
-  return le_np(in, gicov, ave, var, ep, n_outer, n_inner, threshold, layout, S, dist, m,
+  return le_np(in, gicov, ave, var, ep, n_outer, n_inner, threshold, layout, S, dist, m, false,
                as_stream(stream));
+}
+
+int cudanp_le_gicov_placement(const float* in, float* gicov, float* ave, float* var, float* ep,
+                              int64_t n_outer, int64_t n_inner, float threshold, int layout, int S,
+                              int dist, int map, int placement, void* stream) {
+  if (placement == CUDANP_GRAD_REGISTERS)
+    return cudanp_le_gicov(in, gicov, ave, var, ep, n_outer, n_inner, threshold, layout, S, dist,
+                           map, stream);
+  int rc = check_le(in, gicov, n_outer, n_inner, layout, S, dist, map);
+  if (rc) return rc;
+  const int m = map != CUDANP_MAP_AUTO ? map : (layout ? MAP_INTER : MAP_INTRA);
+  if (placement == CUDANP_GRAD_GLOBAL)
+    return le_np(in, gicov, ave, var, ep, n_outer, n_inner, threshold, layout, S, dist, m, true,
+                 as_stream(stream));
+  if (placement != CUDANP_GRAD_SHARED) return fail_invalid("placement");
+  if (layout != 0 || m != MAP_INTRA || !valid_S(S) || !aligned16(in)) {
+    set_error("shared-memory Grad is built for item-major data, the intra-warp map, S = 2^k <= 32 "
+              "and a 16-byte aligned input");
+    return CUDANP_ERR_UNSUPPORTED;
+  }
+  return le_tma(in, gicov, ave, var, ep, n_outer, n_inner, threshold, S, dist, as_stream(stream));
 }
 
 int cudanp_le_gicov_literal(const float* in, float* gicov, float* ave, float* var, float* ep,

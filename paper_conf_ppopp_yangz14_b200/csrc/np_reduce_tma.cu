@@ -95,15 +95,16 @@ reduce_tma_kernel(const T* __restrict__ in, const T* __restrict__ init, T* __res
     mbar_wait(&full[st], (uint32_t)(t / stages) & 1);
     const T* base = ring + st * stage_elems;
     const int ntile = (cnt + TPW - 1) / TPW;
-    // K consecutive warp tiles per step: K independent items per team in
+    // K warp tiles per step (tile0 + k*warps, so a short stage still spreads
+    // over every warp): K independent items per team in
     // flight, so shared-memory and shuffle latencies overlap.
-    for (int tile0 = warp * kRtK; tile0 < ntile; tile0 += kRtWarps * kRtK) {
+    for (int tile0 = warp; tile0 < ntile; tile0 += kRtWarps * kRtK) {
       int il[kRtK];
       const T* row[kRtK];
       V4<T> acc[kRtK];
 #pragma unroll
       for (int k = 0; k < kRtK; ++k) {
-        il[k] = (tile0 + k) * TPW + team.team;
+        il[k] = (tile0 + k * kRtWarps) * TPW + team.team;
         row[k] = base + (int64_t)(il[k] < cnt ? il[k] : 0) * L;
         acc[k] = {id, id, id, id};
       }

@@ -27,6 +27,7 @@ AUTO, INTRA_WARP, INTER_WARP, INTER_WARP_TMA, INTRA_WARP_TMA = 0, 1, 2, 3, 4
 F32, I32 = 0, 1
 SUM, MAX = 0, 1
 S1_LITERAL, DP_THREAD, DP_BLOCK = 1, 2, 3
+GRAD_REGISTERS, GRAD_SHARED, GRAD_GLOBAL = 0, 1, 2   # LE: home of Grad (Fig 6c / 6b / 6a)
 SLAVE_SIZES = (1, 2, 4, 8, 16, 32)
 KIND = {"f32_unit": 0, "f32_signed": 1, "f32_int4": 2, "i32_small": 3, "i32_full": 4,
         "ones_f32": 5, "ones_i32": 6}
@@ -48,6 +49,8 @@ _SIGS = {
     "cudanp_ragged_loop_reduce_literal": [_vp, _vp, _vp, _vp, _i64, _int, _int, _vp],
     "cudanp_le_gicov": [_vp, _vp, _vp, _vp, _vp, _i64, _i64, ctypes.c_float, _int, _int, _int,
                         _int, _vp],
+    "cudanp_le_gicov_placement": [_vp, _vp, _vp, _vp, _vp, _i64, _i64, ctypes.c_float, _int, _int,
+                                  _int, _int, _int, _vp],
     "cudanp_le_gicov_literal": [_vp, _vp, _vp, _vp, _vp, _i64, _i64, ctypes.c_float, _int, _vp],
     "cudanp_tmv_variant": [_int, _vp, _i64, _vp, _vp, _i64, _i64, _vp],
     "cudanp_mv_variant": [_int, _vp, _i64, _vp, _vp, _i64, _i64, _vp],
@@ -279,7 +282,7 @@ def cudanp_ragged_loop_reduce_literal(x, offsets, init=None, out=None, *, op=SUM
 
 
 def cudanp_le_gicov(x, threshold, gicov=None, *, layout=0, S=8, dist=CYCLIC, map=AUTO,
-                    want_stats=True, literal=False, stream=None):
+                    want_stats=True, literal=False, placement=GRAD_REGISTERS, stream=None):
     """LE multi-section item (Figs 5-6): returns (gicov, ave, var, ep).
     x: (N, L) when layout == 0, (L, N) when layout == 1.  gicov entries whose
     test fails are left as given (default: filled with -1)."""
@@ -292,6 +295,10 @@ def cudanp_le_gicov(x, threshold, gicov=None, *, layout=0, S=8, dist=CYCLIC, map
     if literal:
         rc = load().cudanp_le_gicov_literal(_ptr(x), _ptr(gicov), *(_ptr(t) for t in stats), N, L,
                                             threshold, layout, _stream(stream))
+    elif placement != GRAD_REGISTERS:
+        rc = load().cudanp_le_gicov_placement(_ptr(x), _ptr(gicov), *(_ptr(t) for t in stats), N, L,
+                                              threshold, layout, S, dist, map, placement,
+                                              _stream(stream))
     else:
         rc = load().cudanp_le_gicov(_ptr(x), _ptr(gicov), *(_ptr(t) for t in stats), N, L,
                                     threshold, layout, S, dist, map, _stream(stream))

@@ -83,3 +83,36 @@ def test_le_full_size_sampled():
         idx = torch.from_numpy(items).cuda()
         check((g[idx], a[idx], v[idx], e[idx]), ref, np.ascontiguousarray(sub.T), L, thr,
               f"full le S={S} d={d}")
+
+
+def test_le_grad_placements_bit_identical():
+    # Fig 6a/6b/6c: the home of Grad changes where loop 3 reads it, not the
+    # order a slave visits its elements -> bit-identical to the register
+    # partition, and within tolerance of the oracle
+    for N, L in [(1, 4), (35, 8), (300, 150), (1001, 150), (64, 1000), (8, 4096)]:
+        xi = synth.items(N, L, "f32_unit")
+        _, ra, rv, _ = O.le_gicov(xi, 0.0, 0)
+        with np.errstate(divide="ignore"):
+            thr = float(np.median(ra.astype(np.float64) ** 2 / rv))
+        ref = O.le_gicov(xi, thr, 0)
+        xd = dev(xi)
+        for S, d in itertools.product(INTRA_S, (C.CYCLIC, C.BLOCK)):
+            base = [host(t) for t in C.cudanp_le_gicov(xd, thr, S=S, dist=d, map=C.INTRA_WARP)]
+            check([torch.from_numpy(t) for t in base], ref, xi, L, thr, f"le regs N={N} L={L} S={S}")
+            for pl in (C.GRAD_SHARED, C.GRAD_GLOBAL):
+                got = [host(t) for t in C.cudanp_le_gicov(xd, thr, S=S, dist=d, map=C.INTRA_WARP,
+                                                            placement=pl)]
+                for gv, bv, name in zip(got, base, ("gicov", "ave", "var", "ep")):
+                    assert np.array_equal(gv.view(np.uint32), bv.view(np.uint32)), \
+                        f"placement {pl} N={N} L={L} S={S} d={d} {name}"
+    # point-major: the global placement for both maps; shared is item-major only
+    x = np.ascontiguousarray(synth.items(200, 150, "f32_unit").T)
+    xd = dev(x)
+    for m in (C.INTRA_WARP, C.INTER_WARP):
+        base = [host(t) for t in C.cudanp_le_gicov(xd, 0.02, layout=1, S=8, map=m)]
+        got = [host(t) for t in C.cudanp_le_gicov(xd, 0.02, layout=1, S=8, map=m, placement=C.GRAD_GLOBAL)]
+        for gv, bv in zip(got, base):
+            assert np.array_equal(gv.view(np.uint32), bv.view(np.uint32))
+    with pytest.raises(C.CudanpError) as ei:
+        C.cudanp_le_gicov(xd, 0.02, layout=1, S=8, placement=C.GRAD_SHARED)
+    assert ei.value.status == C.ERR_UNSUPPORTED
