@@ -21,6 +21,11 @@
  * memory across them; supported by the reduce, scan, MV and ragged-reduce
  * calls with CUDANP_MAP_AUTO / CUDANP_MAP_INTRA_WARP, and by TMV with the
  * inter-warp map for S <= 128 (CUDANP_ERR_UNSUPPORTED otherwise).
+ * S in {2048, 4096, 8192} (batched reduce only; CUDANP_ERR_INVALID for the
+ * other calls): a team larger than a CTA, one thread-block cluster of 8 CTAs
+ * of S/8 threads per item; the CTAs' partials meet in the master CTA's shared
+ * memory over DSMEM (the inter-warp smem exchange of P:203/P:209 one level
+ * up, np_cluster.cu).  For few outer items with very long loops.
  *
  * Conventions for every call:
  *  - Data pointers are DEVICE pointers owned by the caller; the library never
@@ -37,7 +42,9 @@
  *  - N = 0 or L = 0 is valid: reduce writes init (or the identity) for each
  *    item, scan writes nothing, TMV/MV write 0 when the inner count is 0.
  *  - Misaligned pointers or leading dimensions that are not multiples of 4
- *    are not errors; they take the scalar (non-128-bit) path.
+ *    are not errors; they take the scalar (non-128-bit) path, except the
+ *    intra-warp batched reduce, which peels each row to its 16-byte boundary
+ *    and streams the rest in 128-bit units.
  */
 #ifndef CUDANP_H_
 #define CUDANP_H_

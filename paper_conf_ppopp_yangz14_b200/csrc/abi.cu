@@ -86,9 +86,12 @@ static bool size_ok(int64_t a, int64_t b) {  // a*b*4 bytes addressable
   return a <= (INT64_MAX / 8) / b;
 }
 
-static int check_common(int S, int dist, int map, int64_t n_outer, int64_t n_inner) {
-  if (!valid_S(S) && !valid_big_S(S))
-    return fail_invalid("S must be one of 1,2,4,8,16,32 (or 64..1024 for multi-warp teams)");
+static int check_common(int S, int dist, int map, int64_t n_outer, int64_t n_inner,
+                        bool cluster_ok = false) {
+  if (!valid_S(S) && !valid_big_S(S) && !(cluster_ok && valid_cluster_S(S)))
+    return fail_invalid(cluster_ok ? "S must be one of 1,2,4,8,16,32 (64..1024 multi-warp teams, "
+                                     "2048/4096/8192 cluster teams)"
+                                   : "S must be one of 1,2,4,8,16,32 (or 64..1024 for multi-warp teams)");
   if (dist != CUDANP_DIST_CYCLIC && dist != CUDANP_DIST_BLOCK) return fail_invalid("dist");
   if (map != CUDANP_MAP_AUTO && map != CUDANP_MAP_INTRA_WARP && map != CUDANP_MAP_INTER_WARP)
     return fail_invalid("map");
@@ -298,8 +301,8 @@ int cudanp_mv(const float* A, int64_t lda, const float* x, float* y, int64_t n_o
 // out_per_item: reduce writes one value per item even when L = 0; scan
 // writes N*L values, so out may be NULL when L = 0.
 static int check_batched(const void* in, void* out, int64_t N, int64_t L, int S, int dist, int map,
-                         int dtype, int op, bool out_per_item) {
-  int rc = check_common(S, dist, map, N, L);
+                         int dtype, int op, bool out_per_item, bool cluster_ok = false) {
+  int rc = check_common(S, dist, map, N, L, cluster_ok);
   if (rc) return rc;
   rc = check_dtype_op(dtype, op);
   if (rc) return rc;
@@ -333,7 +336,7 @@ int cudanp_batched_loop_reduce(const void* in, const void* init, void* out, int6
   if (map == CUDANP_MAP_INTRA_WARP_TMA)
     return cudanp_batched_loop_reduce_tma(in, init, out, n_outer, n_inner, dtype, op, S, dist, 0, 0,
                                           stream);
-  int rc = check_batched(in, out, n_outer, n_inner, S, dist, map, dtype, op, true);
+  int rc = check_batched(in, out, n_outer, n_inner, S, dist, map, dtype, op, true, true);
   if (rc) return rc;
   const bool vec = (n_inner % 4 == 0) && aligned16(in);
   return reduce_np(in, init, out, n_outer, n_inner, dtype, op, S, dist, resolve_map(map, false),
@@ -517,7 +520,7 @@ int cudanp_dp_memcopy(const float* in, float* out, int64_t total, int64_t m, int
 int cudanp_launch_info(int op_kind, int64_t n_outer, int64_t n_inner, int dtype, int op, int S,
                        int dist, int map, int vec4, int* block_threads, int64_t* grid_ctas,
                        int* regs_per_thread, int* smem_bytes, int* resolved_map) {
-  int rc = check_common(S, dist, map, n_outer, n_inner);
+  int rc = check_common(S, dist, map, n_outer, n_inner, op_kind == 2);
   if (rc) return rc;
   LaunchInfo info;
   const bool v = vec4 != 0;

@@ -60,12 +60,28 @@ struct SegShare {
 };
 
 // ---------------------------------------------------------------- intra-warp
-template <class T, class Op, int S, int DIST, int KT = kRaggedK>
+// K consecutive warp tiles per warp step.  The step is written in three
+// phases so that nothing waits on a round trip it does not need: (1) the
+// masters' sequential sections for all K items issue their bound loads
+// together; (2) the bounds are broadcast and every slave works
+// out its share; (3) all head/tail scalars and the body's first units are in
+// flight before the first use.  A per-item version (load bounds, shfl, load
+// head, ...) paid K dependent round trips per step and ran short segments at
+// a third of the tuned S=1 rate.
+//
+// UNI: every item has the same trip count L and starts at n*L (the batched
+// reduce when its rows are not 16-byte aligned, L % 4 != 0): the bounds are
+// uniform index math, recomputed by every slave instead of loaded and
+// broadcast, and the same head/body/tail peeling gives each row
+// 128-bit body loads.
+template <class T, class Op, int S, int DIST, int KT = kRaggedK, bool UNI = false>
 __global__ void __launch_bounds__(kRaggedBlock)
 ragged_intra_kernel(const T* __restrict__ in, const int64_t* __restrict__ off,
-                    const T* __restrict__ init, T* __restrict__ out, int64_t N) {
+                    const T* __restrict__ init, T* __restrict__ out, int64_t N, int64_t L) {
+  pdl_entry();
   constexpr int TPW = 32 / S;
   constexpr int K = KT;
+  constexpr int HM = (3 + S - 1) / S;  // head (or tail) scalars per slave, at most
   const IntraTeam<S> team;
   const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
@@ -73,7 +89,19 @@ ragged_intra_kernel(const T* __restrict__ in, const int64_t* __restrict__ off,
   const T id = Op::template identity<T>();
 
   for (int64_t t0 = warp * K; t0 < ntiles; t0 += nwarps * K) {
-    int64_t item[K];
+    int64_t item[K], b[K], e[K];
+    // (1) Sequential section (master only): read the loop bounds.
+#pragma unroll
+    for (int k = 0; k < K; ++k) {
+      item[k] = (t0 + k) * TPW + team.team;
+      b[k] = 0; e[k] = 0;
+      if (UNI) {
+        if (item[k] < N) { b[k] = item[k] * L; e[k] = b[k] + L; }
+      } else if (team.is_master() && item[k] < N) {
+        b[k] = off[item[k]];
+        e[k] = off[item[k] + 1];
+      }
+    }
     const T* p[K];
     int64_t pstep[K];
     int cnt[K];
@@ -81,27 +109,27 @@ ragged_intra_kernel(const T* __restrict__ in, const int64_t* __restrict__ off,
     int trips = 0;
 #pragma unroll
     for (int k = 0; k < K; ++k) {
-      item[k] = (t0 + k) * TPW + team.team;
-      // Sequential section (master only): read the loop bounds ...
-      int64_t b0 = 0, l0 = 0;
-      if (team.is_master() && item[k] < N) {
-        b0 = off[item[k]];
-        l0 = off[item[k] + 1] - b0;
-        if (l0 < 0) l0 = 0;  // a decreasing offset pair is an empty loop
-      }
-      // ... and broadcast them to the slaves.
-      const int64_t b = team.read_from_master(b0);
-      const int64_t len = team.read_from_master(l0);
-      const SegShare<T, S, DIST> sh(in, b, len, team.slave);
+      // (2) ... broadcast them to the slaves.
+      const int64_t bk = UNI ? b[k] : team.read_from_master(b[k]);
+      int64_t len = (UNI ? e[k] : team.read_from_master(e[k])) - bk;
+      if (len < 0) len = 0;  // a decreasing offset pair is an empty loop
+      const SegShare<T, S, DIST> sh(in, bk, len, team.slave);
       p[k] = sh.body;
       pstep[k] = sh.step;
       cnt[k] = sh.cnt;
       trips = max(trips, sh.cnt);
-      // head and tail scalars (< 4 each), dealt over the first slaves
+      // (3) head and tail scalars (< 4 each), dealt over the first slaves
+      const T* tl = in + bk + sh.head + 4 * ((len - sh.head) >> 2);
+      T hv[HM], tv[HM];
+#pragma unroll
+      for (int j = 0; j < HM; ++j) {
+        const int i = team.slave + j * S;
+        hv[j] = i < sh.head ? ldg1(in + bk + i) : id;
+        tv[j] = i < sh.tail ? ldg1(tl + i) : id;
+      }
       part[k] = id;
-      for (int i = team.slave; i < sh.head; i += S) part[k] = Op::apply(part[k], in[b + i]);
-      const T* tl = in + b + sh.head + 4 * ((len - sh.head) >> 2);
-      for (int i = team.slave; i < sh.tail; i += S) part[k] = Op::apply(part[k], tl[i]);
+#pragma unroll
+      for (int j = 0; j < HM; ++j) part[k] = Op::apply(part[k], Op::apply(hv[j], tv[j]));
     }
     trips = (int)__reduce_max_sync(kFull, (unsigned)trips);  // warp-uniform trip count
     V4<T> acc[K];
@@ -273,7 +301,7 @@ static int launch_ragged(const T* in, const int64_t* off, const T* init, T* out,
     auto kern = few ? ragged_intra_kernel<T, Op, S, DIST, 1> : ragged_intra_kernel<T, Op, S, DIST, kRaggedK>;
     const int64_t per_cta = (kRaggedBlock / 32) * (few ? 1 : kRaggedK);
     const int64_t grid = persistent_grid(kern, kRaggedBlock, 0, (ntiles + per_cta - 1) / per_cta);
-    kern<<<(unsigned)grid, kRaggedBlock, 0, st>>>(in, off, init, out, N);
+    launch_pdl(kern, dim3((unsigned)grid), dim3(kRaggedBlock), 0, st, in, off, init, out, N, (int64_t)-1);
   } else {
     auto kern = ragged_inter_kernel<T, Op, S, DIST>;
     const int64_t grid = persistent_grid(kern, 32 * S, 0, (N + 31) / 32);
@@ -310,6 +338,49 @@ int ragged_np(const void* in, const int64_t* off, const void* init, void* out, i
                             : dispatch_ragged_t<float, OpMax>(in, off, init, out, N, S, dist, map, st);
   return op == CUDANP_SUM ? dispatch_ragged_t<int32_t, OpSum>(in, off, init, out, N, S, dist, map, st)
                           : dispatch_ragged_t<int32_t, OpMax>(in, off, init, out, N, S, dist, map, st);
+}
+
+// Batched reduce with rows that are not 16-byte aligned (L % 4 != 0 or a
+// misaligned base): the UNI form of the intra-warp kernel above.
+template <class T, class Op, int S, int DIST>
+static int launch_uniform_peel(const T* in, const T* init, T* out, int64_t N, int64_t L,
+                               cudaStream_t st, LaunchInfo* info) {
+  constexpr int TPW = 32 / S;
+  const int64_t ntiles = (N + TPW - 1) / TPW;
+  const bool few = few_tiles(ragged_intra_kernel<T, Op, S, DIST, kRaggedK, true>, kRaggedBlock, ntiles, kRaggedK);
+  auto kern = few ? ragged_intra_kernel<T, Op, S, DIST, 1, true> : ragged_intra_kernel<T, Op, S, DIST, kRaggedK, true>;
+  const int64_t per_cta = (kRaggedBlock / 32) * (few ? 1 : kRaggedK);
+  const int64_t grid = persistent_grid(kern, kRaggedBlock, 0, (ntiles + per_cta - 1) / per_cta);
+  if (info) {
+    info->block_threads = kRaggedBlock; info->grid = grid; info->map = MAP_INTRA;
+    kernel_attrs(kern, &info->regs, &info->smem);
+    return CUDANP_OK;
+  }
+  if (N == 0) return CUDANP_OK;
+  launch_pdl(kern, dim3((unsigned)grid), dim3(kRaggedBlock), 0, st, in, (const int64_t*)nullptr, init, out, N, L);
+  return check_launch("batched_loop_reduce (peeled rows) launch");
+}
+
+template <class T, class Op>
+static int uniform_peel_t(const void* in, const void* init, void* out, int64_t N, int64_t L, int S,
+                          int dist, cudaStream_t st, LaunchInfo* info) {
+  const T* i = (const T*)in;
+  const T* ini = (const T*)init;
+  T* o = (T*)out;
+  CUDANP_DISPATCH_S(S, {
+    return dist == DIST_CYCLIC ? launch_uniform_peel<T, Op, kS, DIST_CYCLIC>(i, ini, o, N, L, st, info)
+                               : launch_uniform_peel<T, Op, kS, DIST_BLOCK>(i, ini, o, N, L, st, info);
+  });
+  return CUDANP_OK;
+}
+
+int reduce_uniform_peel(const void* in, const void* init, void* out, int64_t N, int64_t L, int dtype,
+                        int op, int S, int dist, cudaStream_t st, LaunchInfo* info) {
+  if (dtype == CUDANP_F32)
+    return op == CUDANP_SUM ? uniform_peel_t<float, OpSum>(in, init, out, N, L, S, dist, st, info)
+                            : uniform_peel_t<float, OpMax>(in, init, out, N, L, S, dist, st, info);
+  return op == CUDANP_SUM ? uniform_peel_t<int32_t, OpSum>(in, init, out, N, L, S, dist, st, info)
+                          : uniform_peel_t<int32_t, OpMax>(in, init, out, N, L, S, dist, st, info);
 }
 
 int ragged_literal(const void* in, const int64_t* off, const void* init, void* out, int64_t N,

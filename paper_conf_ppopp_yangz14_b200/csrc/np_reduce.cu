@@ -305,13 +305,24 @@ static int dispatch_reduce_t(const void* in, const void* init, void* out, int64_
 int reduce_multi(const void*, const void*, void*, int64_t, int64_t, int, int, int, int, bool,
                  cudaStream_t, LaunchInfo*);
 
+int reduce_uniform_peel(const void*, const void*, void*, int64_t, int64_t, int, int, int, int,
+                        cudaStream_t, LaunchInfo*);
+int reduce_cluster(const void*, const void*, void*, int64_t, int64_t, int, int, int, int, bool,
+                   cudaStream_t, LaunchInfo*);
+
 int reduce_np(const void* in, const void* init, void* out, int64_t N, int64_t L, int dtype, int op,
               int S, int dist, int map, bool vec, cudaStream_t st, LaunchInfo* info) {
+  // Rows that are not 16-byte aligned (L % 4 != 0, e.g. Table 1's L = 150):
+  // intra-warp teams peel each row to its 16-byte boundary and stream the
+  // body in 128-bit units (np_ragged.cu, UNI form) instead of scalar loads.
+  if (!vec && S <= 32 && map == MAP_INTRA && L > 0 && ((uintptr_t)in & 3) == 0)
+    return reduce_uniform_peel(in, init, out, N, L, dtype, op, S, dist, st, info);
   if (S > 32) {
     if (map == MAP_INTER) {
       set_error("a team of S > 32 is S/32 consecutive warps: intra-warp (consecutive) map only");
       return CUDANP_ERR_UNSUPPORTED;
     }
+    if (S > 1024) return reduce_cluster(in, init, out, N, L, dtype, op, S, dist, vec, st, info);
     return reduce_multi(in, init, out, N, L, dtype, op, S, dist, vec, st, info);
   }
   if (dtype == CUDANP_F32)

@@ -164,7 +164,8 @@ def test_reduce_parity(case):
 
 
 def test_reduce_scalar_path_misaligned():
-    # a base pointer off 16-byte alignment takes the scalar (V=1) path
+    # a base pointer off 16-byte alignment: intra-warp teams peel each row to
+    # its 16-byte boundary (head/body/tail), inter-warp teams take the scalar path
     N, L = 300, 64
     x = synth.items(N + 1, L, "i32_full").reshape(-1)
     xd = dev(x)
@@ -174,6 +175,32 @@ def test_reduce_scalar_path_misaligned():
     for S, dist, map_ in itertools.product(SS, DISTS, MAPS):
         assert_exact(host(C.cudanp_batched_loop_reduce(view, S=S, dist=dist, map=map_)), ref,
                      f"misaligned S={S} dist={dist} map={map_}")
+
+
+def test_reduce_peeled_rows_every_alignment():
+    """Rows not 16-byte aligned (L % 4 != 0, or a base off by 1-3 elements):
+    the intra-warp kernel peels a head of <= 3 elements, streams the aligned
+    body in 128-bit units and finishes a tail of <= 3; every head/tail length
+    and every (S, dist) against the oracle."""
+    for L in (1, 2, 3, 5, 6, 7, 13, 150, 151, 1023):
+        N = 203
+        x = synth.items(N + 1, L, "i32_full", seed=L).reshape(-1)
+        xf = synth.items(N + 1, L, "f32_int4", seed=L).reshape(-1)
+        xd, xfd = dev(x), dev(xf)
+        for sh in range(4):
+            if sh * 1 + N * L > x.size:
+                continue
+            ref = O.reduce(x[sh:sh + N * L].reshape(N, L))
+            ref_m = O.reduce(x[sh:sh + N * L].reshape(N, L), op=O.MAX)
+            ref_f = O.reduce(xf[sh:sh + N * L].reshape(N, L))
+            v, vf = xd[sh:sh + N * L].view(N, L), xfd[sh:sh + N * L].view(N, L)
+            for S, dist in itertools.product(SS, DISTS):
+                what = f"peel L={L} shift={sh} S={S} dist={dist}"
+                assert_exact(host(C.cudanp_batched_loop_reduce(v, S=S, dist=dist, map=C.INTRA_WARP)), ref, what)
+                assert_exact(host(C.cudanp_batched_loop_reduce(v, op=C.MAX, S=S, dist=dist, map=C.INTRA_WARP)),
+                             ref_m, what + " max")
+                assert_exact(host(C.cudanp_batched_loop_reduce(vf, S=S, dist=dist, map=C.INTRA_WARP)), ref_f,
+                             what + " f32 exact data")
 
 
 def test_reduce_int32_wrap_and_closed_forms():
@@ -599,6 +626,41 @@ def test_big_teams_parity():
             if S <= 128:
                 assert_exact(host(C.cudanp_tmv(dev(A), dev(xt), S=S, dist=dist)), O.tmv(A, xt),
                              f"tmv big S={S} h={h} w={w}")
+
+
+CLUSTER_S = (2048, 4096, 8192)
+
+
+def test_cluster_teams_parity():
+    """S > 1024: the team is a thread-block cluster of 8 CTAs (DSMEM partials
+    into the master CTA, one cluster barrier per item); more items than
+    resident clusters exercise the grid stride and the double-buffered slots."""
+    for N, L in [(1, 1), (3, 0), (5, 8193), (40, 20000), (2500, 96), (9, 65536 + 4)]:
+        x = synth.items(N, L, "i32_full", seed=L)
+        ini = synth.init(N, "i32_full", seed=N)
+        xd, inid = dev(x), dev(ini)
+        ref_s, ref_m = O.reduce(x, init=ini), O.reduce(x, op=O.MAX)
+        xf = synth.items(N, L, "f32_unit", seed=L)
+        xfd = dev(xf)
+        ref_f = O.reduce(xf)
+        for S, dist in itertools.product(CLUSTER_S, DISTS):
+            what = f"cluster S={S} N={N} L={L} dist={dist}"
+            assert_exact(host(C.cudanp_batched_loop_reduce(xd, inid, S=S, dist=dist)), ref_s, what)
+            assert_exact(host(C.cudanp_batched_loop_reduce(xd, op=C.MAX, S=S, dist=dist)), ref_m, what)
+            assert_rel(host(C.cudanp_batched_loop_reduce(xfd, S=S, dist=dist)), ref_f, L, what)
+            if L > 1:  # misaligned rows: scalar units
+                v = xd.view(-1)[1:].view(-1)[: N * (L - 1)].view(N, L - 1)
+                assert_exact(host(C.cudanp_batched_loop_reduce(v, S=S, dist=dist)),
+                             O.reduce(x.reshape(-1)[1:1 + N * (L - 1)].reshape(N, L - 1)), what + " misaligned")
+    with pytest.raises(C.CudanpError) as ei:
+        C.cudanp_batched_loop_reduce(dev(synth.items(4, 64, "i32_full")), S=2048, map=C.INTER_WARP)
+    assert ei.value.status == C.ERR_UNSUPPORTED
+    # cluster sizes are a reduce-only team shape: other calls reject them before launch
+    with pytest.raises(C.CudanpError) as ei:
+        C.cudanp_batched_loop_scan(dev(synth.items(4, 64, "i32_small")), S=2048)
+    assert ei.value.status == C.ERR_INVALID
+    i = C.cudanp_launch_info("reduce", 256, 65536, S=4096)
+    assert i["block_threads"] == 512 and i["grid_ctas"] % 8 == 0
 
 
 def test_launch_info_and_auto_map():

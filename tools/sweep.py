@@ -46,12 +46,27 @@ def emit(rec):
         OUT.flush()
 
 
-def time_ms(fn, reps=5, warm=2):
+_FLUSH = None
+
+
+def flush_l2():
+    """Read a buffer twice the 126 MB L2 so the next launch reads cold HBM.
+    (Reading, not writing: a write-flush leaves ~126 MB of dirty lines whose
+    write-back then competes with the timed kernel.)"""
+    global _FLUSH
+    if _FLUSH is None:
+        _FLUSH = torch.ones(64 << 20, dtype=torch.int32, device="cuda")
+    _FLUSH.max()
+
+
+def time_ms(fn, reps=5, warm=2, flush=False):
     st = torch.cuda.current_stream()
     for _ in range(warm):
         fn()
     ts = []
     for _ in range(reps):
+        if flush:
+            flush_l2()
         a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         a.record(st)
         fn()
@@ -405,11 +420,13 @@ def e9(Ls=(32, 64, 128)):
 
 
 def big():
-    """Teams larger than a warp (S = 64..1024) on the shapes that need them:
-    MV with few long rows (the Fig 14 axis: fixed width, growing height) and a
-    batched reduce over few long items."""
+    """Teams larger than a warp (S = 64..1024) and than a CTA (S = 2048..8192,
+    cluster teams, reduce only) on the shapes that need them: MV with few long
+    rows (the Fig 14 axis: fixed width, growing height) and a batched reduce
+    over few long items.  L2 is flushed before every timed launch (several of
+    these working sets fit the 126 MB L2)."""
     cases = [("mv", h, 65536) for h in (16, 64, 256, 1024, 4096)] + \
-            [("reduce", N, L) for N, L in ((256, 65536), (2048, 16384), (16384, 4096))]
+            [("reduce", N, L) for N, L in ((16, 1 << 22), (64, 1 << 20), (256, 262144), (2048, 16384), (16384, 4096))]
     for op, N, L in cases:
         if op == "mv":
             A = gen((N, L), "f32_unit")
@@ -422,9 +439,9 @@ def big():
             y = torch.empty(N, device="cuda")
             nb = 4 * N * L + 4 * N
             fn = lambda S, d: C.cudanp_batched_loop_reduce(A, None, y, S=S, dist=d, map=C.INTRA_WARP)  # noqa: E731
-        for S in C.SLAVE_SIZES + (64, 128, 256, 512, 1024):
+        for S in C.SLAVE_SIZES + (64, 128, 256, 512, 1024) + ((2048, 4096, 8192) if op == "reduce" else ()):
             for d in (C.CYCLIC, C.BLOCK):
-                med, mn = time_ms(lambda: fn(S, d))
+                med, mn = time_ms(lambda: fn(S, d), flush=True)
                 emit({"config": "BIG", "op": op, "dtype": "f32", "N": N, "L": L, "S": S, "dist": DN[d],
                       "map": "intra", "impl": "np", "t_median_us": round(med * 1e3, 2), "alg_bytes": nb,
                       "gbs": round(nb / (med * 1e-3) / 1e9, 1)})
