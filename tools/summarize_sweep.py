@@ -6,8 +6,19 @@ import json
 import sys
 
 
+def peak_gbs():
+    """The measured copy peak of this pod (MEASURED_PEAKS.json), else the survey's 6537."""
+    import os
+    p = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "MEASURED_PEAKS.json")
+    try:
+        return float(json.load(open(p))["hbm_gbs"])
+    except (OSError, KeyError, ValueError):
+        return 6537.0
+
+
 def main(path, out=None):
     recs = [json.loads(l) for l in open(path) if l.strip()]
+    PEAK = peak_gbs()
     special = [r for r in recs if r["config"] in ("F3", "E9")]
     recs = [r for r in recs if r["config"] not in ("F3", "E9")]
     groups = collections.OrderedDict()
@@ -37,9 +48,19 @@ def main(path, out=None):
         lines.append(
             f"| {cfg} | {op}{(' ' + opn) if opn else ''} | {dt} | {L} | "
             + " | ".join(f"{perS.get(S, float('nan')):.0f}" for S in (1, 2, 4, 8, 16, 32))
-            + f" | {b['S']},{b['dist']},{b['map']} | {b['gbs']:.0f} | {100 * b['gbs'] / 6537:.1f} | "
+            + f" | {b['S']},{b['dist']},{b['map']} | {b['gbs']:.0f} | {100 * b['gbs'] / PEAK:.1f} | "
             + f"{b.get('speedup_vs_s1_tuned', float('nan')):.2f}x | {vs('s1_literal')} | {vs('dp_block')} | "
             + (vs(dp_thr) if dp_thr else "—") + " |")
+    st = [r for r in recs if r["impl"] == "best_np" and "gbs_steady" in r]
+    if st:
+        lines += ["", f"Steady state (20 back-to-back launches per event pair; % of the {PEAK:.0f} GB/s copy peak)", "",
+                  "| config | op | dtype | L | best NP | single GB/s | steady GB/s | steady % | best S=1 | S=1 steady GB/s | NP/S=1 steady |",
+                  "|---|---|---|---|---|---|---|---|---|---|---|"]
+        for r in st:
+            lines.append(f"| {r['config']} | {r['op']}{(' ' + r['opname']) if r.get('opname') else ''} | {r['dtype']} | "
+                         f"{r['L']} | {r['S']},{r['dist']},{r['map']} | {r['gbs']:.0f} | {r['gbs_steady']:.0f} | "
+                         f"{100 * r['gbs_steady'] / PEAK:.1f} | {r['s1_steady']} | {r['gbs_s1_steady']:.0f} | "
+                         f"{r['speedup_vs_s1_steady']:.2f}x |")
     f3 = [r for r in special if r["config"] == "F3"]
     if f3:
         lines += ["", "F3 — Fig 1 memcopy (64M floats): impl, m parents x n children, GB/s", "",

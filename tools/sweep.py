@@ -76,6 +76,24 @@ def time_ms(fn, reps=5, warm=2, flush=False):
     return statistics.median(ts), min(ts)
 
 
+def steady_ms(fn, R=20, reps=5):
+    """Per-launch time of R back-to-back launches between one event pair: the
+    rate a pipeline of repeated calls sees (launch latency and the grid's
+    ramp/tail overlap the neighbouring launches through PDL)."""
+    for _ in range(3):
+        fn()
+    ts = []
+    for _ in range(reps):
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record()
+        for _ in range(R):
+            fn()
+        b.record()
+        b.synchronize()
+        ts.append(a.elapsed_time(b) / R)
+    return statistics.median(ts)
+
+
 def graph_time_ms(fns, reps=5):
     """Capture a CUDA graph calling every fn once; return per-launch time."""
     s = torch.cuda.Stream()
@@ -102,9 +120,11 @@ def graph_time_ms(fns, reps=5):
     return statistics.median(ts), min(ts)
 
 
-def sweep_np(cfg, op, nbytes, run, extra, s1_ref=None, literal=None, comps=(), maps=None):
+def sweep_np(cfg, op, nbytes, run, extra, s1_ref=None, literal=None, comps=(), maps=None, call=None):
     """run(S, dist, map) -> (median_ms, min_ms).  s1_ref: extra no-NP kernel
-    times (e.g. the TMA-staged S=1 TMV) that count toward "tuned S=1"."""
+    times (e.g. the TMA-staged S=1 TMV) that count toward "tuned S=1".
+    call(S, dist, map) -> a one-launch callable: the best NP and the best S=1
+    version are then also timed back to back (steady state)."""
     res = {}
     if maps is None:  # TMV and reduce also have TMA-staged kernels
         maps = (C.INTRA_WARP, C.INTER_WARP) + {"tmv": (C.INTER_WARP_TMA,),
@@ -134,11 +154,19 @@ def sweep_np(cfg, op, nbytes, run, extra, s1_ref=None, literal=None, comps=(), m
               "alg_bytes": nbytes, "gbs": round(nbytes / (t * 1e-3) / 1e9, 1),
               "speedup_of_best_np": round(t / res[best][0], 3)})
     bS, bd, bm = best
+    steady = {}
+    if call is not None:
+        best1 = min((k for k in res if k[0] == 1), key=lambda k: res[k][0])
+        tb, t1 = steady_ms(call(*best)), steady_ms(call(*best1))
+        steady = {"t_steady_us": round(tb * 1e3, 2), "gbs_steady": round(nbytes / (tb * 1e-3) / 1e9, 1),
+                  "s1_steady": f"{best1[0]},{DN[best1[1]]},{MN[best1[2]]}",
+                  "gbs_s1_steady": round(nbytes / (t1 * 1e-3) / 1e9, 1),
+                  "speedup_vs_s1_steady": round(t1 / tb, 3)}
     emit({"config": cfg, "op": op, **extra, "impl": "best_np", "S": bS, "dist": DN[bd], "map": MN[bm],
           "t_median_us": round(res[best][0] * 1e3, 2), "alg_bytes": nbytes,
           "gbs": round(nbytes / (res[best][0] * 1e-3) / 1e9, 1),
           "speedup_vs_s1_tuned": round(s1 / res[best][0], 3),
-          **({"speedup_vs_s1_literal": round(literal / res[best][0], 3)} if literal else {})})
+          **({"speedup_vs_s1_literal": round(literal / res[best][0], 3)} if literal else {}), **steady})
     return res, best
 
 
@@ -239,7 +267,8 @@ def c3(Ls=(32, 64, 128, 256, 80, 150)):
             sweep_np("C3", "reduce", nb,
                      lambda S, d, m: time_ms(lambda: C.cudanp_batched_loop_reduce(x, None, out, op=op, S=S, dist=d, map=m)),
                      {"dtype": "f32" if dtype == C.F32 else "i32", "opname": "sum" if op == C.SUM else "max",
-                      "N": N, "L": L}, literal=lit, comps=comps)
+                      "N": N, "L": L}, literal=lit, comps=comps,
+                     call=lambda S, d, m: (lambda: C.cudanp_batched_loop_reduce(x, None, out, op=op, S=S, dist=d, map=m)))
             del x, out
             torch.cuda.empty_cache()
 
@@ -261,7 +290,8 @@ def c4(Ls=(64, 128, 256, 512, 1024)):
                 lambda: C.cudanp_batched_loop_scan_variant(C.DP_THREAD, xp, None, op_), N, Np))
             sweep_np("C4", "scan", nb,
                      lambda S, d, m: time_ms(lambda: C.cudanp_batched_loop_scan(x, None, out, S=S, dist=d, map=m), reps=3),
-                     {"dtype": "f32" if dtype == C.F32 else "i32", "N": N, "L": L}, literal=lit, comps=comps)
+                     {"dtype": "f32" if dtype == C.F32 else "i32", "N": N, "L": L}, literal=lit, comps=comps,
+                     call=lambda S, d, m: (lambda: C.cudanp_batched_loop_scan(x, None, out, S=S, dist=d, map=m)))
             del x, out
             torch.cuda.empty_cache()
 
