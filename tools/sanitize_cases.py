@@ -65,6 +65,17 @@ def main():
             C.cudanp_ragged_loop_reduce(xr, off, S=S, dist=d)
             if S == 64:
                 C.cudanp_tmv(A, xt, S=S, dist=d, map=C.INTER_WARP, n_outer=70)
+    Xc = dev(synth.items(300, 97, "i32_small"))      # cluster teams: more items than clusters
+    Xcf = dev(synth.items(7, 5003, "f32_unit"))       # (grid stride, both slot buffers), L % 4 != 0
+    for S in (2048, 4096, 8192):
+        for d in (C.CYCLIC, C.BLOCK):
+            C.cudanp_batched_loop_reduce(Xc, None, S=S, dist=d)
+            C.cudanp_batched_loop_reduce(Xcf, None, op=C.MAX, S=S, dist=d)
+    Xp = dev(synth.items(70, 37, "i32_small").reshape(-1))  # peeled rows, every misalignment
+    for sh in range(4):
+        v = Xp[sh:sh + 69 * 37].view(69, 37)
+        for S in Ss:
+            C.cudanp_batched_loop_reduce(v, None, S=S, map=C.INTRA_WARP)
     At = dev(synth.matrix(600, 132, "f32_unit"))   # tall: the rings wrap several times
     xtt = dev(synth.vector(600))
     for S in (1, 2, 4, 8, 16, 32):  # TMA-staged TMV, auto and pinned shapes
