@@ -127,7 +127,7 @@ static int check_tmv_args(const float* A, int64_t lda, const float* x, float* y,
 
 static int check_mv_args(const float* A, int64_t lda, const float* x, float* y, int64_t h,
                          int64_t w, int S, int dist, int map) {
-  int rc = check_common(S, dist, map, h, w);
+  int rc = check_common(S, dist, map, h, w, true);
   if (rc) return rc;
   if (h > 0 && w > 0 && lda < w) return fail_invalid("lda < n_inner (MV row length)");
   if (!size_ok(h, lda)) return fail_invalid("h*lda overflows");
@@ -520,7 +520,7 @@ int cudanp_dp_memcopy(const float* in, float* out, int64_t total, int64_t m, int
 int cudanp_launch_info(int op_kind, int64_t n_outer, int64_t n_inner, int dtype, int op, int S,
                        int dist, int map, int vec4, int* block_threads, int64_t* grid_ctas,
                        int* regs_per_thread, int* smem_bytes, int* resolved_map) {
-  int rc = check_common(S, dist, map, n_outer, n_inner, op_kind == 2);
+  int rc = check_common(S, dist, map, n_outer, n_inner, op_kind == 1 || op_kind == 2);
   if (rc) return rc;
   LaunchInfo info;
   const bool v = vec4 != 0;

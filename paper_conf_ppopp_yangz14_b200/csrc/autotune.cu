@@ -30,12 +30,15 @@ static std::vector<Candidate> candidates(int op_kind) {
       for (int d = 0; d < 2; ++d) c.push_back({S, d, CUDANP_MAP_INTER_WARP_TMA});
     for (int S : {64, 128})
       for (int d = 0; d < 2; ++d) c.push_back({S, d, CUDANP_MAP_INTER_WARP});
-  } else {             // MV / reduce / scan: multi-warp teams (+ the TMA-staged reduce)
+  } else {             // MV / reduce / scan: multi-warp teams (+ the TMA-staged reduce, cluster teams)
     if (op_kind == 2)
       for (int S : small)
         for (int d = 0; d < 2; ++d) c.push_back({S, d, CUDANP_MAP_INTRA_WARP_TMA});
     for (int S : {64, 128, 256, 512, 1024})
       for (int d = 0; d < 2; ++d) c.push_back({S, d, CUDANP_MAP_INTRA_WARP});
+    if (op_kind <= 2)  // MV / reduce: cluster teams
+      for (int S : {2048, 4096, 8192})
+        for (int d = 0; d < 2; ++d) c.push_back({S, d, CUDANP_MAP_INTRA_WARP});
   }
   return c;
 }

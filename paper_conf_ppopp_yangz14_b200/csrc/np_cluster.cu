@@ -33,28 +33,74 @@ __device__ __forceinline__ V4<T> cop4(V4<T> a, V4<T> b) {
   return {Op::apply(a.x, b.x), Op::apply(a.y, b.y), Op::apply(a.z, b.z), Op::apply(a.w, b.w)};
 }
 
+// The cluster-wide team reduction of one item.  Every thread of the cluster
+// calls it with its partial p; the master (rank 0, thread 0) gets the team's
+// result in *res and true.  Level 1: shfl inside each warp; level 2:
+// the CTA's warps through shared memory; level 3: each CTA's partial
+// is stored into the master CTA's slot over DSMEM, one cluster barrier, and
+// the master folds the eight partials in rank order.  Slots are
+// double-buffered by item parity: slots [par] are rewritten two items later,
+// after the next cluster barrier, which rank 0 reaches only after reading
+// them.  wsum is double-buffered the same way, so a warp's write for item
+// i+1 never meets the master thread's read for item i even under CTA-barrier
+// reasoning alone (racecheck does not model the cluster barrier).  The first call waits on the arrive issued at kernel entry (a CTA may
+// touch another CTA's shared memory only once that CTA is known to run).
+template <class Op, int W, class T>
+__device__ __forceinline__ bool cluster_team_reduce(T p, T* wsum, T (*part)[kClusterCtas], T* master_part,
+                                                    int par, int rank, bool& started, T* res) {
+  cg::cluster_group cluster = cg::this_cluster();
+  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) p = Op::apply(p, __shfl_xor_sync(kFull, p, o));
+  wsum += par * W;
+  if (lane == 0) wsum[wid] = p;
+  if (!started) {  // CTA-uniform
+    asm volatile("barrier.cluster.wait.aligned;" ::: "memory");
+    started = true;
+  }
+  __syncthreads();
+  if (tid == 0) {
+    T c = wsum[0];
+#pragma unroll
+    for (int k = 1; k < W; ++k) c = Op::apply(c, wsum[k]);
+    master_part[par * kClusterCtas + rank] = c;
+  }
+  cluster.sync();  // release/acquire: every slot is visible to rank 0; wsum reusable
+  if (rank == 0 && tid == 0) {
+    T r = part[par][0];
+#pragma unroll
+    for (int k = 1; k < kClusterCtas; ++k) r = Op::apply(r, part[par][k]);
+    *res = r;
+    return true;
+  }
+  return false;
+}
+
+__device__ __forceinline__ void cluster_arrive_relaxed() {
+  asm volatile("barrier.cluster.arrive.relaxed.aligned;" ::: "memory");
+}
+__device__ __forceinline__ void cluster_wait() {
+  asm volatile("barrier.cluster.wait.aligned;" ::: "memory");
+}
+
+// ---------------------------------------------------------------- batched reduce
 template <class T, class Op, int S, int DIST, bool VEC>
-__global__ void __launch_bounds__(S / kClusterCtas)
+__global__ void __launch_bounds__(S / kClusterCtas, 4096 / S > 0 ? 4096 / S : 1)  // <= 128 registers
 reduce_cluster_kernel(const T* __restrict__ in, const T* __restrict__ init, T* __restrict__ out,
                       int64_t N, int64_t L) {
   pdl_entry();
   constexpr int CTA = S / kClusterCtas;
-  constexpr int W = CTA / 32;
-  __shared__ T wsum[W];
-  __shared__ T part[2][kClusterCtas];  // the master CTA's receive slots, double-buffered
+  __shared__ T wsum[2 * (CTA / 32)];
+  __shared__ T part[2][kClusterCtas];  // the master CTA's receive slots
   cg::cluster_group cluster = cg::this_cluster();
   const int rank = (int)cluster.block_rank();
-  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
-  const int slave = rank * CTA + tid;  // slave id within the cluster-wide team
+  const int slave = rank * CTA + threadIdx.x;  // slave id within the cluster-wide team
   const int64_t nunits = VEC ? (L >> 2) : L;
   const Range<S, DIST> r(nunits, L, VEC ? 4 : 1, slave);
   const int64_t cid = blockIdx.x / kClusterCtas, ncl = gridDim.x / kClusterCtas;
   const T id = Op::template identity<T>();
   T* master_part = cluster.map_shared_rank(&part[0][0], 0);
-  // A CTA may touch another CTA's shared memory only once that CTA is known
-  // to be running: arrive on the cluster barrier now, wait for it just before
-  // the first DSMEM store (the first item's loads overlap the wait).
-  asm volatile("barrier.cluster.arrive.relaxed.aligned;" ::: "memory");
+  cluster_arrive_relaxed();  // waited for before the first DSMEM store
   bool started = false;
   int par = 0;
   for (int64_t item = cid; item < N; item += ncl, par ^= 1) {
@@ -76,35 +122,71 @@ reduce_cluster_kernel(const T* __restrict__ in, const T* __restrict__ init, T* _
       if constexpr (VEC) acc = cop4<T, Op>(acc, ldg4(row + 4 * u));
       else acc.x = Op::apply(acc.x, ldg1(row + u));
     }
-    // Team reduction, level 1: shfl inside each warp ...
-    T p = Op::apply(Op::apply(acc.x, acc.y), Op::apply(acc.z, acc.w));
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) p = Op::apply(p, __shfl_xor_sync(kFull, p, o));
-    // ... level 2: the CTA's warps through shared memory ...
-    if (lane == 0) wsum[wid] = p;
-    if (!started) {  // CTA-uniform
-      asm volatile("barrier.cluster.wait.aligned;" ::: "memory");
-      started = true;
-    }
-    __syncthreads();
-    if (tid == 0) {
-      T c = wsum[0];
-#pragma unroll
-      for (int k = 1; k < W; ++k) c = Op::apply(c, wsum[k]);
-      // ... level 3: the CTA's partial into the master CTA's slot over DSMEM.
-      master_part[par * kClusterCtas + rank] = c;
-    }
-    cluster.sync();  // release/acquire: every slot is visible to rank 0; wsum reusable
-    if (rank == 0 && tid == 0) {  // the master finishes the item alone
-      T res = part[par][0];
-#pragma unroll
-      for (int k = 1; k < kClusterCtas; ++k) res = Op::apply(res, part[par][k]);
-      out[item] = init ? Op::apply(init[item], res) : res;
-    }
-    // Slots [par] are rewritten two items later, after the next cluster.sync,
-    // which rank 0 reaches only after reading them.
+    T res;
+    if (cluster_team_reduce<Op, CTA / 32>(Op::apply(Op::apply(acc.x, acc.y), Op::apply(acc.z, acc.w)),
+                                          wsum, part, master_part, par, rank, started, &res))
+      out[item] = init ? Op::apply(init[item], res) : res;  // the master finishes alone
   }
-  if (!started) asm volatile("barrier.cluster.wait.aligned;" ::: "memory");
+  if (!started) cluster_wait();
+}
+
+// ---------------------------------------------------------------- MV
+// y[i] = sum_j A[i*lda+j] x[j] with a cluster per row: MV with few, long rows
+// (the Fig 14 axis, taken to rows fewer than SMs).
+template <int S, int DIST, bool VEC>
+__global__ void __launch_bounds__(S / kClusterCtas, 4096 / S > 0 ? 4096 / S : 1)  // <= 128 registers
+mv_cluster_kernel(const float* __restrict__ A, int64_t lda, const float* __restrict__ x,
+                  float* __restrict__ y, int64_t h, int64_t w) {
+  pdl_entry();
+  constexpr int CTA = S / kClusterCtas;
+  __shared__ float wsum[2 * (CTA / 32)];
+  __shared__ float part[2][kClusterCtas];
+  cg::cluster_group cluster = cg::this_cluster();
+  const int rank = (int)cluster.block_rank();
+  const int slave = rank * CTA + threadIdx.x;
+  const int64_t nunits = VEC ? (w >> 2) : w;
+  const Range<S, DIST> r(nunits, w, VEC ? 4 : 1, slave);
+  const int64_t cid = blockIdx.x / kClusterCtas, ncl = gridDim.x / kClusterCtas;
+  float* master_part = cluster.map_shared_rank(&part[0][0], 0);
+  cluster_arrive_relaxed();
+  bool started = false;
+  int par = 0;
+  for (int64_t row = cid; row < h; row += ncl, par ^= 1) {
+    const float* a = A + row * lda;
+    V4<float> acc = {0.f, 0.f, 0.f, 0.f};
+    int64_t u = r.begin;
+    constexpr int U = 4;
+    for (; u + (U - 1) * r.step < r.end; u += U * r.step) {
+      V4<float> av[U], xv[U];
+#pragma unroll
+      for (int j = 0; j < U; ++j) {
+        const int64_t uu = u + j * r.step;
+        if constexpr (VEC) { av[j] = ldg4_stream(a + 4 * uu); xv[j] = ldg4(x + 4 * uu); }
+        else { av[j] = {ldg1(a + uu), 0.f, 0.f, 0.f}; xv[j] = {ldg1(x + uu), 0.f, 0.f, 0.f}; }
+      }
+#pragma unroll
+      for (int j = 0; j < U; ++j) {
+        acc.x = fmaf(av[j].x, xv[j].x, acc.x);
+        acc.y = fmaf(av[j].y, xv[j].y, acc.y);
+        acc.z = fmaf(av[j].z, xv[j].z, acc.z);
+        acc.w = fmaf(av[j].w, xv[j].w, acc.w);
+      }
+    }
+    for (; u < r.end; u += r.step) {
+      if constexpr (VEC) {
+        const V4<float> av = ldg4_stream(a + 4 * u), xv = ldg4(x + 4 * u);
+        acc.x = fmaf(av.x, xv.x, acc.x); acc.y = fmaf(av.y, xv.y, acc.y);
+        acc.z = fmaf(av.z, xv.z, acc.z); acc.w = fmaf(av.w, xv.w, acc.w);
+      } else {
+        acc.x = fmaf(ldg1(a + u), ldg1(x + u), acc.x);
+      }
+    }
+    float res;
+    if (cluster_team_reduce<OpSum, CTA / 32>((acc.x + acc.y) + (acc.z + acc.w), wsum, part, master_part,
+                                             par, rank, started, &res))
+      y[row] = res;
+  }
+  if (!started) cluster_wait();
 }
 
 #define CUDANP_DISPATCH_CLUSTER_S(S, ...)                      \
@@ -115,10 +197,9 @@ reduce_cluster_kernel(const T* __restrict__ in, const T* __restrict__ init, T* _
     default: return fail_invalid("S must be 2048, 4096 or 8192 for a cluster team"); \
   }
 
-template <class T>
-static int launch_cluster(void (*kern)(const T*, const T*, T*, int64_t, int64_t), int cta, int64_t N,
-                          cudaStream_t st, LaunchInfo* info, const T* in, const T* init, T* out,
-                          int64_t L) {
+template <typename... KArgs, typename... Args>
+static int launch_cluster(void (*kern)(KArgs...), int cta, int64_t N, cudaStream_t st,
+                          LaunchInfo* info, const char* what, Args... args) {
   cudaLaunchConfig_t cfg = {};
   cfg.blockDim = dim3(cta);
   cfg.dynamicSmemBytes = 0;
@@ -149,13 +230,13 @@ static int launch_cluster(void (*kern)(const T*, const T*, T*, int64_t, int64_t)
   }
   if (N == 0) return CUDANP_OK;
   cfg.gridDim = dim3((unsigned)(clusters * kClusterCtas));
-  cudaError_t e = cudaLaunchKernelEx(&cfg, kern, in, init, out, N, L);
+  cudaError_t e = cudaLaunchKernelEx(&cfg, kern, static_cast<KArgs>(args)...);
   if (e != cudaSuccess) {
-    set_error("batched_loop_reduce (cluster team) launch: %s", cudaGetErrorString(e));
+    set_error("%s: %s", what, cudaGetErrorString(e));
     cudaGetLastError();
     return CUDANP_ERR_CUDA;
   }
-  return check_launch("batched_loop_reduce (cluster team) launch");
+  return check_launch(what);
 }
 
 template <class T, class Op>
@@ -167,7 +248,8 @@ static int reduce_cluster_t(const void* in, const void* init, void* out, int64_t
         dist == DIST_CYCLIC
             ? (vec ? reduce_cluster_kernel<T, Op, kS, DIST_CYCLIC, true> : reduce_cluster_kernel<T, Op, kS, DIST_CYCLIC, false>)
             : (vec ? reduce_cluster_kernel<T, Op, kS, DIST_BLOCK, true> : reduce_cluster_kernel<T, Op, kS, DIST_BLOCK, false>);
-    return launch_cluster<T>(kern, CTA, N, st, info, (const T*)in, (const T*)init, (T*)out, L);
+    return launch_cluster(kern, CTA, N, st, info, "batched_loop_reduce (cluster team) launch",
+                          (const T*)in, (const T*)init, (T*)out, N, L);
   });
   return CUDANP_OK;
 }
@@ -179,6 +261,17 @@ int reduce_cluster(const void* in, const void* init, void* out, int64_t N, int64
                             : reduce_cluster_t<float, OpMax>(in, init, out, N, L, S, dist, vec, st, info);
   return op == CUDANP_SUM ? reduce_cluster_t<int32_t, OpSum>(in, init, out, N, L, S, dist, vec, st, info)
                           : reduce_cluster_t<int32_t, OpMax>(in, init, out, N, L, S, dist, vec, st, info);
+}
+
+int mv_cluster(const float* A, int64_t lda, const float* x, float* y, int64_t h, int64_t w, int S,
+               int dist, bool vec, cudaStream_t st, LaunchInfo* info) {
+  CUDANP_DISPATCH_CLUSTER_S(S, {
+    constexpr int CTA = kS / kClusterCtas;
+    auto kern = dist == DIST_CYCLIC ? (vec ? mv_cluster_kernel<kS, DIST_CYCLIC, true> : mv_cluster_kernel<kS, DIST_CYCLIC, false>)
+                                    : (vec ? mv_cluster_kernel<kS, DIST_BLOCK, true> : mv_cluster_kernel<kS, DIST_BLOCK, false>);
+    return launch_cluster(kern, CTA, h, st, info, "mv (cluster team) launch", A, lda, x, y, h, w);
+  });
+  return CUDANP_OK;
 }
 
 }  // namespace cudanp

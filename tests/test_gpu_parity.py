@@ -661,6 +661,12 @@ def test_cluster_teams_parity():
     assert ei.value.status == C.ERR_INVALID
     i = C.cudanp_launch_info("reduce", 256, 65536, S=4096)
     assert i["block_threads"] == 512 and i["grid_ctas"] % 8 == 0
+    # MV with a cluster per row (few long rows), exact data -> bit-exact
+    for h, w in [(1, 5), (3, 0), (16, 65536), (300, 1000), (7, 4099)]:
+        A = synth.matrix(h, w, "f32_int4", seed=w)
+        xm = synth.vector(w, "f32_int4")
+        for S, dist in itertools.product(CLUSTER_S, DISTS):
+            assert_exact(host(C.cudanp_mv(dev(A), dev(xm), S=S, dist=dist)), O.mv(A, xm), f"mv cluster S={S} h={h} w={w}")
 
 
 def test_launch_info_and_auto_map():

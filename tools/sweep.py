@@ -451,7 +451,7 @@ def e9(Ls=(32, 64, 128)):
 
 def big():
     """Teams larger than a warp (S = 64..1024) and than a CTA (S = 2048..8192,
-    cluster teams, reduce only) on the shapes that need them: MV with few long
+    cluster teams) on the shapes that need them: MV with few long
     rows (the Fig 14 axis: fixed width, growing height) and a batched reduce
     over few long items.  L2 is flushed before every timed launch (several of
     these working sets fit the 126 MB L2)."""
@@ -469,7 +469,7 @@ def big():
             y = torch.empty(N, device="cuda")
             nb = 4 * N * L + 4 * N
             fn = lambda S, d: C.cudanp_batched_loop_reduce(A, None, y, S=S, dist=d, map=C.INTRA_WARP)  # noqa: E731
-        for S in C.SLAVE_SIZES + (64, 128, 256, 512, 1024) + ((2048, 4096, 8192) if op == "reduce" else ()):
+        for S in C.SLAVE_SIZES + (64, 128, 256, 512, 1024, 2048, 4096, 8192):
             for d in (C.CYCLIC, C.BLOCK):
                 med, mn = time_ms(lambda: fn(S, d), flush=True)
                 emit({"config": "BIG", "op": op, "dtype": "f32", "N": N, "L": L, "S": S, "dist": DN[d],
