@@ -358,7 +358,7 @@ int cudanp_batched_loop_reduce_backend(const void* in, const void* init, void* o
 
 int cudanp_batched_loop_scan(const void* in, const void* init, void* out, int64_t n_outer,
                              int64_t n_inner, int dtype, int S, int dist, int map, void* stream) {
-  int rc = check_batched(in, out, n_outer, n_inner, S, dist, map, dtype, CUDANP_SUM, false);
+  int rc = check_batched(in, out, n_outer, n_inner, S, dist, map, dtype, CUDANP_SUM, false, true);
   if (rc) return rc;
   const bool vec = (n_inner % 4 == 0) && aligned16(in) && aligned16(out);
   return scan_np(in, init, out, n_outer, n_inner, dtype, S, dist, resolve_map(map, false), vec,
@@ -520,7 +520,7 @@ int cudanp_dp_memcopy(const float* in, float* out, int64_t total, int64_t m, int
 int cudanp_launch_info(int op_kind, int64_t n_outer, int64_t n_inner, int dtype, int op, int S,
                        int dist, int map, int vec4, int* block_threads, int64_t* grid_ctas,
                        int* regs_per_thread, int* smem_bytes, int* resolved_map) {
-  int rc = check_common(S, dist, map, n_outer, n_inner, op_kind == 1 || op_kind == 2);
+  int rc = check_common(S, dist, map, n_outer, n_inner, op_kind >= 1 && op_kind <= 3);
   if (rc) return rc;
   LaunchInfo info;
   const bool v = vec4 != 0;

@@ -35,7 +35,7 @@ inline bool valid_S(int S) {
 // (consecutive-thread) map, TMV with the inter-warp map for S <= 128.
 inline bool valid_big_S(int S) { return S == 64 || S == 128 || S == 256 || S == 512 || S == 1024; }
 
-// Teams larger than a CTA (batched reduce, MV): one thread-block cluster of 8
+// Teams larger than a CTA (batched reduce and scan, MV): one thread-block cluster of 8
 // CTAs of S/8 threads (np_cluster.cu).
 inline bool valid_cluster_S(int S) { return S == 2048 || S == 4096 || S == 8192; }
 

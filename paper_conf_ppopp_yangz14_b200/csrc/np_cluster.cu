@@ -28,6 +28,14 @@ namespace cudanp {
 
 constexpr int kClusterCtas = 8;  // portable cluster size
 
+template <class T>
+__device__ __forceinline__ T sum4(V4<T> v) {
+  return OpSum::apply(OpSum::apply(v.x, v.y), OpSum::apply(v.z, v.w));
+}
+// a - b, int32 wrapping modulo 2^32 (R13)
+__device__ __forceinline__ float tsub_c(float a, float b) { return a - b; }
+__device__ __forceinline__ int32_t tsub_c(int32_t a, int32_t b) { return (int32_t)((uint32_t)a - (uint32_t)b); }
+
 template <class T, class Op>
 __device__ __forceinline__ V4<T> cop4(V4<T> a, V4<T> b) {
   return {Op::apply(a.x, b.x), Op::apply(a.y, b.y), Op::apply(a.z, b.z), Op::apply(a.w, b.w)};
@@ -189,6 +197,141 @@ mv_cluster_kernel(const float* __restrict__ A, int64_t lda, const float* __restr
   if (!started) cluster_wait();
 }
 
+// ---------------------------------------------------------------- batched scan (block)
+// out[n*L+k] = init[n] + sum_{i<=k} in[n*L+i] with a cluster per item, block
+// distribution (R5): pass 1 sums each slave's chunk; the CTA scans its
+// threads' chunk sums (shfl per warp, shared memory across warps);
+// each CTA publishes its total in its own shared memory and, after one
+// cluster barrier, reads the totals of the lower ranks -- and the master
+// CTA's carry-in init[n], a live-in broadcast over DSMEM --
+// to get its offset; pass 2 re-reads the chunk and stores the running values
+// (every team member stores its own elements).  Only the block
+// distribution is built: a cyclic cluster-wide scan needs a cluster barrier
+// per round of S units.
+template <class T, int S, bool VEC>
+__global__ void __launch_bounds__(S / kClusterCtas, 4096 / S > 0 ? 4096 / S : 1)
+scan_cluster_kernel(const T* __restrict__ in, const T* __restrict__ init, T* __restrict__ out,
+                    int64_t N, int64_t L) {
+  pdl_entry();
+  constexpr int CTA = S / kClusterCtas;
+  constexpr int W = CTA / 32;
+  constexpr int V = VEC ? 4 : 1;
+  __shared__ T wsum[2][W];
+  __shared__ T tot[2];    // this CTA's total (read by higher ranks over DSMEM)
+  __shared__ T cin[2];    // the master CTA's carry-in (read by every rank)
+  __shared__ T off[2];    // this CTA's offset
+  cg::cluster_group cluster = cg::this_cluster();
+  const int rank = (int)cluster.block_rank();
+  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+  const int slave = rank * CTA + tid;
+  const int64_t nunits = VEC ? (L >> 2) : L;
+  const Range<S, DIST_BLOCK> r(nunits, L, V, slave);
+  const int64_t cid = blockIdx.x / kClusterCtas, ncl = gridDim.x / kClusterCtas;
+  cluster_arrive_relaxed();
+  bool started = false;
+  int par = 0;
+  for (int64_t item = cid; item < N; item += ncl, par ^= 1) {
+    const T* irow = in + item * L;
+    T* orow = out + item * L;
+    // pass 1: this slave's chunk sum (U loads in flight, then the adds)
+    constexpr int U = 8;
+    T csum = T(0);
+    int64_t u = r.begin;
+    for (; u + U <= r.end; u += U) {
+      T v[U];
+#pragma unroll
+      for (int j = 0; j < U; ++j) {
+        if constexpr (VEC) v[j] = sum4(ldg4(irow + 4 * (u + j)));
+        else v[j] = ldg1(irow + u + j);
+      }
+#pragma unroll
+      for (int j = 0; j < U; ++j) csum = OpSum::apply(csum, v[j]);
+    }
+    for (; u < r.end; ++u) {
+      if constexpr (VEC) csum = OpSum::apply(csum, sum4(ldg4(irow + 4 * u)));
+      else csum = OpSum::apply(csum, ldg1(irow + u));
+    }
+    // CTA-wide exclusive scan of the chunk sums
+    T incl = csum;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const T t = __shfl_up_sync(kFull, incl, o);
+      if (lane >= o) incl = OpSum::apply(incl, t);
+    }
+    if (lane == 31) wsum[par][wid] = incl;
+    if (!started) {  // CTA-uniform; see cluster_team_reduce
+      cluster_wait();
+      started = true;
+    }
+    __syncthreads();
+    T wpre = T(0), ctot = T(0);
+#pragma unroll 4
+    for (int k = 0; k < W; ++k) {
+      const T q = wsum[par][k];
+      if (k < wid) wpre = OpSum::apply(wpre, q);
+      ctot = OpSum::apply(ctot, q);
+    }
+    if (tid == 0) {
+      tot[par] = ctot;
+      if (rank == 0) cin[par] = init ? init[item] : T(0);  // the master's sequential section
+    }
+    cluster.sync();  // totals and carry-in visible cluster-wide
+    if (wid == 0) {  // offset = carry-in + totals of the lower ranks, over DSMEM
+      T v = T(0);
+      if (lane < rank) v = *cluster.map_shared_rank(&tot[par], lane);
+      if (lane == 31) v = *cluster.map_shared_rank(&cin[par], 0);
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) v = OpSum::apply(v, __shfl_xor_sync(kFull, v, o));
+      if (lane == 0) off[par] = v;
+    }
+    __syncthreads();
+    // pass 2: rescan the chunk from this slave's offset and store
+    T run = OpSum::apply(off[par], OpSum::apply(wpre, tsub_c(incl, csum)));
+    u = r.begin;
+    for (; u + U <= r.end; u += U) {
+      if constexpr (VEC) {
+        V4<T> v[U];
+#pragma unroll
+        for (int j = 0; j < U; ++j) v[j] = ldg4(irow + 4 * (u + j));
+#pragma unroll
+        for (int j = 0; j < U; ++j) {
+          v[j].x = OpSum::apply(run, v[j].x); v[j].y = OpSum::apply(v[j].x, v[j].y);
+          v[j].z = OpSum::apply(v[j].y, v[j].z); v[j].w = OpSum::apply(v[j].z, v[j].w);
+          stg4(orow + 4 * (u + j), v[j]);
+          run = v[j].w;
+        }
+      } else {
+        T v[U];
+#pragma unroll
+        for (int j = 0; j < U; ++j) v[j] = ldg1(irow + u + j);
+#pragma unroll
+        for (int j = 0; j < U; ++j) {
+          run = OpSum::apply(run, v[j]);
+          orow[u + j] = run;
+        }
+      }
+    }
+    for (; u < r.end; ++u) {
+      if constexpr (VEC) {
+        V4<T> v = ldg4(irow + 4 * u);
+        v.x = OpSum::apply(run, v.x); v.y = OpSum::apply(v.x, v.y);
+        v.z = OpSum::apply(v.y, v.z); v.w = OpSum::apply(v.z, v.w);
+        stg4(orow + 4 * u, v);
+        run = v.w;
+      } else {
+        run = OpSum::apply(run, ldg1(irow + u));
+        orow[u] = run;
+      }
+    }
+    // Slots [par] (own tot/cin read remotely, wsum, off) are rewritten two
+    // items later, after the next cluster barrier.
+  }
+  if (!started) cluster_wait();
+  // Other CTAs read this CTA's tot/cin after the last item's barrier: no CTA
+  // may exit (and release its shared memory) before they are done.
+  cluster.sync();
+}
+
 #define CUDANP_DISPATCH_CLUSTER_S(S, ...)                      \
   switch (S) {                                                 \
     case 2048: { constexpr int kS = 2048; __VA_ARGS__; } break; \
@@ -272,6 +415,30 @@ int mv_cluster(const float* A, int64_t lda, const float* x, float* y, int64_t h,
     return launch_cluster(kern, CTA, h, st, info, "mv (cluster team) launch", A, lda, x, y, h, w);
   });
   return CUDANP_OK;
+}
+
+template <class T>
+static int scan_cluster_t(const void* in, const void* init, void* out, int64_t N, int64_t L, int S,
+                          bool vec, cudaStream_t st, LaunchInfo* info) {
+  CUDANP_DISPATCH_CLUSTER_S(S, {
+    constexpr int CTA = kS / kClusterCtas;
+    auto kern = vec ? scan_cluster_kernel<T, kS, true> : scan_cluster_kernel<T, kS, false>;
+    if (!info && (N == 0 || L == 0)) return CUDANP_OK;
+    return launch_cluster(kern, CTA, N, st, info, "batched_loop_scan (cluster team) launch",
+                          (const T*)in, (const T*)init, (T*)out, N, L);
+  });
+  return CUDANP_OK;
+}
+
+int scan_cluster(const void* in, const void* init, void* out, int64_t N, int64_t L, int dtype, int S,
+                 int dist, bool vec, cudaStream_t st, LaunchInfo* info) {
+  if (dist != DIST_BLOCK) {
+    set_error("a cluster-team scan is built for the block distribution only (a cyclic "
+              "cluster-wide scan needs a cluster barrier per round of S units)");
+    return CUDANP_ERR_UNSUPPORTED;
+  }
+  return dtype == CUDANP_F32 ? scan_cluster_t<float>(in, init, out, N, L, S, vec, st, info)
+                             : scan_cluster_t<int32_t>(in, init, out, N, L, S, vec, st, info);
 }
 
 }  // namespace cudanp

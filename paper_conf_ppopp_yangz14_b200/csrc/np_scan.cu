@@ -307,6 +307,8 @@ static int dispatch_scan_t(const void* in, const void* init, void* out, int64_t 
   return CUDANP_OK;
 }
 
+int scan_cluster(const void*, const void*, void*, int64_t, int64_t, int, int, int, bool, cudaStream_t,
+                 LaunchInfo*);
 int scan_multi(const void*, const void*, void*, int64_t, int64_t, int, int, int, bool, cudaStream_t,
                LaunchInfo*);
 
@@ -317,6 +319,7 @@ int scan_np(const void* in, const void* init, void* out, int64_t N, int64_t L, i
       set_error("a team of S > 32 is S/32 consecutive warps: intra-warp (consecutive) map only");
       return CUDANP_ERR_UNSUPPORTED;
     }
+    if (S > 1024) return scan_cluster(in, init, out, N, L, dtype, S, dist, vec, st, info);
     return scan_multi(in, init, out, N, L, dtype, S, dist, vec, st, info);
   }
   if (dtype == CUDANP_F32) return dispatch_scan_t<float>(in, init, out, N, L, S, dist, map, vec, st, info);

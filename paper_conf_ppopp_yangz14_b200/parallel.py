@@ -16,17 +16,30 @@ def shard(n_outer: int, world: int, rank: int) -> tuple[int, int]:
     return C.cudanp_shard_range(n_outer, world, rank)
 
 
-def gather_to_root(local, root_buf, n_total: int, rank: int, world: int, root: int = 0):
+def gather_to_root(local, root_buf, n_total: int, rank: int, world: int, root: int = 0,
+                   async_op: bool = False):
     """Grouped point-to-point gather (NCCL has no gather primitive): every rank
     sends its shard, the root receives shard g into root_buf[begin_g:end_g].
-    Shards may be uneven.  Returns root_buf on the root, None elsewhere."""
+    Shards may be uneven.  Returns root_buf on the root, None elsewhere; with
+    async_op=True returns the list of pending works instead (the caller waits
+    on them -- on NCCL that only orders its current stream after the
+    transfers -- before it reuses `local` or reads root_buf), so the gather of
+    one op's outputs can overlap the next op's kernel."""
     import torch.distributed as dist
     b_me, e_me = shard(n_total, world, rank)
+    if world > 1 and local.is_cuda and dist.get_backend() == "gloo":
+        # test mode only (several ranks sharing one GPU, where NCCL refuses
+        # duplicate devices): gloo moves host memory, so stage through the host
+        cpu_root = root_buf.cpu() if rank == root else None
+        gather_to_root(local.cpu(), cpu_root, n_total, rank, world, root)
+        if rank == root:
+            root_buf.copy_(cpu_root)
+        return [] if async_op else (root_buf if rank == root else None)
     if local.shape[0] != e_me - b_me:
         raise ValueError(f"rank {rank}: local shard has {local.shape[0]} items, expected {e_me - b_me}")
     if world == 1:
         root_buf[b_me:e_me].copy_(local)
-        return root_buf
+        return [] if async_op else root_buf
     ops = []
     if rank == root:
         for g in range(world):
@@ -37,9 +50,11 @@ def gather_to_root(local, root_buf, n_total: int, rank: int, world: int, root: i
                 ops.append(dist.P2POp(dist.irecv, root_buf[b:e], g))
     elif e_me > b_me:
         ops.append(dist.P2POp(dist.isend, local.contiguous(), root))
-    if ops:
-        for r in dist.batch_isend_irecv(ops):
-            r.wait()
+    works = dist.batch_isend_irecv(ops) if ops else []
+    if async_op:
+        return works
+    for r in works:
+        r.wait()
     return root_buf if rank == root else None
 
 

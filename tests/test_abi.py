@@ -56,15 +56,15 @@ def test_bad_slave_size_rejected_before_launch(lib, S):
 
 
 @pytest.mark.parametrize("S", [2048, 4096, 8192])
-def test_cluster_team_sizes_are_reduce_and_mv_only(lib, S):
-    # cluster teams (S > 1024) pass the reduce's and MV's S check (then fail on
-    # the NULL pointers) and are rejected by the other calls, before any launch
+def test_cluster_team_sizes_are_reduce_scan_mv_only(lib, S):
+    # cluster teams (S > 1024) pass the reduce's, scan's and MV's S check (then
+    # fail on the NULL pointers) and are rejected by TMV, before any launch
     assert lib.cudanp_batched_loop_reduce(None, None, None, 10, 10, 0, 0, S, 0, 0, None) == C.ERR_INVALID
     assert "S must be" not in lib.cudanp_last_error().decode()
     assert lib.cudanp_mv(None, 4, None, None, 4, 4, S, 0, 0, None) == C.ERR_INVALID
     assert "S must be" not in lib.cudanp_last_error().decode()
     assert lib.cudanp_batched_loop_scan(None, None, None, 10, 10, 0, S, 0, 0, None) == C.ERR_INVALID
-    assert "S must be" in lib.cudanp_last_error().decode()
+    assert "S must be" not in lib.cudanp_last_error().decode()
     assert lib.cudanp_tmv(None, 4, None, None, 4, 4, S, 0, 0, None) == C.ERR_INVALID
     assert "S must be" in lib.cudanp_last_error().decode()
 

@@ -45,7 +45,15 @@ def _worker(rank, world, port, q):
         items = synth.items(e - b, L, "i32_full", n0=b)
         r_local = torch.from_numpy(O.reduce(items))
         r_root = torch.empty(N, dtype=torch.int32) if rank == 0 else None
-        P.gather_to_root(r_local, r_root, N, rank, world)
+        # asynchronous form (bench.py overlaps the TMV gather with the MV kernel):
+        # two gathers in flight, then wait on every pending work
+        works = P.gather_to_root(r_local, r_root, N, rank, world, async_op=True)
+        r2_root = torch.empty(N, dtype=torch.int32) if rank == 0 else None
+        works += P.gather_to_root(r_local, r2_root, N, rank, world, async_op=True)
+        for wk in works:
+            wk.wait()
+        if rank == 0:
+            assert torch.equal(r_root, r2_root)
         if rank == 0:
             q.put((root.numpy().copy(), r_root.numpy().copy()))
     finally:

@@ -456,7 +456,8 @@ def big():
     over few long items.  L2 is flushed before every timed launch (several of
     these working sets fit the 126 MB L2)."""
     cases = [("mv", h, 65536) for h in (16, 64, 256, 1024, 4096)] + \
-            [("reduce", N, L) for N, L in ((16, 1 << 22), (64, 1 << 20), (256, 262144), (2048, 16384), (16384, 4096))]
+            [("reduce", N, L) for N, L in ((16, 1 << 22), (64, 1 << 20), (256, 262144), (2048, 16384), (16384, 4096))] + \
+            [("scan", N, L) for N, L in ((16, 1 << 22), (256, 262144))]
     for op, N, L in cases:
         if op == "mv":
             A = gen((N, L), "f32_unit")
@@ -464,18 +465,26 @@ def big():
             y = torch.empty(N, device="cuda")
             nb = 4 * N * L + 4 * N + 4 * L
             fn = lambda S, d: C.cudanp_mv(A, x, y, S=S, dist=d, map=C.INTRA_WARP)  # noqa: E731
-        else:
+        elif op == "reduce":
             A = gen((N, L), "f32_unit")
             y = torch.empty(N, device="cuda")
             nb = 4 * N * L + 4 * N
             fn = lambda S, d: C.cudanp_batched_loop_reduce(A, None, y, S=S, dist=d, map=C.INTRA_WARP)  # noqa: E731
+        else:
+            A = gen((N, L), "i32_small", torch.int32, B=1 << 15)
+            y = torch.empty_like(A)
+            nb = 8 * N * L
+            fn = lambda S, d: C.cudanp_batched_loop_scan(A, None, y, S=S, dist=d, map=C.INTRA_WARP)  # noqa: E731
         for S in C.SLAVE_SIZES + (64, 128, 256, 512, 1024, 2048, 4096, 8192):
             for d in (C.CYCLIC, C.BLOCK):
-                med, mn = time_ms(lambda: fn(S, d), flush=True)
-                emit({"config": "BIG", "op": op, "dtype": "f32", "N": N, "L": L, "S": S, "dist": DN[d],
+                try:
+                    med, mn = time_ms(lambda: fn(S, d), flush=True)
+                except C.CudanpError:
+                    continue  # e.g. the cluster-team scan is block-only
+                emit({"config": "BIG", "op": op, "dtype": "f32" if op != "scan" else "i32", "N": N, "L": L, "S": S, "dist": DN[d],
                       "map": "intra", "impl": "np", "t_median_us": round(med * 1e3, 2), "alg_bytes": nb,
                       "gbs": round(nb / (med * 1e-3) / 1e9, 1)})
-        del A
+        del A, y
         torch.cuda.empty_cache()
 
 
