@@ -298,10 +298,6 @@ def run_cudanp(args):
         C.cudanp_tmv(A_t, x_t, out_t, S=St, dist=dt, map=mt, n_outer=wt)
         if evs:
             evs[1].record(st)
-        # NCCL gather of the TMV outputs overlaps the MV kernel; both gathers
-        # are complete (stream-ordered) before the step ends
-        works = (P.gather_to_root(y_t, y_root, n * world, rank, world, async_op=True)
-                 if world > 1 and not fused and native is None else [])
         C.cudanp_mv(A_m, x_m, out_m, S=Sm, dist=dm, map=mm)
         if evs:
             evs[2].record(st)
@@ -309,6 +305,11 @@ def run_cudanp(args):
             native.gather(y_t, y_root, n * world)
             native.gather(y_m, ym_root, n * world)
         elif world > 1 and not fused:
+            # both gathers back to back on NCCL's stream, then one stream wait.
+            # They are not overlapped with the MV kernel on purpose: its
+            # persistent grid is sized to fill every SM, and an NCCL kernel
+            # holding part of one SM would push a CTA of it into a second wave.
+            works = P.gather_to_root(y_t, y_root, n * world, rank, world, async_op=True)
             works += P.gather_to_root(y_m, ym_root, n * world, rank, world, async_op=True)
             for wk in works:
                 wk.wait()
