@@ -103,3 +103,32 @@ def test_tmv_tma_random(h, w4, pad4, S, dist, seed):
     ref = O.tmv(A, x, w) if h else np.zeros(w, np.float32)
     got = host(C.cudanp_tmv(dev(A), dev(x), S=S, dist=dist, map=C.INTER_WARP_TMA, n_outer=w))
     assert_exact(got, ref, f"TMA h={h} w={w} lda={lda} S={S} dist={dist}")
+
+
+BIG_ = st.sampled_from([64, 128, 256, 512, 1024, 2048, 4096, 8192])
+
+
+@settings(max_examples=80, deadline=None, suppress_health_check=list(HealthCheck))
+@given(N=st.integers(0, 300), L=st.integers(0, 20000), S=BIG_, dist=D_, shift=st.integers(0, 3),
+       use_init=st.booleans(), seed=st.integers(0, 10**6))
+def test_big_and_cluster_teams_random(N, L, S, dist, shift, use_init, seed):
+    """Teams larger than a warp (S/32 warps) and than a CTA (a cluster of 8
+    CTAs): reduce (sum and max), scan (the cluster scan is block-only) and MV."""
+    x = synth.gen(1, "i32_small", 0, N * L + shift, B=1 << 15, seed=seed)
+    xd = dev(x)[shift:].view(N, L) if N * L else dev(x)[: 0].view(N, L)
+    xs = x[shift:].reshape(N, L)
+    ini = synth.init(N, "i32_small", B=1 << 15, seed=seed)
+    inid = dev(ini) if use_init and N else None
+    what = f"N={N} L={L} S={S} dist={dist} shift={shift} init={use_init}"
+    assert_exact(host(C.cudanp_batched_loop_reduce(xd, inid, S=S, dist=dist)),
+                 O.reduce(xs, init=ini if use_init else None), "reduce " + what)
+    assert_exact(host(C.cudanp_batched_loop_reduce(xd, None, op=C.MAX, S=S, dist=dist)),
+                 O.reduce(xs, op=O.MAX), "reduce max " + what)
+    if S <= 1024 or dist == C.BLOCK:
+        assert_exact(host(C.cudanp_batched_loop_scan(xd, inid, S=S, dist=dist)),
+                     O.scan(xs, init=ini if use_init else None), "scan " + what)
+    if N and L:
+        h, w = min(N, 64), min(L, 5000)
+        A = synth.matrix(h, w, "f32_int4", seed=seed)
+        xm = synth.vector(w, "f32_int4", seed=seed)
+        assert_exact(host(C.cudanp_mv(dev(A), dev(xm), S=S, dist=dist)), O.mv(A, xm), "mv " + what)
