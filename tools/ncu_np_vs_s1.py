@@ -52,6 +52,10 @@ CASES = [
     ("C4 scan 2M×256 i32", "S=1 inter (no NP)", "--op scan --N 2097152 --L 256 --dtype i32 --S 1 --dist block --map inter", "scan_"),
     ("C4 scan 2M×256 i32", "literal", "--op scan_literal --N 2097152 --L 256 --dtype i32", "scan_"),
     ("C4 scan 2M×256 i32", "NP S=16 cyclic intra", "--op scan --N 2097152 --L 256 --dtype i32 --S 16 --dist cyclic --map intra", "scan_"),
+    ("F2 LE 2M×150 item-major", "literal Fig 5", "--op le_literal --N 2097152 --L 150 --layout 0", "le_"),
+    ("F2 LE 2M×150 item-major", "S=1 intra (no NP)", "--op le --N 2097152 --L 150 --layout 0 --S 1 --dist cyclic --map intra", "le_"),
+    ("F2 LE 2M×150 item-major", "NP S=8 cyclic intra", "--op le --N 2097152 --L 150 --layout 0 --S 8 --dist cyclic --map intra", "le_"),
+    ("F2 LE 2M×150 point-major", "NP S=5 block inter", "--op le --N 2097152 --L 150 --layout 1 --S 5 --dist block --map inter", "le_"),
     ("reduce 16×4M (few items)", "NP S=1024 (one CTA per item)", "--op reduce --N 16 --L 4194304 --S 1024", "reduce_"),
     ("reduce 16×4M (few items)", "NP S=4096 (cluster per item)", "--op reduce --N 16 --L 4194304 --S 4096", "reduce_"),
 ]

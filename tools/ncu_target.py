@@ -20,7 +20,7 @@ def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--op", required=True, choices=["tmv", "mv", "reduce", "scan", "tmv_literal",
                                                     "mv_literal", "reduce_literal", "scan_literal",
-                                                    "ragged", "le", "tmv_tma"])
+                                                    "ragged", "le", "le_literal", "tmv_tma"])
     ap.add_argument("--lens", default="uniform", help="ragged: length distribution")
     ap.add_argument("--layout", type=int, default=0, help="le: 0 item-major, 1 point-major")
     ap.add_argument("--S", type=int, default=8)
@@ -42,10 +42,11 @@ def main():
         C.cudanp_generate(X, "f32_unit")
         o1 = torch.empty(a.N, device="cuda")
         fns = {"ragged": lambda: C.cudanp_ragged_loop_reduce(X, off, None, o1, S=a.S, dist=d, map=m)}
-    elif a.op == "le":
+    elif a.op in ("le", "le_literal"):
         X = torch.empty(*((a.N, a.L) if a.layout == 0 else (a.L, a.N)), device="cuda")
         C.cudanp_generate(X, "f32_unit")
-        fns = {"le": lambda: C.cudanp_le_gicov(X, 0.02, layout=a.layout, S=a.S, dist=d, map=m)}
+        fns = {"le": lambda: C.cudanp_le_gicov(X, 0.02, layout=a.layout, S=a.S, dist=d, map=m),
+               "le_literal": lambda: C.cudanp_le_gicov(X, 0.02, layout=a.layout, literal=True)}
     elif a.op.startswith(("tmv", "mv")):
         A = torch.empty(a.n, a.n, device="cuda")
         C.cudanp_generate(A, "f32_unit")
