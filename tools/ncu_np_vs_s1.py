@@ -61,10 +61,12 @@ CASES = [
 ]
 
 
-def run(out):
+def run(out, only=None):
     os.makedirs(out, exist_ok=True)
     mlist = ",".join(m for m, _, _ in METRICS)
     for i, (cfg, label, args, rx) in enumerate(CASES):
+        if only and only not in cfg:
+            continue
         log = os.path.join(out, f"case{i:02d}.csv")
         cmd = (f"ncu --metrics {mlist} --clock-control none --csv --log-file {log} -k regex:{rx} -s 1 -c 1 "
                f"{sys.executable} {os.path.join(ROOT, 'tools', 'ncu_target.py')} {args} --reps 2")
@@ -131,5 +133,6 @@ if __name__ == "__main__":
     ap.add_argument("mode", choices=["run", "summarize"])
     ap.add_argument("--out", default=os.path.join(ROOT, "gpurun_out", "npvs1"))
     ap.add_argument("--md", default=os.path.join(ROOT, "profiles", "ncu_np_vs_s1.md"))
+    ap.add_argument("--only", default=None, help="run: configs containing this substring")
     a = ap.parse_args()
-    run(a.out) if a.mode == "run" else summarize(a.out, a.md)
+    run(a.out, a.only) if a.mode == "run" else summarize(a.out, a.md)
