@@ -69,8 +69,9 @@ le_tma_kernel(const float* __restrict__ in, float* gicov, float* ave_out, float*
   }
 
   constexpr int TPW = 32 / S;
+  constexpr int HM = (3 + S - 1) / S;
   const IntraTeam<S> team;
-  const Range<S, DIST> r(L, L, 1, team.slave);  // uniform per slave
+  const int sl = team.slave;
   for (int64_t t = 0; t < mine; ++t) {
     const int st = (int)(t % stages);
     const int64_t n0 = ((int64_t)blockIdx.x + t * gridDim.x) * ips;
@@ -82,17 +83,44 @@ le_tma_kernel(const float* __restrict__ in, float* gicov, float* ave_out, float*
       const int il = tile * TPW + team.team;
       const bool ok = il < cnt;
       const float* Grad = base + (int64_t)(ok ? il : 0) * L;  // DEF_Grad (Fig 6b)
-      const int64_t e = ok ? r.end : r.begin;
-      float sum = 0.f;
-      for (int64_t i = r.begin; i < e; i += r.step) sum += Grad[i];  // loops 1+2
+      // The register version's element order (np_le.cu LeSlaveV): head up to
+      // the row's 16-byte boundary (global and shared offsets agree: every
+      // run starts 16-byte aligned), 128-bit body units, tail.
+      const int64_t Lr = ok ? L : 0;
+      int64_t hh = (4 - (int64_t)(((uintptr_t)(in + (n0 + il) * L) >> 2) & 3)) & 3;
+      if (hh > Lr) hh = Lr;
+      const int64_t nu = (Lr - hh) >> 2;
+      const int h = (int)hh, tl = (int)(Lr - hh - 4 * nu);
+      const Range<S, DIST> r(nu, 4 * nu, 4, sl);  // body units of this slave (P:166 / R5)
+      const float* body = Grad + hh;
+      const float* trow = body + 4 * nu;
+      float sum = 0.f;                                                // loops 1+2
+#pragma unroll
+      for (int j = 0; j < HM; ++j) sum += sl + j * S < h ? Grad[sl + j * S] : 0.f;
+      for (int64_t u = r.begin; u < r.end; u += r.step) {
+        const float4 v = *reinterpret_cast<const float4*>(body + 4 * u);
+        sum += v.x; sum += v.y; sum += v.z; sum += v.w;
+      }
+#pragma unroll
+      for (int j = 0; j < HM; ++j) sum += sl + j * S < tl ? trow[sl + j * S] : 0.f;
       sum = team.template reduce<OpSum>(sum);
       const float ave = sum / (float)L;
       float var = 0.f, ep = 0.f;
-      for (int64_t i = r.begin; i < e; i += r.step) {                 // loop 3
-        const float tt = Grad[i] - ave;
+      auto acc3 = [&](float gv) {
+        const float tt = gv - ave;
         var = fmaf(tt, tt, var);
         ep += tt;
+      };
+#pragma unroll
+      for (int j = 0; j < HM; ++j)                                    // loop 3
+        if (sl + j * S < h) acc3(Grad[sl + j * S]);
+      for (int64_t u = r.begin; u < r.end; u += r.step) {
+        const float4 v = *reinterpret_cast<const float4*>(body + 4 * u);
+        acc3(v.x); acc3(v.y); acc3(v.z); acc3(v.w);
       }
+#pragma unroll
+      for (int j = 0; j < HM; ++j)
+        if (sl + j * S < tl) acc3(trow[sl + j * S]);
       var = team.template reduce<OpSum>(var);
       ep = team.template reduce<OpSum>(ep);
       if (team.is_master() && ok) {
