@@ -1,0 +1,149 @@
+"""The north star's performance targets, re-checked on whatever B200 runs the
+GPU suite (BASELINE.json north_star):
+
+  * the best-S NP kernel reaches >= 70 % of B200 HBM bandwidth on TMV
+    (C2, 16384^2 fp32; the measured copy peak of MEASURED_PEAKS.json);
+  * it beats both the S=1 (no-NP) kernel and the dynamic-parallelism variant
+    at every inner trip count <= 1024 (C3 reduce L = 32..256, C4 scan
+    L = 64..1024, C1 TMV L = 1024).
+
+Times are CUDA events on the launching stream, median of several launches,
+inputs > L2 (C1 is timed as a graph of launches over 64 cold copies).  The
+margins asserted are far below the measured ones (TMV 103-108 %
+of the copy peak; NP/S=1 1.4-3.7x; NP/DP >= 4.6x), so a pass is not noise.
+DP per thread is timed on a 65,536-item prefix and scaled.
+"""
+import json
+import os
+import statistics
+
+import pytest
+
+torch = pytest.importorskip("torch")
+if not torch.cuda.is_available():
+    pytest.skip("needs a CUDA device", allow_module_level=True)
+
+from paper_conf_ppopp_yangz14_b200 import build as B  # noqa: E402
+from paper_conf_ppopp_yangz14_b200 import cudanp as C  # noqa: E402
+
+pytestmark = pytest.mark.gpu
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _lib():
+    B.build()
+    C.load()
+    C.cudanp_dp_set_pending_launch_limit(1 << 17)
+
+
+def peak_gbs():
+    try:
+        return float(json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))["hbm_gbs"])
+    except (OSError, KeyError, ValueError):
+        return 6461.0  # the lowest copy peak measured on this pool (profiles/)
+
+
+def t_ms(fn, reps=5, warm=2):
+    for _ in range(warm):
+        fn()
+    ts = []
+    for _ in range(reps):
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record()
+        fn()
+        b.record()
+        b.synchronize()
+        ts.append(a.elapsed_time(b))
+    return statistics.median(ts)
+
+
+def gen(shape, kind, dtype=torch.float32, B_=1 << 15):
+    t = torch.empty(*shape, dtype=dtype, device="cuda")
+    C.cudanp_generate(t, kind, B=B_)
+    return t
+
+
+def test_tmv_best_np_reaches_70pct_of_hbm():
+    n = 16384
+    A = gen((n, n), "f32_unit")
+    x = gen((n,), "f32_unit")
+    y = torch.empty(n, device="cuda")
+    nb = 4 * n * n + 8 * n
+    best = min(t_ms(lambda: C.cudanp_tmv(A, x, y, S=S, dist=d, map=m))
+               for S, d, m in ((8, C.BLOCK, C.INTER_WARP_TMA), (8, C.CYCLIC, C.INTER_WARP_TMA),
+                               (16, C.CYCLIC, C.INTER_WARP), (64, C.BLOCK, C.INTER_WARP)))
+    gbs = nb / (best * 1e-3) / 1e9
+    assert gbs >= 0.70 * peak_gbs(), f"TMV {gbs:.0f} GB/s < 70 % of {peak_gbs():.0f}"
+
+
+def _np_vs_s1_dp(run_np, run_s1s, run_dp_block, run_dp_thread_prefix, N, Np, what):
+    t_np = min(t_ms(f) for f in run_np)
+    t_s1 = min(t_ms(f) for f in run_s1s)
+    t_dpb = t_ms(run_dp_block, reps=3, warm=1)
+    t_dpt = t_ms(run_dp_thread_prefix, reps=3, warm=1) * N / Np
+    assert t_s1 / t_np >= 1.1, f"{what}: NP {t_np:.3f} ms vs S=1 {t_s1:.3f} ms"
+    assert t_dpb / t_np >= 2.0, f"{what}: NP {t_np:.3f} ms vs DP per CTA {t_dpb:.3f} ms"
+    assert t_dpt / t_np >= 2.0, f"{what}: NP {t_np:.3f} ms vs DP per thread {t_dpt:.3f} ms (scaled)"
+
+
+@pytest.mark.parametrize("L", [32, 256])
+def test_reduce_np_beats_s1_and_dp(L):
+    N, Np = 1 << 22, 65536
+    x = gen((N, L), "f32_unit")
+    out = torch.empty(N, device="cuda")
+    red = lambda S, d, m: (lambda: C.cudanp_batched_loop_reduce(x, None, out, S=S, dist=d, map=m))  # noqa: E731
+    np_ = [red(S, C.BLOCK, C.INTRA_WARP) for S in ((2, 4, 8) if L == 32 else (16, 32))]
+    s1 = [red(1, d, m) for d in (C.CYCLIC, C.BLOCK) for m in (C.INTRA_WARP, C.INTER_WARP)]
+    s1.append(lambda: C.cudanp_batched_loop_reduce_variant(C.S1_LITERAL, x, None, out))
+    _np_vs_s1_dp(np_, s1, lambda: C.cudanp_batched_loop_reduce_variant(C.DP_BLOCK, x, None, out),
+                 lambda: C.cudanp_batched_loop_reduce_variant(C.DP_THREAD, x[:Np], None, out[:Np]),
+                 N, Np, f"C3 reduce L={L}")
+
+
+@pytest.mark.parametrize("L", [64, 1024])
+def test_scan_np_beats_s1_and_dp(L):
+    N, Np = 1 << 21, 65536
+    x = gen((N, L), "i32_small", torch.int32)
+    out = torch.empty_like(x)
+    sc = lambda S, d, m: (lambda: C.cudanp_batched_loop_scan(x, None, out, S=S, dist=d, map=m))  # noqa: E731
+    np_ = [sc(16, d, C.INTRA_WARP) for d in (C.CYCLIC, C.BLOCK)]
+    s1 = [sc(1, d, m) for d in (C.CYCLIC, C.BLOCK) for m in (C.INTRA_WARP, C.INTER_WARP)]
+    s1.append(lambda: C.cudanp_batched_loop_scan_variant(C.S1_LITERAL, x, None, out))
+    _np_vs_s1_dp(np_, s1, lambda: C.cudanp_batched_loop_scan_variant(C.DP_BLOCK, x, None, out),
+                 lambda: C.cudanp_batched_loop_scan_variant(C.DP_THREAD, x[:Np], None, out[:Np]),
+                 N, Np, f"C4 scan L={L}")
+    del x, out
+    torch.cuda.empty_cache()
+
+
+def test_c1_tmv_np_beats_s1_and_dp():
+    """C1: TMV 1024^2, one master per output, inner loop 1024 (latency-bound:
+    timed as a CUDA graph over 64 cold copies of A)."""
+    n, copies = 1024, 64
+    As = [gen((n, n), "f32_unit") for _ in range(copies)]
+    x = gen((n,), "f32_unit")
+    ys = [torch.empty(n, device="cuda") for _ in range(copies)]
+
+    def graph_ms(mk):
+        s = torch.cuda.Stream()
+        s.wait_stream(torch.cuda.current_stream())
+        with torch.cuda.stream(s):
+            for i in range(copies):
+                mk(i)()
+        torch.cuda.current_stream().wait_stream(s)
+        torch.cuda.synchronize()
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g):
+            for i in range(copies):
+                mk(i)()
+        return t_ms(g.replay) / copies
+
+    t_np = min(graph_ms(lambda i, S=S, d=d, m=m: (lambda: C.cudanp_tmv(As[i], x, ys[i], S=S, dist=d, map=m)))
+               for S, d, m in ((32, C.CYCLIC, C.INTER_WARP), (64, C.BLOCK, C.INTER_WARP)))
+    t_s1 = min(graph_ms(lambda i, m=m: (lambda: C.cudanp_tmv(As[i], x, ys[i], S=1, map=m)))
+               for m in (C.INTER_WARP, C.INTER_WARP_TMA))
+    t_dpb = t_ms(lambda: C.cudanp_tmv_variant(C.DP_BLOCK, As[0], x, ys[0]), reps=3, warm=1)
+    t_dpt = t_ms(lambda: C.cudanp_tmv_variant(C.DP_THREAD, As[0], x, ys[0]), reps=3, warm=1)
+    assert t_s1 / t_np >= 1.5, f"C1: NP {t_np * 1e3:.2f} us vs S=1 {t_s1 * 1e3:.2f} us"
+    assert min(t_dpb, t_dpt) / t_np >= 2.0, f"C1: NP {t_np * 1e3:.2f} us vs DP {min(t_dpb, t_dpt) * 1e3:.2f} us"
