@@ -21,8 +21,7 @@
  * memory across them; supported by the reduce, scan, MV and ragged-reduce
  * calls with CUDANP_MAP_AUTO / CUDANP_MAP_INTRA_WARP, and by TMV with the
  * inter-warp map for S <= 128 (CUDANP_ERR_UNSUPPORTED otherwise).
- * S in {2048, 4096, 8192} (batched reduce and scan -- block distribution
- * only for the scan, CUDANP_ERR_UNSUPPORTED for cyclic -- and MV;
+ * S in {2048, 4096, 8192} (batched reduce and scan, and MV;
  * CUDANP_ERR_INVALID for TMV): a team larger than a CTA, one thread-block cluster of 8 CTAs
  * of S/8 threads per item; the CTAs' partials meet in the master CTA's shared
  * memory over DSMEM (the inter-warp smem exchange of P:203/P:209 one level

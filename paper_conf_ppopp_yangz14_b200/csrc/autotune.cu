@@ -36,8 +36,8 @@ static std::vector<Candidate> candidates(int op_kind) {
         for (int d = 0; d < 2; ++d) c.push_back({S, d, CUDANP_MAP_INTRA_WARP_TMA});
     for (int S : {64, 128, 256, 512, 1024})
       for (int d = 0; d < 2; ++d) c.push_back({S, d, CUDANP_MAP_INTRA_WARP});
-    for (int S : {2048, 4096, 8192})  // cluster teams (the scan: block distribution only)
-      for (int d = op_kind == 3 ? 1 : 0; d < 2; ++d) c.push_back({S, d, CUDANP_MAP_INTRA_WARP});
+    for (int S : {2048, 4096, 8192})  // cluster teams
+      for (int d = 0; d < 2; ++d) c.push_back({S, d, CUDANP_MAP_INTRA_WARP});
   }
   return c;
 }

@@ -332,6 +332,167 @@ scan_cluster_kernel(const T* __restrict__ in, const T* __restrict__ init, T* __r
   cluster.sync();
 }
 
+// ---------------------------------------------------------------- batched scan (cyclic)
+// Cyclic distribution: unit u belongs to slave u mod S, so in round k
+// (units k*S .. k*S+S-1) CTA `rank` owns the contiguous units
+// k*S + rank*CTA + [0, CTA) -- every warp load is coalesced.  A unit's prefix
+// needs every unit of the earlier rounds and of the lower ranks in its own
+// round; instead of a cluster barrier per round, rounds are processed in
+// chunks of RC rounds, two passes per chunk:
+//   pass 1: each warp scans its units of every round of the chunk
+//           (shfl-up) and keeps the warp totals wt[k][w] in shared
+//           memory; the CTA totals tot[k] are published in its own shared
+//           memory; one cluster barrier;
+//   exchange: thread k reads the 8 CTAs' tot[k] over DSMEM (and the master
+//           CTA's carry-in init[n], read_from_master one level up) and the
+//           CTA turns them into the offset of each (round, warp) -- every CTA
+//           computes the same chunk total, in the same order, for its carry;
+//   pass 2: re-read the chunk (an L2 hit: RC = 16 rounds keep <= 256 KB per SM
+//           in flight between the passes, 37 MB over the GPU; with 32 rounds
+//           and 1024-thread CTAs ncu saw a 14 % L2 hit rate), local scan +
+//           the same warp scan + offset, store.
+// The warp totals come from the same shfl-up scan in both passes, so the
+// offsets and the stored values agree bit for bit.
+constexpr int kScanRC = 16;  // rounds per chunk: <= 256 KB of pass-1 data per SM stays in L2 for pass 2
+constexpr int kScanG = 8;    // rounds whose loads are in flight together
+
+template <class T, int S, bool VEC>
+__global__ void __launch_bounds__(S / kClusterCtas, 4096 / S > 0 ? 4096 / S : 1)
+scan_cluster_cyclic_kernel(const T* __restrict__ in, const T* __restrict__ init,
+                           T* __restrict__ out, int64_t N, int64_t L) {
+  pdl_entry();
+  constexpr int CTA = S / kClusterCtas;
+  constexpr int W = CTA / 32;
+  constexpr int RC = kScanRC;
+  constexpr int G = kScanG;
+  static_assert(RC % G == 0, "whole groups per chunk");
+  static_assert(RC <= 32 && RC * W <= CTA, "one lane per round / per (round, warp)");
+  __shared__ T wt[RC][W];        // warp totals of the chunk's rounds (pass 1)
+  __shared__ T offw[RC][W];      // offset of each (round, warp)
+  __shared__ T tot[2][RC];       // this CTA's per-round totals (read over DSMEM)
+  __shared__ T cin[2];           // the master CTA's carry-in
+  __shared__ T carry_s;
+  cg::cluster_group cluster = cg::this_cluster();
+  const int rank = (int)cluster.block_rank();
+  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+  const int64_t nunits = VEC ? (L >> 2) : L;
+  const int64_t nrounds = (nunits + S - 1) / S;
+  const int64_t cid = blockIdx.x / kClusterCtas, ncl = gridDim.x / kClusterCtas;
+  cluster_arrive_relaxed();
+  bool started = false;
+  int par = 0;
+  auto unit_load = [&](const T* row, int64_t u) -> V4<T> {
+    V4<T> v = {T(0), T(0), T(0), T(0)};
+    if (u < nunits) {
+      if constexpr (VEC) v = ldg4(row + 4 * u);
+      else v.x = ldg1(row + u);
+    }
+    return v;
+  };
+  auto warp_incl = [&](T x) {
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const T t = __shfl_up_sync(kFull, x, o);
+      if (lane >= o) x = OpSum::apply(x, t);
+    }
+    return x;
+  };
+  for (int64_t item = cid; item < N; item += ncl) {
+    const T* irow = in + item * L;
+    T* orow = out + item * L;
+    if (tid == 0) {
+      if (rank == 0) cin[par] = init ? init[item] : T(0);  // the master's sequential section
+      carry_s = T(0);
+    }
+    bool first = true;
+    for (int64_t k0 = 0; k0 < nrounds; k0 += RC, par ^= 1) {
+      const int rc = (int)(nrounds - k0 < RC ? nrounds - k0 : RC);
+      // pass 1: warp totals per round (G rounds' loads in flight at a time)
+      for (int kg = 0; kg < rc; kg += G) {
+        V4<T> v[G];
+#pragma unroll
+        for (int j = 0; j < G; ++j) v[j] = unit_load(irow, (k0 + kg + j) * S + rank * CTA + tid);
+#pragma unroll
+        for (int j = 0; j < G; ++j) {
+          if (kg + j >= rc) break;
+          const T ut = VEC ? OpSum::apply(OpSum::apply(OpSum::apply(v[j].x, v[j].y), v[j].z), v[j].w) : v[j].x;
+          const T wi = warp_incl(ut);
+          if (lane == 31) wt[kg + j][wid] = wi;
+        }
+      }
+      if (!started) {  // CTA-uniform; see cluster_team_reduce
+        cluster_wait();
+        started = true;
+      }
+      __syncthreads();
+      if (tid < rc) {
+        T c = wt[tid][0];
+#pragma unroll
+        for (int w = 1; w < W; ++w) c = OpSum::apply(c, wt[tid][w]);
+        tot[par][tid] = c;
+      }
+      cluster.sync();  // every CTA's tot[par] (and the carry-in) visible cluster-wide
+      // exchange: lane k of warp 0 gathers round k's totals of all ranks
+      if (wid == 0) {
+        T rowt = T(0), low = T(0);
+        if (lane < rc) {
+#pragma unroll
+          for (int r = 0; r < kClusterCtas; ++r) {
+            const T t = *cluster.map_shared_rank(&tot[par][lane], r);
+            rowt = OpSum::apply(rowt, t);
+            if (r < rank) low = OpSum::apply(low, t);
+          }
+        }
+        const T incl = warp_incl(rowt);                   // rounds 0..k of the chunk
+        const T chunk_total = __shfl_sync(kFull, incl, 31);
+        T base = carry_s;
+        if (first) base = OpSum::apply(base, *cluster.map_shared_rank(&cin[par], 0));
+        // offset of round k for this CTA = base + rounds < k + lower ranks in round k
+        const T offk = OpSum::apply(base, OpSum::apply(tsub_c(incl, rowt), low));
+        if (lane < rc) {
+          T o = offk;
+#pragma unroll
+          for (int w = 0; w < W; ++w) {
+            offw[lane][w] = o;
+            o = OpSum::apply(o, wt[lane][w]);
+          }
+        }
+        __syncwarp();
+        if (lane == 0) carry_s = OpSum::apply(base, chunk_total);
+      }
+      first = false;
+      __syncthreads();
+      // pass 2: rescan and store
+      for (int kg = 0; kg < rc; kg += G) {
+        V4<T> vv[G];
+#pragma unroll
+        for (int j = 0; j < G; ++j) vv[j] = unit_load(irow, (k0 + kg + j) * S + rank * CTA + tid);
+#pragma unroll
+        for (int j = 0; j < G; ++j) {
+          if (kg + j >= rc) break;
+          const int64_t u = (k0 + kg + j) * S + rank * CTA + tid;
+          V4<T> v = vv[j];
+          if constexpr (VEC) {
+            v.y = OpSum::apply(v.x, v.y); v.z = OpSum::apply(v.y, v.z); v.w = OpSum::apply(v.z, v.w);
+          }
+          const T ut = VEC ? v.w : v.x;
+          const T wi = warp_incl(ut);
+          const T add = OpSum::apply(offw[kg + j][wid], tsub_c(wi, ut));
+          if (u < nunits) {
+            if constexpr (VEC)
+              stg4(orow + 4 * u, V4<T>{OpSum::apply(add, v.x), OpSum::apply(add, v.y),
+                                       OpSum::apply(add, v.z), OpSum::apply(add, v.w)});
+            else orow[u] = OpSum::apply(add, v.x);
+          }
+        }
+      }
+      __syncthreads();  // wt / offw / carry_s reused by the next chunk
+    }
+  }
+  if (!started) cluster_wait();
+  cluster.sync();  // remote reads of tot/cin are done before any CTA exits
+}
+
 #define CUDANP_DISPATCH_CLUSTER_S(S, ...)                      \
   switch (S) {                                                 \
     case 2048: { constexpr int kS = 2048; __VA_ARGS__; } break; \
@@ -419,10 +580,12 @@ int mv_cluster(const float* A, int64_t lda, const float* x, float* y, int64_t h,
 
 template <class T>
 static int scan_cluster_t(const void* in, const void* init, void* out, int64_t N, int64_t L, int S,
-                          bool vec, cudaStream_t st, LaunchInfo* info) {
+                          int dist, bool vec, cudaStream_t st, LaunchInfo* info) {
   CUDANP_DISPATCH_CLUSTER_S(S, {
     constexpr int CTA = kS / kClusterCtas;
-    auto kern = vec ? scan_cluster_kernel<T, kS, true> : scan_cluster_kernel<T, kS, false>;
+    auto kern = dist == DIST_CYCLIC
+                    ? (vec ? scan_cluster_cyclic_kernel<T, kS, true> : scan_cluster_cyclic_kernel<T, kS, false>)
+                    : (vec ? scan_cluster_kernel<T, kS, true> : scan_cluster_kernel<T, kS, false>);
     if (!info && (N == 0 || L == 0)) return CUDANP_OK;
     return launch_cluster(kern, CTA, N, st, info, "batched_loop_scan (cluster team) launch",
                           (const T*)in, (const T*)init, (T*)out, N, L);
@@ -432,13 +595,8 @@ static int scan_cluster_t(const void* in, const void* init, void* out, int64_t N
 
 int scan_cluster(const void* in, const void* init, void* out, int64_t N, int64_t L, int dtype, int S,
                  int dist, bool vec, cudaStream_t st, LaunchInfo* info) {
-  if (dist != DIST_BLOCK) {
-    set_error("a cluster-team scan is built for the block distribution only (a cyclic "
-              "cluster-wide scan needs a cluster barrier per round of S units)");
-    return CUDANP_ERR_UNSUPPORTED;
-  }
-  return dtype == CUDANP_F32 ? scan_cluster_t<float>(in, init, out, N, L, S, vec, st, info)
-                             : scan_cluster_t<int32_t>(in, init, out, N, L, S, vec, st, info);
+  return dtype == CUDANP_F32 ? scan_cluster_t<float>(in, init, out, N, L, S, dist, vec, st, info)
+                             : scan_cluster_t<int32_t>(in, init, out, N, L, S, dist, vec, st, info);
 }
 
 }  // namespace cudanp

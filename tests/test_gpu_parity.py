@@ -655,27 +655,25 @@ def test_cluster_teams_parity():
     with pytest.raises(C.CudanpError) as ei:
         C.cudanp_batched_loop_reduce(dev(synth.items(4, 64, "i32_full")), S=2048, map=C.INTER_WARP)
     assert ei.value.status == C.ERR_UNSUPPORTED
-    # TMV has no cluster team (CUDANP_ERR_INVALID before launch); the scan's is block-only
+    # TMV has no cluster team (CUDANP_ERR_INVALID before launch)
     with pytest.raises(C.CudanpError) as ei:
         C.cudanp_tmv(dev(synth.matrix(8, 8, "f32_int4")), dev(synth.vector(8, "f32_int4")), S=2048)
     assert ei.value.status == C.ERR_INVALID
-    with pytest.raises(C.CudanpError) as ei:
-        C.cudanp_batched_loop_scan(dev(synth.items(4, 64, "i32_small")), S=2048, dist=C.CYCLIC)
-    assert ei.value.status == C.ERR_UNSUPPORTED
-    # scan with a cluster per item (block distribution), int32 bit-exact with carry-in, fp32 exact data
-    for N, L in [(1, 1), (3, 0), (5, 8193), (40, 20000), (2500, 96), (9, 65540), (4, 5)]:
+    # scan with a cluster per item (cyclic: chunked two-pass with per-round totals over DSMEM;
+    # block: chunk sums), int32 bit-exact with carry-in, fp32 exact data
+    for N, L in [(1, 1), (3, 0), (5, 8193), (40, 20000), (2500, 96), (9, 65540), (4, 5), (2, 600001), (3, 1 << 20)]:
         xs = synth.items(N, L, "i32_small", B=1 << 15, seed=L)
         ini = synth.init(N, "i32_small", seed=N)
         xf = synth.items(N, L, "f32_int4", seed=L)
         ref_s, ref_f = O.scan(xs, init=ini), O.scan(xf)
         xsd, inid, xfd = dev(xs), dev(ini), dev(xf)
-        for S in CLUSTER_S:
-            what = f"scan cluster S={S} N={N} L={L}"
-            assert_exact(host(C.cudanp_batched_loop_scan(xsd, inid, S=S, dist=C.BLOCK)), ref_s, what)
-            assert_exact(host(C.cudanp_batched_loop_scan(xfd, S=S, dist=C.BLOCK)), ref_f, what + " f32")
+        for S, dist in itertools.product(CLUSTER_S, DISTS):
+            what = f"scan cluster S={S} N={N} L={L} dist={dist}"
+            assert_exact(host(C.cudanp_batched_loop_scan(xsd, inid, S=S, dist=dist)), ref_s, what)
+            assert_exact(host(C.cudanp_batched_loop_scan(xfd, S=S, dist=dist)), ref_f, what + " f32")
             if L > 1:  # misaligned rows: scalar units
                 v = xsd.view(-1)[1:1 + N * (L - 1)].view(N, L - 1)
-                assert_exact(host(C.cudanp_batched_loop_scan(v, inid, S=S, dist=C.BLOCK)),
+                assert_exact(host(C.cudanp_batched_loop_scan(v, inid, S=S, dist=dist)),
                              O.scan(xs.reshape(-1)[1:1 + N * (L - 1)].reshape(N, L - 1), init=ini),
                              what + " misaligned")
     i = C.cudanp_launch_info("reduce", 256, 65536, S=4096)

@@ -124,9 +124,8 @@ def test_big_and_cluster_teams_random(N, L, S, dist, shift, use_init, seed):
                  O.reduce(xs, init=ini if use_init else None), "reduce " + what)
     assert_exact(host(C.cudanp_batched_loop_reduce(xd, None, op=C.MAX, S=S, dist=dist)),
                  O.reduce(xs, op=O.MAX), "reduce max " + what)
-    if S <= 1024 or dist == C.BLOCK:
-        assert_exact(host(C.cudanp_batched_loop_scan(xd, inid, S=S, dist=dist)),
-                     O.scan(xs, init=ini if use_init else None), "scan " + what)
+    assert_exact(host(C.cudanp_batched_loop_scan(xd, inid, S=S, dist=dist)),
+                 O.scan(xs, init=ini if use_init else None), "scan " + what)
     if N and L:
         h, w = min(N, 64), min(L, 5000)
         A = synth.matrix(h, w, "f32_int4", seed=seed)

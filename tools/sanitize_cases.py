@@ -71,8 +71,9 @@ def main():
         for d in (C.CYCLIC, C.BLOCK):
             C.cudanp_batched_loop_reduce(Xc, None, S=S, dist=d)
             C.cudanp_batched_loop_reduce(Xcf, None, op=C.MAX, S=S, dist=d)
-        C.cudanp_batched_loop_scan(Xc, None, S=S, dist=C.BLOCK)
-        C.cudanp_batched_loop_scan(Xcf, None, S=S, dist=C.BLOCK)
+        for d in (C.CYCLIC, C.BLOCK):
+            C.cudanp_batched_loop_scan(Xc, None, S=S, dist=d)
+            C.cudanp_batched_loop_scan(Xcf, None, S=S, dist=d)
         C.cudanp_mv(A, xm, S=S, dist=C.CYCLIC)
     Xp = dev(synth.items(70, 37, "i32_small").reshape(-1))  # peeled rows, every misalignment
     for sh in range(4):
