@@ -457,9 +457,16 @@ def big():
     these working sets fit the 126 MB L2)."""
     cases = [("mv", h, 65536) for h in (16, 64, 256, 1024, 4096)] + \
             [("reduce", N, L) for N, L in ((16, 1 << 22), (64, 1 << 20), (256, 262144), (2048, 16384), (16384, 4096))] + \
-            [("scan", N, L) for N, L in ((16, 1 << 22), (256, 262144))]
+            [("scan", N, L) for N, L in ((16, 1 << 22), (256, 262144))] + \
+            [("tmv", w, h) for w, h in ((256, 262144), (1024, 65536), (4096, 16384))]
     for op, N, L in cases:
-        if op == "mv":
+        if op == "tmv":  # N = columns (masters), L = rows (the loop)
+            A = gen((L, N), "f32_unit")
+            x = gen((L,), "f32_unit", stream_id=2)
+            y = torch.empty(N, device="cuda")
+            nb = 4 * N * L + 4 * N + 4 * L
+            fn = lambda S, d: C.cudanp_tmv(A, x, y, S=S, dist=d, map=C.INTER_WARP if S > 32 else C.AUTO)  # noqa: E731
+        elif op == "mv":
             A = gen((N, L), "f32_unit")
             x = gen((L,), "f32_unit", stream_id=2)
             y = torch.empty(N, device="cuda")
@@ -475,7 +482,9 @@ def big():
             y = torch.empty_like(A)
             nb = 8 * N * L
             fn = lambda S, d: C.cudanp_batched_loop_scan(A, None, y, S=S, dist=d, map=C.INTRA_WARP)  # noqa: E731
-        for S in C.SLAVE_SIZES + (64, 128, 256, 512, 1024, 2048, 4096, 8192):
+        sizes = (C.SLAVE_SIZES + (64, 128, 1024)) if op == "tmv" else \
+            (C.SLAVE_SIZES + (64, 128, 256, 512, 1024, 2048, 4096, 8192))
+        for S in sizes:
             for d in (C.CYCLIC, C.BLOCK):
                 try:
                     med, mn = time_ms(lambda: fn(S, d), flush=True)
