@@ -20,8 +20,8 @@
  * 32"): a team of S/32 consecutive warps, shfl inside each warp and shared
  * memory across them; supported by the reduce, scan, MV and ragged-reduce
  * calls with CUDANP_MAP_AUTO / CUDANP_MAP_INTRA_WARP, and by TMV with the
- * inter-warp map for S <= 128 and S = 1024 -- a cluster of 8 CTAs of
- * 8 column-masters x 128 slave warps, partials combined over DSMEM
+ * inter-warp map for S <= 128 and S = 256 / 1024 -- a cluster of 8 CTAs of
+ * 8 column-masters x 32 / 128 slave warps, partials combined over DSMEM
  * (CUDANP_ERR_UNSUPPORTED otherwise).
  * S in {2048, 4096, 8192} (batched reduce and scan, and MV;
  * CUDANP_ERR_INVALID for TMV): a team larger than a CTA, one thread-block cluster of 8 CTAs

@@ -28,7 +28,7 @@ static std::vector<Candidate> candidates(int op_kind) {
   if (op_kind == 0) {  // TMV: TMA-staged inter-warp, and inter-warp teams up to 128
     for (int S : small)
       for (int d = 0; d < 2; ++d) c.push_back({S, d, CUDANP_MAP_INTER_WARP_TMA});
-    for (int S : {64, 128, 1024})  // 1024: a cluster of 8 CTAs per column group
+    for (int S : {64, 128, 256, 1024})  // 256 / 1024: a cluster of 8 CTAs per column group
       for (int d = 0; d < 2; ++d) c.push_back({S, d, CUDANP_MAP_INTER_WARP});
   } else {             // MV / reduce / scan: multi-warp teams (+ the TMA-staged reduce, cluster teams)
     if (op_kind == 2)

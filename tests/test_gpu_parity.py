@@ -626,14 +626,14 @@ def test_big_teams_parity():
             if S <= 128:
                 assert_exact(host(C.cudanp_tmv(dev(A), dev(xt), S=S, dist=dist)), O.tmv(A, xt),
                              f"tmv big S={S} h={h} w={w}")
-    # TMV with a cluster team per column group (S = 1024: 8 CTAs x 128 slave warps)
+    # TMV with a cluster team per column group (S = 256 / 1024: 8 CTAs x 32 / 128 slave warps)
     for h, w in [(5, 4096), (64, 1000), (300, 260), (20000, 36), (70000, 3), (1, 1), (0, 7)]:
         A = synth.matrix(h, w, "f32_int4", seed=w)
         xt = synth.vector(h, "f32_int4")
         ref = O.tmv(A, xt) if h else np.zeros(w, np.float32)
-        for dist in DISTS:
-            assert_exact(host(C.cudanp_tmv(dev(A), dev(xt), S=1024, dist=dist)), ref,
-                         f"tmv cluster h={h} w={w} dist={dist}")
+        for S, dist in itertools.product((256, 1024), DISTS):
+            assert_exact(host(C.cudanp_tmv(dev(A), dev(xt), S=S, dist=dist)), ref,
+                         f"tmv cluster S={S} h={h} w={w} dist={dist}")
 
 
 CLUSTER_S = (2048, 4096, 8192)

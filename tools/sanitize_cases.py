@@ -75,9 +75,10 @@ def main():
             C.cudanp_batched_loop_scan(Xc, None, S=S, dist=d)
             C.cudanp_batched_loop_scan(Xcf, None, S=S, dist=d)
         C.cudanp_mv(A, xm, S=S, dist=C.CYCLIC)
-    for d in (C.CYCLIC, C.BLOCK):  # TMV cluster team (S = 1024)
-        C.cudanp_tmv(A, xt, S=1024, dist=d, map=C.INTER_WARP, n_outer=70)
-        C.cudanp_tmv(A4, xt, S=1024, dist=d, map=C.INTER_WARP)
+    for S in (256, 1024):  # TMV cluster teams
+        for d in (C.CYCLIC, C.BLOCK):
+            C.cudanp_tmv(A, xt, S=S, dist=d, map=C.INTER_WARP, n_outer=70)
+            C.cudanp_tmv(A4, xt, S=S, dist=d, map=C.INTER_WARP)
     Xp = dev(synth.items(70, 37, "i32_small").reshape(-1))  # peeled rows, every misalignment
     for sh in range(4):
         v = Xp[sh:sh + 69 * 37].view(69, 37)

@@ -482,7 +482,7 @@ def big():
             y = torch.empty_like(A)
             nb = 8 * N * L
             fn = lambda S, d: C.cudanp_batched_loop_scan(A, None, y, S=S, dist=d, map=C.INTRA_WARP)  # noqa: E731
-        sizes = (C.SLAVE_SIZES + (64, 128, 1024)) if op == "tmv" else \
+        sizes = (C.SLAVE_SIZES + (64, 128, 256, 1024)) if op == "tmv" else \
             (C.SLAVE_SIZES + (64, 128, 256, 512, 1024, 2048, 4096, 8192))
         for S in sizes:
             for d in (C.CYCLIC, C.BLOCK):
