@@ -78,7 +78,7 @@ def main():
           "us": round(graph_us([lambda i=i: C.cudanp_tmv(As[i][:0], x[:0], ys[i], S=32, dist=C.CYCLIC,
                                                          map=C.INTER_WARP, n_outer=n)
                                 for i in range(copies)]), 3)})
-    for S in (8, 16, 32, 64, 128):
+    for S in (8, 16, 32, 64, 128, 256, 1024):  # 256 / 1024: cluster teams
         for d in (C.CYCLIC, C.BLOCK):
             us = graph_us([lambda i=i: C.cudanp_tmv(As[i], x, ys[i], S=S, dist=d, map=C.INTER_WARP)
                            for i in range(copies)])
