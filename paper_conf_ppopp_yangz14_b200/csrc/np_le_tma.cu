@@ -16,6 +16,7 @@
 // and the master stores.  Each slave visits its elements in the
 // same order as the register version, so results are bit-identical to it.
 #include "common.cuh"
+#include "np_le_acc.cuh"
 #include "np_team.cuh"
 #include "np_tma.cuh"
 
@@ -94,33 +95,27 @@ le_tma_kernel(const float* __restrict__ in, float* gicov, float* ave_out, float*
       const Range<S, DIST> r(nu, 4 * nu, 4, sl);  // body units of this slave (P:166 / R5)
       const float* body = Grad + hh;
       const float* trow = body + 4 * nu;
-      float sum = 0.f;                                                // loops 1+2
-#pragma unroll
-      for (int j = 0; j < HM; ++j) sum += sl + j * S < h ? Grad[sl + j * S] : 0.f;
-      for (int64_t u = r.begin; u < r.end; u += r.step) {
+      auto unit = [&](int64_t u) {
         const float4 v = *reinterpret_cast<const float4*>(body + 4 * u);
-        sum += v.x; sum += v.y; sum += v.z; sum += v.w;
-      }
-#pragma unroll
-      for (int j = 0; j < HM; ++j) sum += sl + j * S < tl ? trow[sl + j * S] : 0.f;
-      sum = team.template reduce<OpSum>(sum);
-      const float ave = sum / (float)L;                               // P:309
-      float var = 0.f, ep = 0.f;
-      auto acc3 = [&](float gv) {
-        const float tt = gv - ave;
-        var = fmaf(tt, tt, var);
-        ep += tt;
+        return V4<float>{v.x, v.y, v.z, v.w};
       };
+      LeSum acc;                                                      // loops 1+2
 #pragma unroll
-      for (int j = 0; j < HM; ++j)                                    // loop 3
-        if (sl + j * S < h) acc3(Grad[sl + j * S]);
-      for (int64_t u = r.begin; u < r.end; u += r.step) {
-        const float4 v = *reinterpret_cast<const float4*>(body + 4 * u);
-        acc3(v.x); acc3(v.y); acc3(v.z); acc3(v.w);
-      }
+      for (int j = 0; j < HM; ++j) acc.head(sl + j * S < h ? Grad[sl + j * S] : 0.f);
+      for (int64_t u = r.begin; u < r.end; u += r.step) acc.body(unit(u));
+#pragma unroll
+      for (int j = 0; j < HM; ++j) acc.tail(sl + j * S < tl ? trow[sl + j * S] : 0.f);
+      const float sum = team.template reduce<OpSum>(acc.result());
+      const float ave = sum / (float)L;                               // P:309
+      LeVarEp a(ave);                                                 // loop 3
 #pragma unroll
       for (int j = 0; j < HM; ++j)
-        if (sl + j * S < tl) acc3(trow[sl + j * S]);
+        if (sl + j * S < h) a.head(Grad[sl + j * S]);
+      for (int64_t u = r.begin; u < r.end; u += r.step) a.body(unit(u));
+#pragma unroll
+      for (int j = 0; j < HM; ++j)
+        if (sl + j * S < tl) a.tail(trow[sl + j * S]);
+      float var = a.var(), ep = a.ep();
       var = team.template reduce<OpSum>(var);
       ep = team.template reduce<OpSum>(ep);
       if (team.is_master() && ok) {
