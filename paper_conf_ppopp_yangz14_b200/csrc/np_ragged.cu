@@ -20,7 +20,7 @@
 namespace cudanp {
 
 #ifndef CUDANP_RAGGED_K
-#define CUDANP_RAGGED_K 4
+#define CUDANP_RAGGED_K 2
 #endif
 #ifndef CUDANP_RAGGED_UNROLL
 #define CUDANP_RAGGED_UNROLL 4

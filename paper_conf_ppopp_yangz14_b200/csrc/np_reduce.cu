@@ -21,7 +21,7 @@ namespace cudanp {
 
 constexpr int kReduceBlock = 256;  // intra-warp CTA: 8 warps
 #ifndef CUDANP_REDUCE_K
-#define CUDANP_REDUCE_K 4
+#define CUDANP_REDUCE_K 2
 #endif
 constexpr int kReduceK = CUDANP_REDUCE_K;  // warp tiles in flight per warp (intra)
 
