@@ -14,6 +14,11 @@
 
 namespace cudanp {
 
+#ifndef CUDANP_MULTI_U
+#define CUDANP_MULTI_U 4
+#endif
+constexpr int kMultiU = CUDANP_MULTI_U;  // units per thread batched before the fold (reduce, MV)
+
 // a - b with int32 wrapping modulo 2^32 (R13)
 __device__ __forceinline__ float tsub(float a, float b) { return a - b; }
 __device__ __forceinline__ int32_t tsub(int32_t a, int32_t b) { return (int32_t)((uint32_t)a - (uint32_t)b); }
@@ -43,7 +48,7 @@ reduce_multi_kernel(const T* __restrict__ in, const T* __restrict__ init, T* __r
     V4<T> acc = {id, id, id, id};
     if (ok) {
       int64_t u = r.begin;
-      constexpr int U = 4;
+      constexpr int U = kMultiU;
       for (; u + (U - 1) * r.step < r.end; u += U * r.step) {
         V4<T> v[U];
 #pragma unroll
@@ -84,7 +89,7 @@ mv_multi_kernel(const float* __restrict__ A, int64_t lda, const float* __restric
     V4<float> acc = {0.f, 0.f, 0.f, 0.f};
     if (ok) {
       int64_t u = r.begin;
-      constexpr int U = 4;
+      constexpr int U = kMultiU;
       for (; u + (U - 1) * r.step < r.end; u += U * r.step) {
         V4<float> av[U], xv[U];
 #pragma unroll
