@@ -174,6 +174,18 @@ int cudanp_batched_loop_scan(const void* in, const void* init, void* out,
 int cudanp_ragged_loop_reduce(const void* in, const int64_t* offsets, const void* init, void* out,
                               int64_t n_outer, int dtype, int op, int S, int dist, int map,
                               void* stream);
+/* Ragged reduce with the team size chosen per segment at run time: each lane
+ * of a warp is the master of one segment; segments shorter than `threshold`
+ * elements are reduced by their master alone (S = 1, 128-bit body units),
+ * longer ones by the whole warp as a team of 32 (cyclic units, shfl
+ * reduction), the masters taking turns -- the master decides in its
+ * sequential section whether to wake its slaves for a loop whose bound it has
+ * just read (the imbalance of P:340 under length mixes).  Same
+ * result contract as cudanp_ragged_loop_reduce; threshold >= 1, else
+ * CUDANP_ERR_INVALID. */
+int cudanp_ragged_loop_reduce_adaptive(const void* in, const int64_t* offsets, const void* init,
+                                       void* out, int64_t n_outer, int dtype, int op,
+                                       int64_t threshold, void* stream);
 /* Comparison: one thread per segment, serial loop (Fig 2 style). */
 int cudanp_ragged_loop_reduce_literal(const void* in, const int64_t* offsets, const void* init,
                                       void* out, int64_t n_outer, int dtype, int op, void* stream);

@@ -277,6 +277,138 @@ static int launch_ragged_multi(const T* in, const int64_t* off, const T* init, T
 #undef CUDANP_RAGGED_BIG
 }
 
+// ---------------------------------------------------------------- adaptive team size
+// Segment lengths vary (exponential mixes, P:340's imbalance): a fixed S
+// either wastes slaves on short segments or leaves long ones to one thread.
+// Here the team size is chosen per segment at run time, the way the master
+// decides in its sequential section whether to wake its slaves for a loop
+// whose bound it has just read: each lane is the master of one
+// segment of the warp's 32; segments shorter than `thresh` are run by their
+// master alone (S = 1, 128-bit body units), and each longer one is run by
+// the whole warp as a team of 32 (cyclic units), the masters taking
+// turns (ballot of the long ones, bounds broadcast by shfl from their
+// master), with a butterfly team reduction; the master stores
+// (P:327).  Every segment is still reduced by exactly one team.
+template <class T, class Op>
+__global__ void __launch_bounds__(kRaggedBlock)
+ragged_adaptive_kernel(const T* __restrict__ in, const int64_t* __restrict__ off,
+                       const T* __restrict__ init, T* __restrict__ out, int64_t N, int64_t thresh) {
+  pdl_entry();
+  constexpr int K = 2;  // tiles of 32 segments per warp step: their bound loads overlap
+  const int lane = threadIdx.x & 31;
+  const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  const int64_t ntiles = (N + 31) / 32;
+  const T id = Op::template identity<T>();
+  for (int64_t t0 = warp * K; t0 < ntiles; t0 += nwarps * K) {
+    int64_t item[K], b[K], len[K];
+#pragma unroll
+    for (int k = 0; k < K; ++k) {  // sequential sections: each master reads its loop bounds
+      item[k] = (t0 + k) * 32 + lane;
+      b[k] = 0; len[k] = 0;
+      if (item[k] < N) {
+        b[k] = off[item[k]];
+        len[k] = off[item[k] + 1] - b[k];
+        if (len[k] < 0) len[k] = 0;
+      }
+    }
+    T part[K];
+    // short segments: each master alone (a team of one); all K items' loads in flight
+    {
+      const T* p[K];
+      int cnt[K];
+      int64_t stp[K];
+      int trips = 0;
+#pragma unroll
+      for (int k = 0; k < K; ++k) {
+        const int64_t ls = len[k] >= thresh ? 0 : len[k];
+        const SegShare<T, 1, DIST_CYCLIC> sh(in, b[k], ls, 0);
+        p[k] = sh.body; cnt[k] = sh.cnt; stp[k] = sh.step;
+        trips = max(trips, sh.cnt);
+        T hv[3], tv[3];
+        const T* tl = in + b[k] + sh.head + 4 * ((ls - sh.head) >> 2);
+#pragma unroll
+        for (int j = 0; j < 3; ++j) {
+          hv[j] = j < sh.head ? ldg1(in + b[k] + j) : id;
+          tv[j] = j < sh.tail ? ldg1(tl + j) : id;
+        }
+        part[k] = Op::apply(Op::apply(Op::apply(hv[0], hv[1]), hv[2]), Op::apply(Op::apply(tv[0], tv[1]), tv[2]));
+      }
+      V4<T> acc[K];
+#pragma unroll
+      for (int k = 0; k < K; ++k) acc[k] = {id, id, id, id};
+#pragma unroll 2
+      for (int j = 0; j < trips; ++j) {
+        V4<T> v[K];
+#pragma unroll
+        for (int k = 0; k < K; ++k) {
+          v[k] = j < cnt[k] ? ldg4(p[k]) : V4<T>{id, id, id, id};
+          p[k] += stp[k];
+        }
+#pragma unroll
+        for (int k = 0; k < K; ++k) acc[k] = op4r<T, Op>(acc[k], v[k]);
+      }
+#pragma unroll
+      for (int k = 0; k < K; ++k)
+        part[k] = Op::apply(part[k], Op::apply(Op::apply(acc[k].x, acc[k].y), Op::apply(acc[k].z, acc[k].w)));
+    }
+    // long segments: the whole warp as one team, masters taking turns
+#pragma unroll
+    for (int k = 0; k < K; ++k) {
+      unsigned m = __ballot_sync(kFull, len[k] >= thresh);
+      while (m) {
+        const int src = __ffs(m) - 1;
+        m &= m - 1;
+        const int64_t bb = __shfl_sync(kFull, b[k], src);   // read_from_master
+        const int64_t ll = __shfl_sync(kFull, len[k], src);
+        const SegShare<T, 32, DIST_CYCLIC> sh(in, bb, ll, lane);
+        T pv = id;
+        if (lane < sh.head) pv = Op::apply(pv, ldg1(in + bb + lane));
+        const T* tl = in + bb + sh.head + 4 * ((ll - sh.head) >> 2);
+        if (lane < sh.tail) pv = Op::apply(pv, ldg1(tl + lane));
+        V4<T> acc[4] = {{id, id, id, id}, {id, id, id, id}, {id, id, id, id}, {id, id, id, id}};
+        const T* p = sh.body;
+        int c = 0;
+        for (; c + 3 < sh.cnt; c += 4, p += 4 * sh.step) {
+          V4<T> v[4];
+#pragma unroll
+          for (int j = 0; j < 4; ++j) v[j] = ldg4(p + j * sh.step);
+#pragma unroll
+          for (int j = 0; j < 4; ++j) acc[j] = op4r<T, Op>(acc[j], v[j]);
+        }
+        for (; c < sh.cnt; ++c, p += sh.step) acc[0] = op4r<T, Op>(acc[0], ldg4(p));
+        const V4<T> a4 = op4r<T, Op>(op4r<T, Op>(acc[0], acc[1]), op4r<T, Op>(acc[2], acc[3]));
+        pv = Op::apply(pv, Op::apply(Op::apply(a4.x, a4.y), Op::apply(a4.z, a4.w)));
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) pv = Op::apply(pv, __shfl_xor_sync(kFull, pv, o));
+        if (lane == src) part[k] = pv;
+      }
+      if (item[k] < N) out[item[k]] = init ? Op::apply(init[item[k]], part[k]) : part[k];
+    }
+  }
+}
+
+template <class T, class Op>
+static int launch_ragged_adaptive(const T* in, const int64_t* off, const T* init, T* out, int64_t N,
+                                  int64_t thresh, cudaStream_t st) {
+  if (N == 0) return CUDANP_OK;
+  auto kern = ragged_adaptive_kernel<T, Op>;
+  const int64_t grid = persistent_grid(kern, kRaggedBlock, 0, (N + 2 * kRaggedBlock - 1) / (2 * kRaggedBlock));
+  launch_pdl(kern, dim3((unsigned)grid), dim3(kRaggedBlock), 0, st, in, off, init, out, N, thresh);
+  return check_launch("ragged_loop_reduce (adaptive teams) launch");
+}
+
+int ragged_adaptive(const void* in, const int64_t* off, const void* init, void* out, int64_t N,
+                    int dtype, int op, int64_t thresh, cudaStream_t st) {
+  if (dtype == CUDANP_F32)
+    return op == CUDANP_SUM
+               ? launch_ragged_adaptive<float, OpSum>((const float*)in, off, (const float*)init, (float*)out, N, thresh, st)
+               : launch_ragged_adaptive<float, OpMax>((const float*)in, off, (const float*)init, (float*)out, N, thresh, st);
+  return op == CUDANP_SUM
+             ? launch_ragged_adaptive<int32_t, OpSum>((const int32_t*)in, off, (const int32_t*)init, (int32_t*)out, N, thresh, st)
+             : launch_ragged_adaptive<int32_t, OpMax>((const int32_t*)in, off, (const int32_t*)init, (int32_t*)out, N, thresh, st);
+}
+
 // ---------------------------------------------------------------- S=1 literal
 template <class T, class Op>
 __global__ void __launch_bounds__(256)

@@ -47,6 +47,7 @@ _SIGS = {
     "cudanp_batched_loop_reduce_backend": [_vp, _vp, _vp, _i64, _i64, _int, _int, _int, _int, _vp],
     "cudanp_ragged_loop_reduce": [_vp, _vp, _vp, _vp, _i64, _int, _int, _int, _int, _int, _vp],
     "cudanp_ragged_loop_reduce_literal": [_vp, _vp, _vp, _vp, _i64, _int, _int, _vp],
+    "cudanp_ragged_loop_reduce_adaptive": [_vp, _vp, _vp, _vp, _i64, _int, _int, _i64, _vp],
     "cudanp_le_gicov": [_vp, _vp, _vp, _vp, _vp, _i64, _i64, ctypes.c_float, _int, _int, _int,
                         _int, _vp],
     "cudanp_le_gicov_placement": [_vp, _vp, _vp, _vp, _vp, _i64, _i64, ctypes.c_float, _int, _int,
@@ -267,6 +268,20 @@ def cudanp_ragged_loop_reduce(x, offsets, init=None, out=None, *, op=SUM, S=8, d
     _check(load().cudanp_ragged_loop_reduce(_ptr(x), _ptr(offsets), _ptr(init), _ptr(out), N,
                                             _dtype_code(x), op, S, dist, map, _stream(stream)),
            "cudanp_ragged_loop_reduce")
+    return out
+
+
+def cudanp_ragged_loop_reduce_adaptive(x, offsets, init=None, out=None, *, op=SUM, threshold=128,
+                                       stream=None):
+    """Ragged reduce with the team size chosen per segment (S = 1 below
+    `threshold` elements, a warp-wide team of 32 above)."""
+    import torch
+    N = offsets.shape[0] - 1
+    if out is None:
+        out = torch.empty(N, dtype=x.dtype, device=x.device)
+    _check(load().cudanp_ragged_loop_reduce_adaptive(_ptr(x), _ptr(offsets), _ptr(init), _ptr(out), N,
+                                                     _dtype_code(x), op, threshold, _stream(stream)),
+           "cudanp_ragged_loop_reduce_adaptive")
     return out
 
 

@@ -99,3 +99,29 @@ def test_ragged_big_teams():
                     assert_exact(host(C.cudanp_ragged_loop_reduce(dev(x), dev(off), S=S, dist=d)), ref, what)
                     assert_exact(host(C.cudanp_ragged_loop_reduce(dev(x), dev(off), op=C.MAX, S=S, dist=d)),
                                  refm, what)
+
+
+@pytest.mark.parametrize("kind,op,exact", [("i32_full", C.SUM, True), ("i32_full", C.MAX, True),
+                                           ("f32_signed", C.MAX, True), ("f32_unit", C.SUM, False)])
+def test_ragged_adaptive_parity(kind, op, exact):
+    """Team size chosen per segment: below the threshold the master alone, above
+    it the whole warp; mixes of both in one warp, every alignment."""
+    for N, mean, dist in CASES + [(3000, 90, "exp"), (40, 5000, "exp")]:
+        lens = synth.lengths(N, mean, dist, seed=N + mean)
+        off = synth.offsets_from_lengths(lens)
+        for shift in (0, 1, 3):
+            x = synth.gen(1, kind, 0, int(off[-1]) + 3)
+            offs = off + shift
+            ini = synth.init(N, kind)
+            ref_i = O.ragged_reduce(x, offs, op=op, init=ini)
+            xd, od, inid = dev(x), dev(offs), dev(ini)
+            for th in (1, 7, 64, 128, 1 << 40):
+                got = host(C.cudanp_ragged_loop_reduce_adaptive(xd, od, inid, op=op, threshold=th))
+                what = f"adaptive {kind} op={op} N={N} mean={mean} shift={shift} th={th}"
+                if exact:
+                    assert_exact(got, ref_i, what)
+                else:
+                    assert_rel(got, ref_i, int(lens.max()) if N else 1, what)
+    with pytest.raises(C.CudanpError):
+        C.cudanp_ragged_loop_reduce_adaptive(dev(synth.gen(1, "i32_full", 0, 8)),
+                                             dev(synth.offsets_from_lengths(np.array([3, 5]))), threshold=0)

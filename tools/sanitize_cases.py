@@ -56,6 +56,8 @@ def main():
                 C.cudanp_le_gicov(le, 0.01, S=S, dist=d, map=m)
         for be in (C.SHFL, C.SMEM, C.REDUX):
             C.cudanp_batched_loop_reduce_backend(Xi4, inii, S=S, backend=be)
+    for th in (1, 4, 16):  # ragged reduce with the team size chosen per segment
+        C.cudanp_ragged_loop_reduce_adaptive(xr, off, threshold=th)
     for S in (64, 256, 1024):  # multi-warp teams
         for d in (C.CYCLIC, C.BLOCK):
             for X, ini in ((Xf, inif), (Xi, inii)):

@@ -344,9 +344,13 @@ def r1(means=(16, 64, 256, 1024)):
                               "L": f"{dist}{mean}", "S": S, "dist": DN[d], "map": "intra", "impl": "np",
                               "t_median_us": round(med * 1e3, 2), "alg_bytes": nb,
                               "gbs": round(nb / (med * 1e-3) / 1e9, 1)})
+            comps = [("s1_literal", lit)]
+            for th in (64, 128, 256, 512):  # adaptive team size per segment
+                comps.append((f"adaptive_t{th}", time_ms(
+                    lambda: C.cudanp_ragged_loop_reduce_adaptive(x, off, None, out, threshold=th))[0]))
             sweep_np("R1", "ragged_reduce", nb,
                      lambda S, d, m: time_ms(lambda: C.cudanp_ragged_loop_reduce(x, off, None, out, S=S, dist=d, map=m)),
-                     {"dtype": "f32", "N": N, "L": f"{dist}{mean}"}, literal=lit, comps=[("s1_literal", lit)])
+                     {"dtype": "f32", "N": N, "L": f"{dist}{mean}"}, literal=lit, comps=comps)
             del x, out, off
             torch.cuda.empty_cache()
 
