@@ -28,7 +28,11 @@ F32, I32 = 0, 1
 SUM, MAX = 0, 1
 S1_LITERAL, DP_THREAD, DP_BLOCK = 1, 2, 3
 GRAD_REGISTERS, GRAD_SHARED, GRAD_GLOBAL = 0, 1, 2   # LE: home of Grad (Fig 6c / 6b / 6a)
-SLAVE_SIZES = (1, 2, 4, 8, 16, 32)
+SLAVE_SIZES = (1, 2, 4, 8, 16, 32)                    # one warp (intra) or S warps (inter)
+MULTI_WARP_SIZES = (64, 128, 256, 512, 1024)          # S/32 warps of one CTA (reduce, scan, MV;
+                                                      # TMV: 64, 128 inter-warp)
+CLUSTER_SIZES = (2048, 4096, 8192)                    # a cluster of 8 CTAs (reduce, scan, MV);
+TMV_CLUSTER_SIZES = (256, 1024)                       # TMV: 8 CTAs x 8 masters x 32/128 warps
 KIND = {"f32_unit": 0, "f32_signed": 1, "f32_int4": 2, "i32_small": 3, "i32_full": 4,
         "ones_f32": 5, "ones_i32": 6}
 SEED = 20140215
