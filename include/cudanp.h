@@ -20,14 +20,16 @@
  * 32"): a team of S/32 consecutive warps, shfl inside each warp and shared
  * memory across them; supported by the reduce, scan, MV and ragged-reduce
  * calls with CUDANP_MAP_AUTO / CUDANP_MAP_INTRA_WARP, and by TMV with the
- * inter-warp map for S <= 128 and S = 256 / 1024 -- a cluster of 8 CTAs of
- * 8 column-masters x 32 / 128 slave warps, partials combined over DSMEM
- * (CUDANP_ERR_UNSUPPORTED otherwise).
- * S in {2048, 4096, 8192} (batched reduce and scan, and MV;
- * CUDANP_ERR_INVALID for TMV): a team larger than a CTA, one thread-block cluster of 8 CTAs
- * of S/8 threads per item; the CTAs' partials meet in the master CTA's shared
- * memory over DSMEM (the inter-warp smem exchange of P:203/P:209 one level
- * up, np_cluster.cu).  For few outer items with very long loops.
+ * inter-warp map for S = 64 / 128 (8 column-masters x S slave warps per CTA).
+ * Teams larger than a CTA -- one thread-block cluster of 8 CTAs per item, the
+ * CTAs' partials (and scan totals) meeting in shared memory over DSMEM, the
+ * inter-warp smem exchange of P:203/P:209 one level up (np_cluster.cu), for
+ * few outer items with very long loops:
+ *   S in {2048, 4096, 8192}: batched reduce, batched scan and MV (S/8
+ *     threads per CTA); CUDANP_ERR_INVALID for TMV;
+ *   S in {256, 1024} with the inter-warp map: TMV (8 column-masters x 32 /
+ *     128 slave warps per CTA).
+ * Other (S, map) combinations return CUDANP_ERR_UNSUPPORTED.
  *
  * Conventions for every call:
  *  - Data pointers are DEVICE pointers owned by the caller; the library never
