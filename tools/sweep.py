@@ -120,7 +120,8 @@ def graph_time_ms(fns, reps=5):
     return statistics.median(ts), min(ts)
 
 
-def sweep_np(cfg, op, nbytes, run, extra, s1_ref=None, literal=None, comps=(), maps=None, call=None):
+def sweep_np(cfg, op, nbytes, run, extra, s1_ref=None, literal=None, comps=(), maps=None, call=None,
+             big=()):
     """run(S, dist, map) -> (median_ms, min_ms).  s1_ref: extra no-NP kernel
     times (e.g. the TMA-staged S=1 TMV) that count toward "tuned S=1".
     call(S, dist, map) -> a one-launch callable: the best NP and the best S=1
@@ -129,7 +130,9 @@ def sweep_np(cfg, op, nbytes, run, extra, s1_ref=None, literal=None, comps=(), m
     if maps is None:  # TMV and reduce also have TMA-staged kernels
         maps = (C.INTRA_WARP, C.INTER_WARP) + {"tmv": (C.INTER_WARP_TMA,),
                                                "reduce": (C.INTRA_WARP_TMA,)}.get(op, ())
-    for S, d, m in itertools.product(C.SLAVE_SIZES, (C.CYCLIC, C.BLOCK), maps):
+    cands = list(itertools.product(C.SLAVE_SIZES, (C.CYCLIC, C.BLOCK), maps)) + \
+        [(S, d, m) for S, m in big for d in (C.CYCLIC, C.BLOCK)]
+    for S, d, m in cands:
         try:
             res[(S, d, m)] = run(S, d, m)
         except C.CudanpError:
@@ -219,8 +222,13 @@ def c2():
         # part of the product path): torch.mv on the same operands = cuBLAS sgemv
         At = A.t() if op == "tmv" else A
         comps.append(("cublas_sgemv", time_ms(lambda: torch.mv(At, x, out=y))[0]))
+        # teams larger than a warp (MV: S/32 warps of a CTA; TMV: 8-master inter-warp CTAs
+        # and clusters)
+        big = ([(S, C.INTRA_WARP) for S in C.MULTI_WARP_SIZES] if op == "mv" else
+               [(S, C.INTER_WARP) for S in (64, 128) + C.TMV_CLUSTER_SIZES])
         sweep_np("C2", op, nb, lambda S, d, m: time_ms(lambda: fnp(A, x, y, S=S, dist=d, map=m)),
-                 {"dtype": "f32", "N": n, "L": n}, s1_ref=s1_ref, literal=lit, comps=comps)
+                 {"dtype": "f32", "N": n, "L": n}, s1_ref=s1_ref, literal=lit, comps=comps, big=big,
+                 call=lambda S, d, m: (lambda: fnp(A, x, y, S=S, dist=d, map=m)))
     tma_sweep("C2", A, x, y, n)
     del A
 
