@@ -358,7 +358,8 @@ def r1(means=(16, 64, 256, 1024)):
                     lambda: C.cudanp_ragged_loop_reduce_adaptive(x, off, None, out, threshold=th))[0]))
             sweep_np("R1", "ragged_reduce", nb,
                      lambda S, d, m: time_ms(lambda: C.cudanp_ragged_loop_reduce(x, off, None, out, S=S, dist=d, map=m)),
-                     {"dtype": "f32", "N": N, "L": f"{dist}{mean}"}, literal=lit, comps=comps)
+                     {"dtype": "f32", "N": N, "L": f"{dist}{mean}"}, literal=lit, comps=comps,
+                     call=lambda S, d, m: (lambda: C.cudanp_ragged_loop_reduce(x, off, None, out, S=S, dist=d, map=m)))
             del x, out, off
             torch.cuda.empty_cache()
 
