@@ -472,6 +472,9 @@ def big():
             [("reduce", N, L) for N, L in ((16, 1 << 22), (64, 1 << 20), (256, 262144), (2048, 16384), (16384, 4096))] + \
             [("scan", N, L) for N, L in ((16, 1 << 22), (256, 262144))] + \
             [("tmv", w, h) for w, h in ((256, 262144), (1024, 65536), (4096, 16384))]
+    only = os.environ.get("CUDANP_BIG_OPS")  # e.g. "scan": restrict an A/B run to one op
+    if only:
+        cases = [c for c in cases if c[0] in only.split(",")]
     for op, N, L in cases:
         if op == "tmv":  # N = columns (masters), L = rows (the loop)
             A = gen((L, N), "f32_unit")
