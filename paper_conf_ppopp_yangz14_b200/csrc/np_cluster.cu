@@ -355,6 +355,16 @@ scan_cluster_kernel(const T* __restrict__ in, const T* __restrict__ init, T* __r
 // offsets and the stored values agree bit for bit.
 constexpr int kScanRC = 16;  // rounds per chunk: <= 256 KB of pass-1 data per SM stays in L2 for pass 2
 constexpr int kScanG = 8;    // rounds whose loads are in flight together
+// CUDANP_SCL_PF=1: pass 2's first group of loads (L2 hits) is issued before the
+// cluster barrier, so its latency overlaps the barrier and the exchange.
+// CUDANP_SCL_PF=2: also the next chunk's (or next item's) first pass-1 group is
+// issued right after pass 2's last loads, under pass 2's scans and stores.
+// A/B (profiles/exp_sclpf_*_r01o.jsonl, 16 x 4M and 256 x 256K int32): PF=1
+// +2-5 % on every cyclic cluster size, PF=2 up to -14 % (the 1024-thread CTAs'
+// 64-register cap spills the second group), so PF=1 is the default.
+#ifndef CUDANP_SCL_PF
+#define CUDANP_SCL_PF 1
+#endif
 
 template <class T, int S, bool VEC>
 __global__ void __launch_bounds__(S / kClusterCtas, 4096 / S > 0 ? 4096 / S : 1)
@@ -397,6 +407,8 @@ scan_cluster_cyclic_kernel(const T* __restrict__ in, const T* __restrict__ init,
     }
     return x;
   };
+  V4<T> nx[G];             // PF=2: the next chunk's first pass-1 group
+  bool have_nx = false;
   for (int64_t item = cid; item < N; item += ncl) {
     const T* irow = in + item * L;
     T* orow = out + item * L;
@@ -410,8 +422,13 @@ scan_cluster_cyclic_kernel(const T* __restrict__ in, const T* __restrict__ init,
       // pass 1: warp totals per round (G rounds' loads in flight at a time)
       for (int kg = 0; kg < rc; kg += G) {
         V4<T> v[G];
+        if (CUDANP_SCL_PF >= 2 && kg == 0 && have_nx) {
 #pragma unroll
-        for (int j = 0; j < G; ++j) v[j] = unit_load(irow, (k0 + kg + j) * S + rank * CTA + tid);
+          for (int j = 0; j < G; ++j) v[j] = nx[j];
+        } else {
+#pragma unroll
+          for (int j = 0; j < G; ++j) v[j] = unit_load(irow, (k0 + kg + j) * S + rank * CTA + tid);
+        }
 #pragma unroll
         for (int j = 0; j < G; ++j) {
           if (kg + j >= rc) break;
@@ -419,6 +436,11 @@ scan_cluster_cyclic_kernel(const T* __restrict__ in, const T* __restrict__ init,
           const T wi = warp_incl(ut);
           if (lane == 31) wt[kg + j][wid] = wi;
         }
+      }
+      V4<T> vv[G];
+      if constexpr (CUDANP_SCL_PF) {
+#pragma unroll
+        for (int j = 0; j < G; ++j) vv[j] = unit_load(irow, (k0 + j) * S + rank * CTA + tid);
       }
       if (!started) {  // CTA-uniform; see cluster_team_reduce
         cluster_wait();
@@ -464,9 +486,21 @@ scan_cluster_cyclic_kernel(const T* __restrict__ in, const T* __restrict__ init,
       __syncthreads();
       // pass 2: rescan and store
       for (int kg = 0; kg < rc; kg += G) {
-        V4<T> vv[G];
+        if (!CUDANP_SCL_PF || kg > 0) {
 #pragma unroll
-        for (int j = 0; j < G; ++j) vv[j] = unit_load(irow, (k0 + kg + j) * S + rank * CTA + tid);
+          for (int j = 0; j < G; ++j) vv[j] = unit_load(irow, (k0 + kg + j) * S + rank * CTA + tid);
+        }
+        if (CUDANP_SCL_PF >= 2 && kg + G >= rc) {  // last group: issue the next chunk's first loads
+          const bool same = k0 + RC < nrounds;
+          const int64_t nitem = same ? item : item + ncl;
+          const int64_t nk0 = same ? k0 + RC : 0;
+          have_nx = nitem < N;
+          if (have_nx) {
+            const T* nrow = in + nitem * L;
+#pragma unroll
+            for (int j = 0; j < G; ++j) nx[j] = unit_load(nrow, (nk0 + j) * S + rank * CTA + tid);
+          }
+        }
 #pragma unroll
         for (int j = 0; j < G; ++j) {
           if (kg + j >= rc) break;
