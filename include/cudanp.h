@@ -16,6 +16,15 @@
  *         CUDANP_MAP_INTER_WARP (team = one lane in each of S warps)
  *         (P:189-191), CUDANP_MAP_AUTO choosing per the rules of P:340-342.
  * S = 1 means no nesting: the tuned one-thread-per-item kernel.
+ * S in {3, 5, 10, 15} (Fig 12; "for inter-warp NP, such
+ * limitation can be removed"): teams that are not a power of two, built for
+ * the inter-warp map of the four hot-path calls (and cudanp_le_gicov);
+ * CUDANP_MAP_AUTO resolves to inter-warp for them, CUDANP_MAP_INTRA_WARP
+ * returns CUDANP_ERR_UNSUPPORTED.
+ * S = CUDANP_S_AUTO (0): the library chooses (S, dist, map) for the shape
+ * (cudanp_choose_version; `dist` is then ignored, `map` kept unless AUTO) --
+ * the paper's version selection as a rule distilled from the
+ * B200 sweeps, with no timing at call time (cudanp_autotune times them).
  * S in {64, 128, 256, 512, 1024} ("shared-memory fallback when S exceeds
  * 32"): a team of S/32 consecutive warps, shfl inside each warp and shared
  * memory across them; supported by the reduce, scan, MV and ragged-reduce
@@ -78,6 +87,7 @@ typedef enum {
                                     TMA bulk-copy ring (= cudanp_batched_loop_reduce_tma) */
 } cudanp_map;
 typedef enum { CUDANP_F32 = 0, CUDANP_I32 = 1 } cudanp_dtype;
+enum { CUDANP_S_AUTO = 0 }; /* S argument: the library picks the team size */
 typedef enum { CUDANP_SUM = 0, CUDANP_MAX = 1 } cudanp_op;
 
 /* ------------------------------------------------------------------------
@@ -89,7 +99,12 @@ typedef enum { CUDANP_SUM = 0, CUDANP_MAX = 1 } cudanp_op;
  * runs over the h = n_inner rows.  A: n_inner x lda fp32 (lda >= n_outer),
  * x: n_inner fp32, y: n_outer fp32.  fp32 FMA accumulation; the S partial
  * sums are combined by the team reduction.  map = CUDANP_MAP_INTER_WARP_TMA
- * runs cudanp_tmv_tma (S <= 32; its alignment preconditions apply). */
+ * runs the TMA-staged kernel (cudanp_tmv_tma) when S is a power of two <= 32
+ * and its preconditions hold, else the LDG inter-warp kernel (same result
+ * contract; never CUDANP_ERR_UNSUPPORTED for alignment).  CUDANP_MAP_AUTO
+ * takes the TMA-staged kernel under the same conditions when the matrix is
+ * wide (2 x ceil(n_outer/128) >= SM count), else the LDG inter-warp kernel
+ * (adjacent masters read adjacent columns). */
 int cudanp_tmv(const float* A, int64_t lda, const float* x, float* y,
                int64_t n_outer, int64_t n_inner, int S, int dist, int map, void* stream);
 
@@ -102,9 +117,13 @@ int cudanp_tmv(const float* A, int64_t lda, const float* x, float* y,
  * full/empty mbarrier pair per stage) and the slaves consume their rows,
  * cyclic or block (R5).  The shape makes the whole grid resident
  * at once.  Same result contract as cudanp_tmv (the S partial
- * sums meet in slave order).  Needs A and y 16-byte aligned, lda % 4 == 0,
- * n_outer % 4 == 0 and both sizes < 2^31, else CUDANP_ERR_UNSUPPORTED
- * (cudanp_tmv handles any case). */
+ * sums meet in slave order).  Needs A 16-byte aligned, lda % 4 == 0 and both
+ * sizes < 2^31 (TMA coordinates are int32), else CUDANP_ERR_UNSUPPORTED
+ * (cudanp_tmv handles any case); x and y need no alignment (y is written
+ * with scalar stores, so y may point into another buffer, e.g. a fused
+ * gather's root + begin).  Columns past n_outer and rows past n_inner are
+ * zero-filled by TMA and never stored; rows of a block-distribution box
+ * that belong to the next slave are skipped, not multiplied by zero. */
 int cudanp_tmv_tma(const float* A, int64_t lda, const float* x, float* y,
                    int64_t n_outer, int64_t n_inner, int S, int dist, void* stream);
 /* Same with the launch shape pinned (tuning / the sweep): cols in {0 = auto,
@@ -294,12 +313,26 @@ int cudanp_autotune(int op_kind, const void* a, const void* b, void* out, int64_
  * report the kernel's block size, grid size, registers per thread, static
  * shared memory bytes and the resolved map.  `op_kind`: 0 tmv, 1 mv,
  * 2 reduce, 3 scan, 4 TMA-staged tmv, 5 TMA-staged reduce (dynamic shared
- * memory of their rings in smem_bytes).  Any out pointer may be NULL.
+ * memory of their rings in smem_bytes).  vec4 != 0 states that the operands
+ * are 16-byte aligned with rows a multiple of 4 elements (the 128-bit and TMA
+ * paths).  S = CUDANP_S_AUTO and MAP_AUTO resolve as in the calls; the
+ * resolved map (CUDANP_MAP_INTER_WARP_TMA when TMV takes the TMA kernel), S
+ * and dist are returned.  Any out pointer may be NULL.
  * ---------------------------------------------------------------------- */
 int cudanp_launch_info(int op_kind, int64_t n_outer, int64_t n_inner, int dtype, int op,
                        int S, int dist, int map, int vec4,
                        int* block_threads, int64_t* grid_ctas, int* regs_per_thread,
-                       int* smem_bytes, int* resolved_map);
+                       int* smem_bytes, int* resolved_map, int* S_used, int* dist_used);
+
+/* The (S, dist, map) that S = CUDANP_S_AUTO selects for op_kind (0 tmv, 1 mv,
+ * 2 reduce, 3 scan) on N = n_outer items of L = n_inner iterations, given
+ * `map` (AUTO, or a map to keep) and vec4 as above.  Rule:
+ * TMV wide -> TMA S = 8 cyclic, else inter-warp S = clamp(SMs*1024/N, 8, 64);
+ * MV intra S = clamp(L/64, 1, 256); reduce intra S = clamp(L/8, 1, 32);
+ * scan intra S = clamp(L/4, 1, 16); reduce/scan/MV teams grow (up to S/32
+ * warps, slaves keeping >= 8 elements) while N*S < SMs*1024. */
+int cudanp_choose_version(int op_kind, int64_t n_outer, int64_t n_inner, int vec4, int map,
+                          int* S, int* dist, int* map_out);
 
 /* ------------------------------------------------------------------------
  * Multi-GPU helper (one process per GPU; outer items are independent,

@@ -88,15 +88,24 @@ static bool size_ok(int64_t a, int64_t b) {  // a*b*4 bytes addressable
   return a <= (INT64_MAX / 8) / b;
 }
 
+// inter_ok: the call also builds the non-power-of-two inter-warp teams
+// (valid_inter_S; intra-warp then returns CUDANP_ERR_UNSUPPORTED).
 static int check_common(int S, int dist, int map, int64_t n_outer, int64_t n_inner,
-                        bool cluster_ok = false) {
-  if (!valid_S(S) && !valid_big_S(S) && !(cluster_ok && valid_cluster_S(S)))
-    return fail_invalid(cluster_ok ? "S must be one of 1,2,4,8,16,32 (64..1024 multi-warp teams, "
-                                     "2048/4096/8192 cluster teams)"
-                                   : "S must be one of 1,2,4,8,16,32 (or 64..1024 for multi-warp teams)");
+                        bool cluster_ok = false, bool inter_ok = false) {
+  if (!valid_S(S) && !valid_big_S(S) && !(cluster_ok && valid_cluster_S(S)) &&
+      !(inter_ok && valid_inter_S(S)))
+    return fail_invalid(cluster_ok ? "S must be one of 1,2,4,8,16,32 (3,5,10,15 inter-warp; 64..1024 "
+                                     "multi-warp teams, 2048/4096/8192 cluster teams)"
+                                   : "S must be one of 1,2,4,8,16,32 (3,5,10,15 inter-warp; 64..1024 "
+                                     "multi-warp teams)");
   if (dist != CUDANP_DIST_CYCLIC && dist != CUDANP_DIST_BLOCK) return fail_invalid("dist");
   if (map != CUDANP_MAP_AUTO && map != CUDANP_MAP_INTRA_WARP && map != CUDANP_MAP_INTER_WARP)
     return fail_invalid("map");
+  if (valid_inter_S(S) && map == CUDANP_MAP_INTRA_WARP) {
+    set_error("intra-warp teams need S = 2^k <= 32 (P:342); S = %d runs with the inter-warp map "
+              "(P:447)", S);
+    return CUDANP_ERR_UNSUPPORTED;
+  }
   if (n_outer < 0 || n_inner < 0) return fail_invalid("negative size");
   if (!size_ok(n_outer, n_inner)) return fail_invalid("size overflows int64 byte offsets");
   return CUDANP_OK;
@@ -111,14 +120,116 @@ static int check_dtype_op(int dtype, int op) {
 // MAP_AUTO per P:340-342 / P:486: keep the access pattern coalesced.  TMV's
 // masters (columns) are adjacent in memory -> inter-warp; MV rows and
 // item-major reduce/scan rows are contiguous per master -> intra-warp.
-static int resolve_map(int map, bool is_tmv) {
+// A team that is not a power of two exists only as an inter-warp team.
+static int resolve_map(int map, bool is_tmv, int S = 1) {
   if (map != CUDANP_MAP_AUTO) return map;
-  return is_tmv ? MAP_INTER : MAP_INTRA;
+  return (is_tmv || valid_inter_S(S)) ? MAP_INTER : MAP_INTRA;
+}
+
+// ---------------------------------------------------------------- version choice
+static int floor_pow2(int64_t v) {
+  int p = 1;
+  while ((int64_t)p * 2 <= v && p < (1 << 30)) p *= 2;
+  return p;
+}
+static int clampi(int v, int lo, int hi) { return v < lo ? lo : (v > hi ? hi : v); }
+
+// TMA staging of TMV pays when the 128-column strips give at least half the
+// SMs a CTA each (the regime where the 4-wide LDG kernel is also used); on
+// narrower matrices (C1, 1024 columns: TMA S = 32 5.1 us vs LDG inter-warp
+// 3.2 us, profiles/sweep_r01n.jsonl) the LDG inter-warp kernel with more
+// slaves per column spreads the few columns better.
+static bool tmv_wide(int64_t w) { return 2 * ((w + 127) / 128) >= sm_count(); }
+// TMA preconditions: A 16-byte aligned, row pitch a multiple of 16 bytes,
+// coordinates in int32, something to stream.  y is stored with scalar stores
+// and x with ordinary loads, so neither needs alignment.
+static bool tma_ok(const float* A, int64_t lda, int64_t w, int64_t h) {
+  return aligned16(A) && lda % 4 == 0 && w > 0 && h > 0 && w < (int64_t(1) << 31) &&
+         h < (int64_t(1) << 31);
+}
+
+// The library's choice of (S, dist, map) when the caller passes S = 0
+// (CUDANP_S_AUTO): the paper picks the version by exhaustive search (P:413,
+// P:486); this rule encodes what that search found on B200 (DESIGN.md §6,
+// profiles/sweep_r01n.jsonl, bench_r01*.json), so no call has to time
+// anything.  T = SMs x 1024 threads is "enough threads to fill the GPU":
+// when N x S falls short, the team grows (NP pays when outer
+// TLP is short), up to a team whose slaves still get >= 8 elements each.
+//   TMV: wide + TMA-able -> TMA, S = 8 cyclic (C2 best); else inter-warp LDG
+//        with S = clamp(T / w, 8, 64), block when S >= 64 (C1 best: 64 block).
+//   MV:  intra, S = clamp(L / 64, 1, 256) cyclic (C2 best: S = 256), grown.
+//   reduce: intra, S = clamp(L / 8, 1, 32) (C3: 4/8/16/32 at L = 32..256),
+//        block above L = 32 (L % 4 != 0: L / 16), grown.
+//   scan: intra, S = clamp(L / 4, 1, 16) (C4: 16), cyclic from L = 128, grown.
+// A map other than AUTO is kept (and the S chosen for it).
+int choose_version(int op_kind, int64_t N, int64_t L, bool vec, bool tma, int map_in, int* S,
+                   int* dist, int* map) {
+  const int64_t T = (int64_t)sm_count() * 1024;
+  auto grow = [&](int s, int cap) {
+    while ((int64_t)s * 2 <= cap && N * s < T) s *= 2;
+    return s;
+  };
+  const int cap_l8 = clampi(floor_pow2(L / 8), 1, 1024);
+  int s = 1, d = CUDANP_DIST_CYCLIC, m = map_in;
+  switch (op_kind) {
+    case 0:  // TMV: N = w columns, L = h rows
+      if ((map_in == CUDANP_MAP_AUTO || map_in == CUDANP_MAP_INTER_WARP_TMA) && tma && tmv_wide(N)) {
+        s = 8; d = CUDANP_DIST_CYCLIC; m = CUDANP_MAP_INTER_WARP_TMA;
+        break;
+      }
+      if (m == CUDANP_MAP_INTER_WARP_TMA) m = CUDANP_MAP_INTER_WARP;  // fallback (not TMA-able)
+      if (m == CUDANP_MAP_INTRA_WARP) {
+        s = clampi(floor_pow2(N > 0 ? T / N : 32), 1, 32);
+      } else {
+        m = CUDANP_MAP_INTER_WARP;
+        s = clampi(floor_pow2(N > 0 ? T / N : 64), 8, 64);
+        d = s >= 64 ? CUDANP_DIST_BLOCK : CUDANP_DIST_CYCLIC;
+      }
+      s = clampi(s, 1, clampi(floor_pow2(L / 4), 1, 64));
+      break;
+    case 1:  // MV
+      if (m == CUDANP_MAP_INTER_WARP) {
+        s = clampi(floor_pow2(L / 128), 1, 32);
+      } else {
+        m = CUDANP_MAP_INTRA_WARP;
+        s = clampi(floor_pow2(L / 64), 1, 256);
+        s = grow(s, cap_l8 > s ? cap_l8 : s);
+      }
+      break;
+    case 2:  // batched reduce
+      if (m == CUDANP_MAP_INTER_WARP) {
+        s = clampi(floor_pow2(L / 32), 1, 32);
+      } else {
+        m = CUDANP_MAP_INTRA_WARP;
+        s = clampi(floor_pow2(vec ? L / 8 : L / 16), 1, 32);
+        d = L > 32 ? CUDANP_DIST_BLOCK : CUDANP_DIST_CYCLIC;
+        s = grow(s, cap_l8);
+        if (s > 32) d = CUDANP_DIST_CYCLIC;
+      }
+      break;
+    case 3:  // batched scan
+      if (m == CUDANP_MAP_INTER_WARP) {
+        s = clampi(floor_pow2(L / 32), 1, 32);
+      } else {
+        m = CUDANP_MAP_INTRA_WARP;
+        s = clampi(floor_pow2(L / 4), 1, 16);
+        d = L >= 128 ? CUDANP_DIST_CYCLIC : CUDANP_DIST_BLOCK;
+        s = grow(s, cap_l8);
+        if (s > 32) d = CUDANP_DIST_CYCLIC;
+      }
+      break;
+    default:
+      return fail_invalid("op_kind");
+  }
+  *S = s;
+  *dist = d;
+  *map = m;
+  return CUDANP_OK;
 }
 
 static int check_tmv_args(const float* A, int64_t lda, const float* x, float* y, int64_t w,
                           int64_t h, int S, int dist, int map) {
-  int rc = check_common(S, dist, map, w, h);
+  int rc = check_common(S, dist, map, w, h, false, true);
   if (rc) return rc;
   if (w > 0 && h > 0 && lda < w) return fail_invalid("lda < n_outer (TMV row length)");
   if (!size_ok(h, lda)) return fail_invalid("h*lda overflows");
@@ -129,7 +240,7 @@ static int check_tmv_args(const float* A, int64_t lda, const float* x, float* y,
 
 static int check_mv_args(const float* A, int64_t lda, const float* x, float* y, int64_t h,
                          int64_t w, int S, int dist, int map) {
-  int rc = check_common(S, dist, map, h, w, true);
+  int rc = check_common(S, dist, map, h, w, true, true);
   if (rc) return rc;
   if (h > 0 && w > 0 && lda < w) return fail_invalid("lda < n_inner (MV row length)");
   if (!size_ok(h, lda)) return fail_invalid("h*lda overflows");
@@ -245,7 +356,7 @@ static cudaStream_t as_stream(void* s) { return (cudaStream_t)s; }
 
 extern "C" {
 
-int cudanp_version(void) { return 100; }
+int cudanp_version(void) { return 200; }
 
 const char* cudanp_status_string(int status) {
   switch (status) {
@@ -260,13 +371,27 @@ const char* cudanp_status_string(int status) {
 
 const char* cudanp_last_error(void) { return g_err; }
 
+// Version selection inside the call.  S = CUDANP_S_AUTO
+// picks (S, dist, map) by choose_version.  MAP_AUTO takes the TMA-staged
+// inter-warp kernel when its preconditions hold, S <= 32 is a power of two
+// and the matrix is wide (tmv_wide), else the LDG inter-warp kernel (P:340:
+// masters = adjacent columns).  MAP_INTER_WARP_TMA falls back to the LDG
+// inter-warp kernel (same result contract) where TMA cannot run.
 int cudanp_tmv(const float* A, int64_t lda, const float* x, float* y, int64_t n_outer,
                int64_t n_inner, int S, int dist, int map, void* stream) {
-  if (map == CUDANP_MAP_INTER_WARP_TMA)
-    return cudanp_tmv_tma_ex(A, lda, x, y, n_outer, n_inner, S, dist, 0, -1, 0, stream);
-  int rc = check_tmv_args(A, lda, x, y, n_outer, n_inner, S, dist, map);
+  const bool tma = tma_ok(A, lda, n_outer, n_inner);
+  if (S == CUDANP_S_AUTO) {
+    if (map < CUDANP_MAP_AUTO || map > CUDANP_MAP_INTER_WARP_TMA) return fail_invalid("map");
+    choose_version(0, n_outer, n_inner, tmv_vec(A, lda, y, n_outer), tma, map, &S, &dist, &map);
+  }
+  const int m = map == CUDANP_MAP_INTER_WARP_TMA ? CUDANP_MAP_INTER_WARP : map;
+  int rc = check_tmv_args(A, lda, x, y, n_outer, n_inner, S, dist, m);
   if (rc) return rc;
-  return tmv_np(A, lda, x, y, n_outer, n_inner, S, dist, resolve_map(map, true),
+  const bool use_tma = valid_S(S) && tma &&
+                       (map == CUDANP_MAP_INTER_WARP_TMA || (map == CUDANP_MAP_AUTO && tmv_wide(n_outer)));
+  if (use_tma)
+    return tmv_tma(A, lda, x, y, n_outer, n_inner, S, dist, 0, -1, 0, as_stream(stream), nullptr);
+  return tmv_np(A, lda, x, y, n_outer, n_inner, S, dist, resolve_map(m, true, S),
                 tmv_vec(A, lda, y, n_outer), as_stream(stream), nullptr);
 }
 
@@ -278,9 +403,8 @@ int cudanp_tmv_tma_ex(const float* A, int64_t lda, const float* x, float* y, int
   if (n_outer == 0) return CUDANP_OK;
   if (n_inner == 0)  // nothing to stream: the plain kernel writes the zeros
     return tmv_np(A, lda, x, y, n_outer, n_inner, S, dist, MAP_INTER, false, as_stream(stream), nullptr);
-  if (!(aligned16(A) && aligned16(y) && lda % 4 == 0 && n_outer % 4 == 0 &&
-        n_outer < (int64_t(1) << 31) && n_inner < (int64_t(1) << 31))) {
-    set_error("TMA path needs 16-byte aligned A and y, lda %% 4 == 0, n_outer %% 4 == 0, sizes < 2^31");
+  if (!tma_ok(A, lda, n_outer, n_inner)) {
+    set_error("TMA path needs a 16-byte aligned A, lda %% 4 == 0 and sizes < 2^31");
     return CUDANP_ERR_UNSUPPORTED;
   }
   return tmv_tma(A, lda, x, y, n_outer, n_inner, S, dist, cols, rows_sel, stages, as_stream(stream),
@@ -294,9 +418,13 @@ int cudanp_tmv_tma(const float* A, int64_t lda, const float* x, float* y, int64_
 
 int cudanp_mv(const float* A, int64_t lda, const float* x, float* y, int64_t n_outer,
               int64_t n_inner, int S, int dist, int map, void* stream) {
+  if (S == CUDANP_S_AUTO) {
+    if (map < CUDANP_MAP_AUTO || map > CUDANP_MAP_INTER_WARP) return fail_invalid("map");
+    choose_version(1, n_outer, n_inner, mv_vec(A, lda, x, n_inner), false, map, &S, &dist, &map);
+  }
   int rc = check_mv_args(A, lda, x, y, n_outer, n_inner, S, dist, map);
   if (rc) return rc;
-  return mv_np(A, lda, x, y, n_outer, n_inner, S, dist, resolve_map(map, false),
+  return mv_np(A, lda, x, y, n_outer, n_inner, S, dist, resolve_map(map, false, S),
                mv_vec(A, lda, x, n_inner), as_stream(stream), nullptr);
 }
 
@@ -304,7 +432,7 @@ int cudanp_mv(const float* A, int64_t lda, const float* x, float* y, int64_t n_o
 // writes N*L values, so out may be NULL when L = 0.
 static int check_batched(const void* in, void* out, int64_t N, int64_t L, int S, int dist, int map,
                          int dtype, int op, bool out_per_item, bool cluster_ok = false) {
-  int rc = check_common(S, dist, map, N, L, cluster_ok);
+  int rc = check_common(S, dist, map, N, L, cluster_ok, cluster_ok);
   if (rc) return rc;
   rc = check_dtype_op(dtype, op);
   if (rc) return rc;
@@ -335,13 +463,18 @@ int cudanp_batched_loop_reduce_tma(const void* in, const void* init, void* out, 
 int cudanp_batched_loop_reduce(const void* in, const void* init, void* out, int64_t n_outer,
                                int64_t n_inner, int dtype, int op, int S, int dist, int map,
                                void* stream) {
-  if (map == CUDANP_MAP_INTRA_WARP_TMA)
+  if (map == CUDANP_MAP_INTRA_WARP_TMA && S != CUDANP_S_AUTO)
     return cudanp_batched_loop_reduce_tma(in, init, out, n_outer, n_inner, dtype, op, S, dist, 0, 0,
                                           stream);
+  const bool vec = (n_inner % 4 == 0) && aligned16(in);
+  if (S == CUDANP_S_AUTO) {
+    if (map < CUDANP_MAP_AUTO || map > CUDANP_MAP_INTRA_WARP_TMA) return fail_invalid("map");
+    if (map == CUDANP_MAP_INTRA_WARP_TMA) map = CUDANP_MAP_INTRA_WARP;
+    choose_version(2, n_outer, n_inner, vec, false, map, &S, &dist, &map);
+  }
   int rc = check_batched(in, out, n_outer, n_inner, S, dist, map, dtype, op, true, true);
   if (rc) return rc;
-  const bool vec = (n_inner % 4 == 0) && aligned16(in);
-  return reduce_np(in, init, out, n_outer, n_inner, dtype, op, S, dist, resolve_map(map, false),
+  return reduce_np(in, init, out, n_outer, n_inner, dtype, op, S, dist, resolve_map(map, false, S),
                    vec, as_stream(stream), nullptr);
 }
 
@@ -360,10 +493,14 @@ int cudanp_batched_loop_reduce_backend(const void* in, const void* init, void* o
 
 int cudanp_batched_loop_scan(const void* in, const void* init, void* out, int64_t n_outer,
                              int64_t n_inner, int dtype, int S, int dist, int map, void* stream) {
+  const bool vec = (n_inner % 4 == 0) && aligned16(in) && aligned16(out);
+  if (S == CUDANP_S_AUTO) {
+    if (map < CUDANP_MAP_AUTO || map > CUDANP_MAP_INTER_WARP) return fail_invalid("map");
+    choose_version(3, n_outer, n_inner, vec, false, map, &S, &dist, &map);
+  }
   int rc = check_batched(in, out, n_outer, n_inner, S, dist, map, dtype, CUDANP_SUM, false, true);
   if (rc) return rc;
-  const bool vec = (n_inner % 4 == 0) && aligned16(in) && aligned16(out);
-  return scan_np(in, init, out, n_outer, n_inner, dtype, S, dist, resolve_map(map, false), vec,
+  return scan_np(in, init, out, n_outer, n_inner, dtype, S, dist, resolve_map(map, false, S), vec,
                  as_stream(stream), nullptr);
 }
 
@@ -530,12 +667,26 @@ int cudanp_dp_memcopy(const float* in, float* out, int64_t total, int64_t m, int
 // ---------------------------------------------------------------- launch info
 int cudanp_launch_info(int op_kind, int64_t n_outer, int64_t n_inner, int dtype, int op, int S,
                        int dist, int map, int vec4, int* block_threads, int64_t* grid_ctas,
-                       int* regs_per_thread, int* smem_bytes, int* resolved_map) {
-  int rc = check_common(S, dist, map, n_outer, n_inner, op_kind >= 1 && op_kind <= 3);
+                       int* regs_per_thread, int* smem_bytes, int* resolved_map, int* S_used,
+                       int* dist_used) {
+  const bool v = vec4 != 0;
+  if (S == CUDANP_S_AUTO && op_kind >= 0 && op_kind <= 3) {
+    if (map < CUDANP_MAP_AUTO || map > (op_kind == 0 ? CUDANP_MAP_INTER_WARP_TMA : CUDANP_MAP_INTER_WARP))
+      return fail_invalid("map");
+    choose_version(op_kind, n_outer, n_inner, v, v, map, &S, &dist, &map);
+  }
+  // TMV: MAP_AUTO / MAP_INTER_WARP_TMA resolve as cudanp_tmv does (vec4 stands
+  // for the TMA preconditions).
+  if (op_kind == 0 && valid_S(S) && v && n_outer > 0 && n_inner > 0 &&
+      (map == CUDANP_MAP_INTER_WARP_TMA || (map == CUDANP_MAP_AUTO && tmv_wide(n_outer))))
+    op_kind = 4;
+  if (op_kind == 0 && map == CUDANP_MAP_INTER_WARP_TMA) map = CUDANP_MAP_INTER_WARP;
+  if (op_kind == 4) map = CUDANP_MAP_INTER_WARP;
+  int rc = check_common(S, dist, map, n_outer, n_inner, op_kind >= 1 && op_kind <= 3,
+                        op_kind <= 3);
   if (rc) return rc;
   LaunchInfo info;
-  const bool v = vec4 != 0;
-  const int m = resolve_map(map, op_kind == 0);
+  const int m = resolve_map(map, op_kind == 0, S);
   switch (op_kind) {
     case 0: rc = tmv_np(nullptr, 0, nullptr, nullptr, n_outer, n_inner, S, dist, m, v, 0, &info); break;
     case 1: rc = mv_np(nullptr, 0, nullptr, nullptr, n_outer, n_inner, S, dist, m, v, 0, &info); break;
@@ -563,8 +714,20 @@ int cudanp_launch_info(int op_kind, int64_t n_outer, int64_t n_inner, int dtype,
   if (grid_ctas) *grid_ctas = info.grid;
   if (regs_per_thread) *regs_per_thread = info.regs;
   if (smem_bytes) *smem_bytes = info.smem;
-  if (resolved_map) *resolved_map = info.map;
+  if (resolved_map) *resolved_map = op_kind == 4 ? CUDANP_MAP_INTER_WARP_TMA : info.map;
+  if (S_used) *S_used = S;
+  if (dist_used) *dist_used = dist;
   return CUDANP_OK;
+}
+
+int cudanp_choose_version(int op_kind, int64_t n_outer, int64_t n_inner, int vec4, int map, int* S,
+                          int* dist, int* map_out) {
+  if (op_kind < 0 || op_kind > 3) return fail_invalid("op_kind");
+  if (n_outer < 0 || n_inner < 0) return fail_invalid("negative size");
+  if (map < CUDANP_MAP_AUTO || map > (op_kind == 0 ? CUDANP_MAP_INTER_WARP_TMA : CUDANP_MAP_INTER_WARP))
+    return fail_invalid("map");
+  if (!S || !dist || !map_out) return fail_invalid("NULL output");
+  return choose_version(op_kind, n_outer, n_inner, vec4 != 0, vec4 != 0, map, S, dist, map_out);
 }
 
 // ---------------------------------------------------------------- CUDA IPC (f4)

@@ -102,9 +102,14 @@ int cudanp_autotune(int op_kind, const void* a, const void* b, void* out, int64_
         cudaEventElapsedTime(&ms, e0, e1);
         ms /= reps;
       }
-    } else if (r == CUDANP_ERR_CUDA && c[i].map < CUDANP_MAP_INTER_WARP_TMA) {
-      rc = r;
-      break;
+    } else if (r == CUDANP_ERR_CUDA) {
+      // A launch that the device refused (a configuration this device cannot
+      // run) skips the candidate; a device that faulted ends the search.
+      if (cudaStreamSynchronize(st) != cudaSuccess || cudaGetLastError() != cudaSuccess) {
+        rc = check_launch("autotune: device error after a candidate");
+        if (!rc) rc = CUDANP_ERR_CUDA;
+        break;
+      }
     }
     if (ms_table) ms_table[i] = ms;
     if (ms < best_ms) { best_ms = ms; best = (int)i; }

@@ -30,6 +30,13 @@ inline int check_launch(const char* what) {
 inline bool valid_S(int S) {
   return S == 1 || S == 2 || S == 4 || S == 8 || S == 16 || S == 32;
 }
+// Inter-warp teams need not be a power of two (the padding limit of
+// intra-warp NP "can be removed" for inter-warp NP; Fig 12, uses 3, 5,
+// 10 and 15): these S are built for the inter-warp map of TMV, MV, the
+// batched reduce and the batched scan (and the LE kernel, np_le.cu).
+inline bool valid_inter_S(int S) { return S == 3 || S == 5 || S == 10 || S == 15; }
+template <int S> constexpr bool kPow2 = S > 0 && (S & (S - 1)) == 0;
+
 // Teams larger than a warp (S/32 consecutive warps; shfl within each warp,
 // shared memory across them): batched reduce/scan and MV with the intra-warp
 // (consecutive-thread) map, TMV with the inter-warp map for S <= 128.
@@ -126,4 +133,13 @@ struct LaunchInfo {
     case 16: { constexpr int kS = 16; __VA_ARGS__; } break; \
     case 32: { constexpr int kS = 32; __VA_ARGS__; } break; \
     default: return fail_invalid("S must be one of 1,2,4,8,16,32"); \
+  }
+// The non-power-of-two inter-warp team sizes (valid_inter_S).
+#define CUDANP_DISPATCH_S_INTER(S, ...)                  \
+  switch (S) {                                           \
+    case 3: { constexpr int kS = 3; __VA_ARGS__; } break;   \
+    case 5: { constexpr int kS = 5; __VA_ARGS__; } break;   \
+    case 10: { constexpr int kS = 10; __VA_ARGS__; } break; \
+    case 15: { constexpr int kS = 15; __VA_ARGS__; } break; \
+    default: return fail_invalid("inter-warp S must be one of 1..32 listed in cudanp.h"); \
   }

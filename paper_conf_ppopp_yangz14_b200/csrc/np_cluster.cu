@@ -32,9 +32,15 @@ template <class T>
 __device__ __forceinline__ T sum4(V4<T> v) {
   return OpSum::apply(OpSum::apply(v.x, v.y), OpSum::apply(v.z, v.w));
 }
-// a - b, int32 wrapping modulo 2^32 (R13)
-__device__ __forceinline__ float tsub_c(float a, float b) { return a - b; }
-__device__ __forceinline__ int32_t tsub_c(int32_t a, int32_t b) { return (int32_t)((uint32_t)a - (uint32_t)b); }
+// Exclusive prefix inside a warp from the inclusive one: the previous lane's
+// inclusive value (0 for lane 0).  Taken by a shuffle, not as incl - own, so
+// an fp32 exclusive value is the sum of the earlier lanes' terms themselves
+// (no cancellation error).  Every lane of the warp must call it.
+template <class T>
+__device__ __forceinline__ T warp_prev(T incl) {
+  const T t = __shfl_up_sync(kFull, incl, 1);
+  return (threadIdx.x & 31) == 0 ? T(0) : t;
+}
 
 template <class T, class Op>
 __device__ __forceinline__ V4<T> cop4(V4<T> a, V4<T> b) {
@@ -90,38 +96,6 @@ __device__ __forceinline__ void cluster_arrive_relaxed() {
 __device__ __forceinline__ void cluster_wait() {
   asm volatile("barrier.cluster.wait.aligned;" ::: "memory");
 }
-
-// Push-mode exchange primitives (CUDANP_SCL_PUSH): a value is stored into
-// another CTA's shared memory with st.async, its bytes counted on that CTA's
-// mbarrier, so the receiver waits on its own barrier instead of a cluster-wide
-// barrier (whose release half drains every outstanding global store).
-__device__ __forceinline__ uint32_t mapa_u32(const void* p, int rank) {
-  uint32_t r;
-  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"((uint32_t)__cvta_generic_to_shared(p)), "r"(rank));
-  return r;
-}
-__device__ __forceinline__ void st_async_b32(uint32_t raddr, uint32_t v, uint32_t rbar) {
-  asm volatile("st.async.shared::cluster.mbarrier::complete_tx::bytes.b32 [%0], %1, [%2];"
-               ::"r"(raddr), "r"(v), "r"(rbar) : "memory");
-}
-__device__ __forceinline__ void mbar_init_u32(uint64_t* b, uint32_t count) {
-  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"((uint32_t)__cvta_generic_to_shared(b)), "r"(count) : "memory");
-}
-__device__ __forceinline__ void mbar_arm(uint64_t* b, uint32_t bytes) {
-  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"((uint32_t)__cvta_generic_to_shared(b)), "r"(bytes) : "memory");
-}
-__device__ __forceinline__ void mbar_wait_cluster(uint64_t* b, uint32_t parity) {
-  asm volatile(
-      "{\n .reg .pred p;\n"
-      "WAITC_%=:\n"
-      " mbarrier.try_wait.parity.acquire.cluster.shared::cta.b64 p, [%0], %1;\n"
-      " @!p bra WAITC_%=;\n}" ::"r"((uint32_t)__cvta_generic_to_shared(b)), "r"(parity) : "memory");
-}
-__device__ __forceinline__ void fence_mbar_init_cluster() {
-  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-}
-__device__ __forceinline__ uint32_t as_u32(float v) { return __float_as_uint(v); }
-__device__ __forceinline__ uint32_t as_u32(int32_t v) { return (uint32_t)v; }
 
 // ---------------------------------------------------------------- batched reduce
 template <class T, class Op, int S, int DIST, bool VEC>
@@ -318,7 +292,7 @@ scan_cluster_kernel(const T* __restrict__ in, const T* __restrict__ init, T* __r
     }
     __syncthreads();
     // pass 2: rescan the chunk from this slave's offset and store
-    T run = OpSum::apply(off[par], OpSum::apply(wpre, tsub_c(incl, csum)));
+    T run = OpSum::apply(off[par], OpSum::apply(wpre, warp_prev(incl)));
     u = r.begin;
     for (; u + U <= r.end; u += U) {
       if constexpr (VEC) {
@@ -373,9 +347,8 @@ scan_cluster_kernel(const T* __restrict__ in, const T* __restrict__ init, T* __r
 // chunks of RC rounds, two passes per chunk:
 //   pass 1: each warp scans its units of every round of the chunk
 //           (shfl-up) and keeps the warp totals wt[k][w] in shared
-//           memory; the CTA totals tot[k] are pushed into every CTA's shared
-//           memory (CUDANP_SCL_PUSH, below, off by default) or published
-//           locally behind one cluster barrier (default);
+//           memory; the CTA totals tot[k] are published locally behind one
+//           cluster barrier;
 //   exchange: thread k reads the 8 CTAs' tot[k] (and the master
 //           CTA's carry-in init[n], read_from_master one level up) and the
 //           CTA turns them into the offset of each (round, warp) -- every CTA
@@ -392,20 +365,10 @@ constexpr int kScanG = 8;    // rounds whose loads are in flight together
 // cluster barrier, so its latency overlaps the barrier and the exchange.
 // CUDANP_SCL_PF=2: also the next chunk's (or next item's) first pass-1 group is
 // issued right after pass 2's last loads, under pass 2's scans and stores.
-// CUDANP_SCL_PUSH=1: the per-chunk cluster barrier is replaced by pushes of the
-// per-round totals (and rank 0's carry-in) into every CTA's shared memory with
-// st.async, counted on a double-buffered receiver-side mbarrier.  A rank pushes
-// chunk c+2 into parity slot p only after it has received everyone's chunk c+1,
-// which each receiver pushes only after reading slot p for chunk c, so no
-// barrier guards the reuse.  The cluster barrier's release half (MEMBAR.ALL.GPU)
-// drained every outstanding pass-2 store before each exchange; the pushes do
-// not: +5-9 % on every cyclic cluster size (profiles/exp_push_*_r01p.jsonl),
-// parity green, memcheck and racecheck clean -- but compute-sanitizer synccheck
-// reports warp 0 divergent at the CTA barrier after the exchange (also with a
-// single spinning lane, which loses the gain), so it stays off by default.
-#ifndef CUDANP_SCL_PUSH
-#define CUDANP_SCL_PUSH 0
-#endif
+// A push exchange (st.async of the per-round totals into every CTA's shared
+// memory, counted on mbarriers, instead of the cluster barrier) was measured
+// at +5-9 % in round 1 but rejected: compute-sanitizer synccheck reported a
+// divergent warp at the CTA barrier after the exchange.
 // A/B (profiles/exp_sclpf_*_r01o.jsonl, 16 x 4M and 256 x 256K int32): PF=1
 // +2-5 % on every cyclic cluster size, PF=2 up to -14 % (the 1024-thread CTAs'
 // 64-register cap spills the second group), so PF=1 is the default.
@@ -429,25 +392,12 @@ scan_cluster_cyclic_kernel(const T* __restrict__ in, const T* __restrict__ init,
   __shared__ T tot[2][RC];       // this CTA's per-round totals (read over DSMEM)
   __shared__ T cin[2];           // the master CTA's carry-in
   __shared__ T carry_s;
-  constexpr bool PUSH = CUDANP_SCL_PUSH != 0;
-  constexpr uint32_t kPushBytes = (kClusterCtas * RC + 1) * 4;  // every rank's RC totals + the carry-in
-  __shared__ T rcv[2][kClusterCtas][RC];  // PUSH: totals pushed by each rank
-  __shared__ T rcin[2];                   // PUSH: carry-in pushed by rank 0
-  __shared__ __align__(8) uint64_t mb[2];
-  uint32_t mph = 0;                       // PUSH: phase bit of mb[0] (bit 0) and mb[1] (bit 1)
   cg::cluster_group cluster = cg::this_cluster();
   const int rank = (int)cluster.block_rank();
   const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
   const int64_t nunits = VEC ? (L >> 2) : L;
   const int64_t nrounds = (nunits + S - 1) / S;
   const int64_t cid = blockIdx.x / kClusterCtas, ncl = gridDim.x / kClusterCtas;
-  if (PUSH && tid == 0) {
-    mbar_init_u32(&mb[0], 1);
-    mbar_init_u32(&mb[1], 1);
-    mbar_arm(&mb[0], kPushBytes);
-    mbar_arm(&mb[1], kPushBytes);
-    fence_mbar_init_cluster();
-  }
   cluster_arrive_relaxed();
   bool started = false;
   int par = 0;
@@ -507,44 +457,20 @@ scan_cluster_cyclic_kernel(const T* __restrict__ in, const T* __restrict__ init,
         started = true;
       }
       __syncthreads();
-      if constexpr (PUSH) {
-        if (wid == 0) {
-          T c = T(0);
-          if (lane < rc) {
-            c = wt[lane][0];
+      if (tid < rc) {
+        T c = wt[tid][0];
 #pragma unroll
-            for (int w = 1; w < W; ++w) c = OpSum::apply(c, wt[lane][w]);
-          }
-          if (lane < RC) {  // rounds >= rc push 0 so the byte count is constant
-#pragma unroll
-            for (int r = 0; r < kClusterCtas; ++r)
-              st_async_b32(mapa_u32(&rcv[par][rank][lane], r), as_u32(c), mapa_u32(&mb[par], r));
-          } else if (lane == 31 && rank == 0) {
-            const T ci = (first && init) ? init[item] : T(0);  // the master's sequential section
-            for (int r = 0; r < kClusterCtas; ++r)
-              st_async_b32(mapa_u32(&rcin[par], r), as_u32(ci), mapa_u32(&mb[par], r));
-          }
-          mbar_wait_cluster(&mb[par], (mph >> par) & 1u);
-          mph ^= 1u << par;
-          __syncwarp();
-          if (lane == 0) mbar_arm(&mb[par], kPushBytes);  // next use of this buffer (chunk + 2)
-        }
-      } else {
-        if (tid < rc) {
-          T c = wt[tid][0];
-#pragma unroll
-          for (int w = 1; w < W; ++w) c = OpSum::apply(c, wt[tid][w]);
-          tot[par][tid] = c;
-        }
-        cluster.sync();  // every CTA's tot[par] (and the carry-in) visible cluster-wide
+        for (int w = 1; w < W; ++w) c = OpSum::apply(c, wt[tid][w]);
+        tot[par][tid] = c;
       }
+      cluster.sync();  // every CTA's tot[par] (and the carry-in) visible cluster-wide
       // exchange: lane k of warp 0 gathers round k's totals of all ranks
       if (wid == 0) {
         T rowt = T(0), low = T(0);
         if (lane < rc) {
 #pragma unroll
           for (int r = 0; r < kClusterCtas; ++r) {
-            const T t = PUSH ? rcv[par][r][lane] : *cluster.map_shared_rank(&tot[par][lane], r);
+            const T t = *cluster.map_shared_rank(&tot[par][lane], r);
             rowt = OpSum::apply(rowt, t);
             if (r < rank) low = OpSum::apply(low, t);
           }
@@ -552,9 +478,9 @@ scan_cluster_cyclic_kernel(const T* __restrict__ in, const T* __restrict__ init,
         const T incl = warp_incl(rowt);                   // rounds 0..k of the chunk
         const T chunk_total = __shfl_sync(kFull, incl, 31);
         T base = carry_s;
-        if (first) base = OpSum::apply(base, PUSH ? rcin[par] : *cluster.map_shared_rank(&cin[par], 0));
+        if (first) base = OpSum::apply(base, *cluster.map_shared_rank(&cin[par], 0));
         // offset of round k for this CTA = base + rounds < k + lower ranks in round k
-        const T offk = OpSum::apply(base, OpSum::apply(tsub_c(incl, rowt), low));
+        const T offk = OpSum::apply(base, OpSum::apply(warp_prev(incl), low));
         if (lane < rc) {
           T o = offk;
 #pragma unroll
@@ -595,7 +521,7 @@ scan_cluster_cyclic_kernel(const T* __restrict__ in, const T* __restrict__ init,
           }
           const T ut = VEC ? v.w : v.x;
           const T wi = warp_incl(ut);
-          const T add = OpSum::apply(offw[kg + j][wid], tsub_c(wi, ut));
+          const T add = OpSum::apply(offw[kg + j][wid], warp_prev(wi));
           if (u < nunits) {
             if constexpr (VEC)
               stg4(orow + 4 * u, V4<T>{OpSum::apply(add, v.x), OpSum::apply(add, v.y),
@@ -640,8 +566,12 @@ static int launch_cluster(void (*kern)(KArgs...), int cta, int64_t N, cudaStream
   int resident = 0;
   cfg.gridDim = dim3(kClusterCtas);
   if (cudaOccupancyMaxActiveClusters(&resident, (void*)kern, &cfg) != cudaSuccess || resident < 1) {
+    // No 8-CTA cluster of this kernel can be co-scheduled here (e.g. an MPS
+    // SM limit or a MIG slice): a valid team size this device cannot run.
     cudaGetLastError();
-    resident = 1;
+    set_error("%s: no cluster of %d CTAs x %d threads can be resident on this device", what,
+              kClusterCtas, cta);
+    return CUDANP_ERR_UNSUPPORTED;
   }
   int64_t clusters = N < (int64_t)resident * 8 ? N : (int64_t)resident * 8;
   if (clusters < 1) clusters = 1;

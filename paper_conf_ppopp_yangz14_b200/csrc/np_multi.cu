@@ -19,10 +19,6 @@ namespace cudanp {
 #endif
 constexpr int kMultiU = CUDANP_MULTI_U;  // units per thread batched before the fold (reduce, MV)
 
-// a - b with int32 wrapping modulo 2^32 (R13)
-__device__ __forceinline__ float tsub(float a, float b) { return a - b; }
-__device__ __forceinline__ int32_t tsub(int32_t a, int32_t b) { return (int32_t)((uint32_t)a - (uint32_t)b); }
-
 template <class T, class Op>
 __device__ __forceinline__ V4<T> mop4(V4<T> a, V4<T> b) {
   return {Op::apply(a.x, b.x), Op::apply(a.y, b.y), Op::apply(a.z, b.z), Op::apply(a.w, b.w)};
@@ -163,8 +159,7 @@ scan_multi_kernel(const T* __restrict__ in, const T* __restrict__ init, T* __res
         }
         const T tot = VEC ? v.w : v.x;
         T all;
-        const T incl = team.inclusive_scan(tot, sm, &all);
-        const T add = OpSum::apply(carry, tsub(incl, tot));  // carry + exclusive prefix
+        const T add = OpSum::apply(carry, team.exclusive_scan(tot, sm, &all));  // carry + exclusive prefix
         if (uok) {
           if constexpr (VEC)
             stg4(orow + 4 * u, V4<T>{OpSum::apply(v.x, add), OpSum::apply(v.y, add),
@@ -187,8 +182,7 @@ scan_multi_kernel(const T* __restrict__ in, const T* __restrict__ init, T* __res
         }
       }
       T all;
-      const T incl = team.inclusive_scan(csum, sm, &all);
-      T run = OpSum::apply(carry, tsub(incl, csum));
+      T run = OpSum::apply(carry, team.exclusive_scan(csum, sm, &all));
       if (ok) {
         for (int64_t u = r.begin; u < r.end; ++u) {
           if constexpr (VEC) {

@@ -249,6 +249,10 @@ template <class T, class Op, int S, int DIST, bool VEC>
 static int launch_reduce_map(const T* in, const T* init, T* out, int64_t N, int64_t L, int map,
                              cudaStream_t st, LaunchInfo* info) {
   if (map == MAP_INTRA) {
+   if constexpr (!kPow2<S>) {
+    set_error("intra-warp teams need S = 2^k <= 32 (P:342); S = %d is built for the inter-warp map", S);
+    return CUDANP_ERR_UNSUPPORTED;
+   } else {
     constexpr int TPW = 32 / S;
     const int64_t ntiles = (N + TPW - 1) / TPW;
     const bool few = few_tiles(reduce_intra_kernel<T, Op, S, DIST, VEC>, kReduceBlock, ntiles, kReduceK);
@@ -270,6 +274,7 @@ static int launch_reduce_map(const T* in, const T* init, T* out, int64_t N, int6
     }
     if (N == 0) return CUDANP_OK;
     launch_pdl(kern, dim3((unsigned)grid), dim3(kReduceBlock), 0, st, in, init, out, N, L);
+   }
   } else {
     auto kern = reduce_inter_kernel<T, Op, S, DIST, VEC>;
     const int64_t grid = persistent_grid(kern, 32 * S, 0, (N + 31) / 32);
@@ -290,15 +295,20 @@ static int dispatch_reduce_t(const void* in, const void* init, void* out, int64_
   const T* i = (const T*)in;
   const T* ini = (const T*)init;
   T* o = (T*)out;
-  CUDANP_DISPATCH_S(S, {
-    if (dist == DIST_CYCLIC) {
-      return vec ? launch_reduce_map<T, Op, kS, DIST_CYCLIC, true>(i, ini, o, N, L, map, st, info)
-                 : launch_reduce_map<T, Op, kS, DIST_CYCLIC, false>(i, ini, o, N, L, map, st, info);
-    } else {
-      return vec ? launch_reduce_map<T, Op, kS, DIST_BLOCK, true>(i, ini, o, N, L, map, st, info)
-                 : launch_reduce_map<T, Op, kS, DIST_BLOCK, false>(i, ini, o, N, L, map, st, info);
+#define CUDANP_REDUCE_BODY                                                                          \
+    if (dist == DIST_CYCLIC) {                                                                      \
+      return vec ? launch_reduce_map<T, Op, kS, DIST_CYCLIC, true>(i, ini, o, N, L, map, st, info)  \
+                 : launch_reduce_map<T, Op, kS, DIST_CYCLIC, false>(i, ini, o, N, L, map, st, info); \
+    } else {                                                                                        \
+      return vec ? launch_reduce_map<T, Op, kS, DIST_BLOCK, true>(i, ini, o, N, L, map, st, info)   \
+                 : launch_reduce_map<T, Op, kS, DIST_BLOCK, false>(i, ini, o, N, L, map, st, info);  \
     }
-  });
+  if (valid_inter_S(S)) {
+    CUDANP_DISPATCH_S_INTER(S, { CUDANP_REDUCE_BODY });
+  } else {
+    CUDANP_DISPATCH_S(S, { CUDANP_REDUCE_BODY });
+  }
+#undef CUDANP_REDUCE_BODY
   return CUDANP_OK;
 }
 

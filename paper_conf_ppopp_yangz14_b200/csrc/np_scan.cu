@@ -262,6 +262,10 @@ template <class T, int S, int DIST, bool VEC>
 static int launch_scan_map(const T* in, const T* init, T* out, int64_t N, int64_t L, int map,
                            cudaStream_t st, LaunchInfo* info) {
   if (map == MAP_INTRA) {
+   if constexpr (!kPow2<S>) {
+    set_error("intra-warp teams need S = 2^k <= 32 (P:342); S = %d is built for the inter-warp map", S);
+    return CUDANP_ERR_UNSUPPORTED;
+   } else {
     constexpr int TPW = 32 / S;
     const int64_t ntiles = (N + TPW - 1) / TPW;
     const bool few = few_tiles(scan_intra_kernel<T, S, DIST, VEC>, kScanBlock, ntiles, kScanK);
@@ -275,6 +279,7 @@ static int launch_scan_map(const T* in, const T* init, T* out, int64_t N, int64_
     }
     if (N == 0 || L == 0) return CUDANP_OK;
     launch_pdl(kern, dim3((unsigned)grid), dim3(kScanBlock), 0, st, in, init, out, N, L);
+   }
   } else {
     auto kern = scan_inter_kernel<T, S, DIST, VEC>;
     const int64_t grid = persistent_grid(kern, 32 * S, 0, (N + 31) / 32);
@@ -295,15 +300,20 @@ static int dispatch_scan_t(const void* in, const void* init, void* out, int64_t 
   const T* i = (const T*)in;
   const T* ini = (const T*)init;
   T* o = (T*)out;
-  CUDANP_DISPATCH_S(S, {
-    if (dist == DIST_CYCLIC) {
-      return vec ? launch_scan_map<T, kS, DIST_CYCLIC, true>(i, ini, o, N, L, map, st, info)
-                 : launch_scan_map<T, kS, DIST_CYCLIC, false>(i, ini, o, N, L, map, st, info);
-    } else {
-      return vec ? launch_scan_map<T, kS, DIST_BLOCK, true>(i, ini, o, N, L, map, st, info)
-                 : launch_scan_map<T, kS, DIST_BLOCK, false>(i, ini, o, N, L, map, st, info);
+#define CUDANP_SCAN_BODY                                                                        \
+    if (dist == DIST_CYCLIC) {                                                                  \
+      return vec ? launch_scan_map<T, kS, DIST_CYCLIC, true>(i, ini, o, N, L, map, st, info)    \
+                 : launch_scan_map<T, kS, DIST_CYCLIC, false>(i, ini, o, N, L, map, st, info);  \
+    } else {                                                                                    \
+      return vec ? launch_scan_map<T, kS, DIST_BLOCK, true>(i, ini, o, N, L, map, st, info)     \
+                 : launch_scan_map<T, kS, DIST_BLOCK, false>(i, ini, o, N, L, map, st, info);   \
     }
-  });
+  if (valid_inter_S(S)) {
+    CUDANP_DISPATCH_S_INTER(S, { CUDANP_SCAN_BODY });
+  } else {
+    CUDANP_DISPATCH_S(S, { CUDANP_SCAN_BODY });
+  }
+#undef CUDANP_SCAN_BODY
   return CUDANP_OK;
 }
 

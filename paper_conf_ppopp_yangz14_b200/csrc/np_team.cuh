@@ -318,15 +318,21 @@ struct MultiTeam {
     __syncthreads();
     return r;
   }
-  // Inclusive scan over the S team threads; *total = the team's sum.
+  // Exclusive scan over the S team threads (the sum of the lower slaves'
+  // values); *total = the team's sum.  Inside a warp the exclusive value is
+  // the previous lane's inclusive value (a shuffle), not incl - v, so fp32
+  // prefixes carry no cancellation error.
   template <class T>
-  __device__ __forceinline__ T inclusive_scan(T v, T* sm /*[teams*W]*/, T* total) const {
+  __device__ __forceinline__ T exclusive_scan(T v, T* sm /*[teams*W]*/, T* total) const {
+    T incl = v;
 #pragma unroll
     for (int o = 1; o < 32; o <<= 1) {
-      const T t = __shfl_up_sync(kFull, v, o);
-      if (lane >= o) v = OpSum::apply(v, t);
+      const T t = __shfl_up_sync(kFull, incl, o);
+      if (lane >= o) incl = OpSum::apply(incl, t);
     }
-    if (lane == 31) sm[team * W + wit] = v;
+    const T prev = __shfl_up_sync(kFull, incl, 1);
+    const T wexcl = lane == 0 ? T(0) : prev;
+    if (lane == 31) sm[team * W + wit] = incl;
     __syncthreads();
     T off = T(0), tot = T(0);
 #pragma unroll 4
@@ -337,7 +343,7 @@ struct MultiTeam {
     }
     __syncthreads();
     *total = tot;
-    return OpSum::apply(off, v);
+    return OpSum::apply(off, wexcl);
   }
   // read_from_master through a per-team shared slot.
   template <class T>

@@ -17,6 +17,9 @@
 //  block : S boxes of R/S rows per stage, one from each slave's contiguous
 //          chunk [s*c, (s+1)*c) (c = ceil(h/S)).
 // Rows past h come back zero-filled by TMA and are masked before x is read.
+// A block stage's box may run past the slave's chunk into the next slave's
+// rows (RK need not divide c); those rows are skipped (no FMA), so a
+// non-finite value there cannot leak into this slave's sum.
 #include <cuda.h>
 
 #include "common.cuh"
@@ -112,6 +115,9 @@ tmv_tma_kernel(const __grid_constant__ CUtensorMap mapA, const float* __restrict
       // x does not depend on the TMA: issue its loads before waiting on the
       // stage so their latency hides behind the tile's arrival.
       float xs[RK];
+      // block: is every row of this tile inside the slave's chunk and below h?
+      const bool whole = DIST == DIST_CYCLIC ||
+                         ((int64_t)(t + 1) * RK <= c && s * c + (int64_t)(t + 1) * RK <= h);
 #pragma unroll
       for (int kk = 0; kk < RK; ++kk) {
         int64_t row;
@@ -132,6 +138,10 @@ tmv_tma_kernel(const __grid_constant__ CUtensorMap mapA, const float* __restrict
       for (int kk = 0; kk < RK; ++kk) {
         const int lr = DIST == DIST_CYCLIC ? kk * S + s : s * RK + kk;
         const float xv = xs[kk];
+        if (DIST == DIST_BLOCK && !whole) {  // ragged last tile: skip rows outside the chunk
+          const int64_t k = (int64_t)t * RK + kk;
+          if (!(k < c && s * c + k < h)) continue;
+        }
         const float* ap = tile + lr * COLS + lane * V;
         if constexpr (V == 4) {
           const float4 a = *reinterpret_cast<const float4*>(ap);

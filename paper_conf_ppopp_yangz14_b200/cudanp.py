@@ -28,7 +28,9 @@ F32, I32 = 0, 1
 SUM, MAX = 0, 1
 S1_LITERAL, DP_THREAD, DP_BLOCK = 1, 2, 3
 GRAD_REGISTERS, GRAD_SHARED, GRAD_GLOBAL = 0, 1, 2   # LE: home of Grad (Fig 6c / 6b / 6a)
+S_AUTO = 0                                            # S argument: the library picks (S, dist, map)
 SLAVE_SIZES = (1, 2, 4, 8, 16, 32)                    # one warp (intra) or S warps (inter)
+INTER_ONLY_SIZES = (3, 5, 10, 15)                     # non-power-of-two: inter-warp map only
 MULTI_WARP_SIZES = (64, 128, 256, 512, 1024)          # S/32 warps of one CTA (reduce, scan, MV;
                                                       # TMV: 64, 128 inter-warp)
 CLUSTER_SIZES = (2048, 4096, 8192)                    # a cluster of 8 CTAs (reduce, scan, MV);
@@ -71,7 +73,10 @@ _SIGS = {
                         ctypes.POINTER(ctypes.c_float), ctypes.POINTER(_int), _vp],
     "cudanp_launch_info": [_int, _i64, _i64, _int, _int, _int, _int, _int, _int,
                            ctypes.POINTER(_int), ctypes.POINTER(_i64), ctypes.POINTER(_int),
-                           ctypes.POINTER(_int), ctypes.POINTER(_int)],
+                           ctypes.POINTER(_int), ctypes.POINTER(_int), ctypes.POINTER(_int),
+                           ctypes.POINTER(_int)],
+    "cudanp_choose_version": [_int, _i64, _i64, _int, _int, ctypes.POINTER(_int), ctypes.POINTER(_int),
+                              ctypes.POINTER(_int)],
     "cudanp_group_unique_id": [_vp],
     "cudanp_group_create": [_vp, _int, _int, ctypes.POINTER(_vp)],
     "cudanp_group_destroy": [_vp],
@@ -160,12 +165,87 @@ def _dtype_code(t) -> int:
     raise TypeError(f"unsupported dtype {t.dtype}: float32 or int32")
 
 
-# ---------------------------------------------------------------- hot-path calls
-def cudanp_tmv(A, x, y=None, *, S=32, dist=CYCLIC, map=AUTO, n_outer=None, stream=None):
-    """y[j] = sum_i A[i, j] * x[i] (Fig 2).  A: (h, lda) fp32 row-major."""
+# ---------------------------------------------------------------- argument checks
+# The C ABI takes raw pointers plus sizes and a leading dimension; these checks
+# make sure the tensors handed over really have that layout, dtype and length,
+# so a strided view or a short buffer raises here instead of being misread.
+def _mat(A, what: str):
+    """(rows, cols, lda) of a row-major fp32 CUDA matrix; lda = A.stride(0)."""
     import torch
-    h, lda = A.shape
-    w = lda if n_outer is None else n_outer
+    if not isinstance(A, torch.Tensor) or A.dim() != 2:
+        raise ValueError(f"{what}: A must be a 2-D tensor")
+    if A.dtype != torch.float32:
+        raise TypeError(f"{what}: A must be float32 (got {A.dtype})")
+    rows, cols = A.shape
+    if rows > 0 and cols > 1 and A.stride(1) != 1:
+        raise ValueError(f"{what}: A must have unit column stride (row-major; use A.contiguous())")
+    lda = A.stride(0) if rows > 1 else cols
+    if rows > 1 and cols > 0 and lda < cols:
+        raise ValueError(f"{what}: A rows overlap (stride(0) = {lda} < {cols} columns)")
+    return rows, cols, lda
+
+
+def _buf(t, n: int, dtype, what: str) -> None:
+    """t holds at least n contiguous elements of dtype (raw int pointers pass)."""
+    import torch
+    if t is None or isinstance(t, int):
+        return
+    if not isinstance(t, torch.Tensor):
+        raise TypeError(f"{what} must be a CUDA tensor")
+    if t.dtype != dtype:
+        raise TypeError(f"{what} must be {dtype} (got {t.dtype})")
+    if not t.is_contiguous():
+        raise ValueError(f"{what} must be contiguous")
+    if t.numel() < n:
+        raise ValueError(f"{what} holds {t.numel()} elements, needs {n}")
+
+
+def _items(x, what: str):
+    """(N, L) of an item-major [N][L] batch (contiguous, fp32 or int32)."""
+    import torch
+    if not isinstance(x, torch.Tensor) or x.dim() != 2:
+        raise ValueError(f"{what}: input must be a 2-D (N, L) tensor")
+    _dtype_code(x)
+    if not x.is_contiguous():
+        raise ValueError(f"{what}: input must be contiguous item-major (N, L) (use .contiguous())")
+    return x.shape
+
+
+# ---------------------------------------------------------------- hot-path calls
+def _tmv_args(A, x, y, n_outer, what):
+    import torch
+    h, cols, lda = _mat(A, what)
+    w = cols if n_outer is None else n_outer
+    if w > cols:
+        raise ValueError(f"{what}: n_outer {w} > A's {cols} columns")
+    _buf(x, h, torch.float32, f"{what}: x")
+    _buf(y, w, torch.float32, f"{what}: y")
+    return h, w, lda
+
+
+def _mv_args(A, x, y, n_inner, what):
+    import torch
+    h, cols, lda = _mat(A, what)
+    w = cols if n_inner is None else n_inner
+    if w > cols:
+        raise ValueError(f"{what}: n_inner {w} > A's {cols} columns")
+    _buf(x, w, torch.float32, f"{what}: x")
+    _buf(y, h, torch.float32, f"{what}: y")
+    return h, w, lda
+
+
+def _batched_args(x, init, out, per_item: bool, what):
+    N, L = _items(x, what)
+    _buf(init, N, x.dtype, f"{what}: init")
+    _buf(out, N if per_item else N * L, x.dtype, f"{what}: out")
+    return N, L
+
+
+def cudanp_tmv(A, x, y=None, *, S=S_AUTO, dist=CYCLIC, map=AUTO, n_outer=None, stream=None):
+    """y[j] = sum_i A[i, j] * x[i] (Fig 2).  A: (h, >= w) fp32, unit column
+    stride, lda = A.stride(0)."""
+    import torch
+    h, w, lda = _tmv_args(A, x, y, n_outer, "cudanp_tmv")
     if y is None:
         y = torch.empty(w, dtype=torch.float32, device=A.device)
     _check(load().cudanp_tmv(_ptr(A), lda, _ptr(x), _ptr(y), w, h, S, dist, map, _stream(stream)),
@@ -178,8 +258,7 @@ def cudanp_tmv_tma(A, x, y=None, *, S=8, dist=CYCLIC, n_outer=None, stream=None,
     """TMV with TMA-staged tiles (inter-warp map); same result contract as cudanp_tmv.
     cols / rows_sel / stages pin the launch shape (cudanp_tmv_tma_ex); defaults = auto."""
     import torch
-    h, lda = A.shape
-    w = lda if n_outer is None else n_outer
+    h, w, lda = _tmv_args(A, x, y, n_outer, "cudanp_tmv_tma")
     if y is None:
         y = torch.empty(w, dtype=torch.float32, device=A.device)
     if cols == 0 and rows_sel == -1 and stages == 0:
@@ -191,11 +270,11 @@ def cudanp_tmv_tma(A, x, y=None, *, S=8, dist=CYCLIC, n_outer=None, stream=None,
     return y
 
 
-def cudanp_mv(A, x, y=None, *, S=32, dist=CYCLIC, map=AUTO, n_inner=None, stream=None):
-    """y[i] = sum_j A[i, j] * x[j].  A: (h, lda) fp32 row-major."""
+def cudanp_mv(A, x, y=None, *, S=S_AUTO, dist=CYCLIC, map=AUTO, n_inner=None, stream=None):
+    """y[i] = sum_j A[i, j] * x[j].  A: (h, >= w) fp32, unit column stride,
+    lda = A.stride(0)."""
     import torch
-    h, lda = A.shape
-    w = lda if n_inner is None else n_inner
+    h, w, lda = _mv_args(A, x, y, n_inner, "cudanp_mv")
     if y is None:
         y = torch.empty(h, dtype=torch.float32, device=A.device)
     _check(load().cudanp_mv(_ptr(A), lda, _ptr(x), _ptr(y), h, w, S, dist, map, _stream(stream)),
@@ -203,11 +282,11 @@ def cudanp_mv(A, x, y=None, *, S=32, dist=CYCLIC, map=AUTO, n_inner=None, stream
     return y
 
 
-def cudanp_batched_loop_reduce(x, init=None, out=None, *, op=SUM, S=8, dist=CYCLIC, map=AUTO,
+def cudanp_batched_loop_reduce(x, init=None, out=None, *, op=SUM, S=S_AUTO, dist=CYCLIC, map=AUTO,
                                stream=None):
     """out[n] = init[n] (op) fold_i x[n, i].  x: (N, L) fp32/int32."""
     import torch
-    N, L = x.shape
+    N, L = _batched_args(x, init, out, True, "cudanp_batched_loop_reduce")
     if out is None:
         out = torch.empty(N, dtype=x.dtype, device=x.device)
     _check(load().cudanp_batched_loop_reduce(_ptr(x), _ptr(init), _ptr(out), N, L, _dtype_code(x),
@@ -224,7 +303,7 @@ def cudanp_batched_loop_reduce_backend(x, init=None, out=None, *, op=SUM, S=8, b
     """Fig 16 ablation: intra-warp cyclic reduce with the team reduction done by
     shfl (0), shared memory (1) or redux.sync (2)."""
     import torch
-    N, L = x.shape
+    N, L = _batched_args(x, init, out, True, "cudanp_batched_loop_reduce_backend")
     if out is None:
         out = torch.empty(N, dtype=x.dtype, device=x.device)
     _check(load().cudanp_batched_loop_reduce_backend(_ptr(x), _ptr(init), _ptr(out), N, L,
@@ -238,7 +317,7 @@ def cudanp_batched_loop_reduce_tma(x, init=None, out=None, *, op=SUM, S=8, dist=
                                    stage_bytes=0, stages=0, stream=None):
     """cudanp_batched_loop_reduce with the rows staged by TMA bulk copies (same result)."""
     import torch
-    N, L = x.shape
+    N, L = _batched_args(x, init, out, True, "cudanp_batched_loop_reduce_tma")
     if out is None:
         out = torch.empty(N, dtype=x.dtype, device=x.device)
     _check(load().cudanp_batched_loop_reduce_tma(_ptr(x), _ptr(init), _ptr(out), N, L, _dtype_code(x),
@@ -247,10 +326,10 @@ def cudanp_batched_loop_reduce_tma(x, init=None, out=None, *, op=SUM, S=8, dist=
     return out
 
 
-def cudanp_batched_loop_scan(x, init=None, out=None, *, S=8, dist=CYCLIC, map=AUTO, stream=None):
+def cudanp_batched_loop_scan(x, init=None, out=None, *, S=S_AUTO, dist=CYCLIC, map=AUTO, stream=None):
     """Inclusive scan out[n, k] = init[n] + sum_{i<=k} x[n, i]."""
     import torch
-    N, L = x.shape
+    N, L = _batched_args(x, init, out, False, "cudanp_batched_loop_scan")
     if out is None:
         out = torch.empty_like(x)
     _check(load().cudanp_batched_loop_scan(_ptr(x), _ptr(init), _ptr(out), N, L, _dtype_code(x),
@@ -259,14 +338,30 @@ def cudanp_batched_loop_scan(x, init=None, out=None, *, S=8, dist=CYCLIC, map=AU
     return out
 
 
+def _ragged_args(x, offsets, init, out, what):
+    """N of a CSR batch.  The offsets' values (0 <= off[n] <= off[n+1] <=
+    x.numel()) live on the device and are the caller's contract."""
+    import torch
+    if not isinstance(x, torch.Tensor) or x.dim() != 1 or not x.is_contiguous():
+        raise ValueError(f"{what}: values must be a contiguous 1-D tensor")
+    _dtype_code(x)
+    if not isinstance(offsets, torch.Tensor) or offsets.dim() != 1 or offsets.shape[0] < 1:
+        raise ValueError(f"{what}: offsets must be a 1-D tensor of N+1 entries")
+    if offsets.dtype != torch.int64:
+        raise TypeError("offsets must be int64")
+    _buf(offsets, offsets.shape[0], torch.int64, f"{what}: offsets")
+    N = offsets.shape[0] - 1
+    _buf(init, N, x.dtype, f"{what}: init")
+    _buf(out, N, x.dtype, f"{what}: out")
+    return N
+
+
 def cudanp_ragged_loop_reduce(x, offsets, init=None, out=None, *, op=SUM, S=8, dist=CYCLIC,
                               map=AUTO, stream=None):
     """out[n] = init[n] (op) fold_{offsets[n] <= i < offsets[n+1]} x[i] (P:193).
     x: 1-D fp32/int32; offsets: 1-D int64 of N+1 entries."""
     import torch
-    if offsets.dtype != torch.int64:
-        raise TypeError("offsets must be int64")
-    N = offsets.shape[0] - 1
+    N = _ragged_args(x, offsets, init, out, "cudanp_ragged_loop_reduce")
     if out is None:
         out = torch.empty(N, dtype=x.dtype, device=x.device)
     _check(load().cudanp_ragged_loop_reduce(_ptr(x), _ptr(offsets), _ptr(init), _ptr(out), N,
@@ -280,7 +375,7 @@ def cudanp_ragged_loop_reduce_adaptive(x, offsets, init=None, out=None, *, op=SU
     """Ragged reduce with the team size chosen per segment (S = 1 below
     `threshold` elements, a warp-wide team of 32 above)."""
     import torch
-    N = offsets.shape[0] - 1
+    N = _ragged_args(x, offsets, init, out, "cudanp_ragged_loop_reduce_adaptive")
     if out is None:
         out = torch.empty(N, dtype=x.dtype, device=x.device)
     _check(load().cudanp_ragged_loop_reduce_adaptive(_ptr(x), _ptr(offsets), _ptr(init), _ptr(out), N,
@@ -291,7 +386,7 @@ def cudanp_ragged_loop_reduce_adaptive(x, offsets, init=None, out=None, *, op=SU
 
 def cudanp_ragged_loop_reduce_literal(x, offsets, init=None, out=None, *, op=SUM, stream=None):
     import torch
-    N = offsets.shape[0] - 1
+    N = _ragged_args(x, offsets, init, out, "cudanp_ragged_loop_reduce_literal")
     if out is None:
         out = torch.empty(N, dtype=x.dtype, device=x.device)
     _check(load().cudanp_ragged_loop_reduce_literal(_ptr(x), _ptr(offsets), _ptr(init), _ptr(out),
@@ -306,7 +401,10 @@ def cudanp_le_gicov(x, threshold, gicov=None, *, layout=0, S=8, dist=CYCLIC, map
     x: (N, L) when layout == 0, (L, N) when layout == 1.  gicov entries whose
     test fails are left as given (default: filled with -1)."""
     import torch
+    if not isinstance(x, torch.Tensor) or x.dim() != 2 or x.dtype != torch.float32 or not x.is_contiguous():
+        raise ValueError("cudanp_le_gicov: x must be a contiguous 2-D float32 tensor")
     N, L = (x.shape if layout == 0 else x.shape[::-1])
+    _buf(gicov, N, torch.float32, "cudanp_le_gicov: gicov")
     if gicov is None:
         gicov = torch.full((N,), -1.0, dtype=torch.float32, device=x.device)
     stats = [torch.empty(N, dtype=torch.float32, device=x.device) for _ in range(3)] \
@@ -328,8 +426,7 @@ def cudanp_le_gicov(x, threshold, gicov=None, *, layout=0, S=8, dist=CYCLIC, map
 # ---------------------------------------------------------------- comparison kernels
 def cudanp_tmv_variant(impl, A, x, y=None, *, n_outer=None, stream=None):
     import torch
-    h, lda = A.shape
-    w = lda if n_outer is None else n_outer
+    h, w, lda = _tmv_args(A, x, y, n_outer, "cudanp_tmv_variant")
     if y is None:
         y = torch.empty(w, dtype=torch.float32, device=A.device)
     _check(load().cudanp_tmv_variant(impl, _ptr(A), lda, _ptr(x), _ptr(y), w, h, _stream(stream)),
@@ -339,8 +436,7 @@ def cudanp_tmv_variant(impl, A, x, y=None, *, n_outer=None, stream=None):
 
 def cudanp_mv_variant(impl, A, x, y=None, *, n_inner=None, stream=None):
     import torch
-    h, lda = A.shape
-    w = lda if n_inner is None else n_inner
+    h, w, lda = _mv_args(A, x, y, n_inner, "cudanp_mv_variant")
     if y is None:
         y = torch.empty(h, dtype=torch.float32, device=A.device)
     _check(load().cudanp_mv_variant(impl, _ptr(A), lda, _ptr(x), _ptr(y), h, w, _stream(stream)),
@@ -350,7 +446,7 @@ def cudanp_mv_variant(impl, A, x, y=None, *, n_inner=None, stream=None):
 
 def cudanp_batched_loop_reduce_variant(impl, x, init=None, out=None, *, op=SUM, stream=None):
     import torch
-    N, L = x.shape
+    N, L = _batched_args(x, init, out, True, "cudanp_batched_loop_reduce_variant")
     if out is None:
         out = torch.empty(N, dtype=x.dtype, device=x.device)
     _check(load().cudanp_batched_loop_reduce_variant(impl, _ptr(x), _ptr(init), _ptr(out), N, L,
@@ -360,7 +456,7 @@ def cudanp_batched_loop_reduce_variant(impl, x, init=None, out=None, *, op=SUM, 
 
 
 def cudanp_batched_loop_scan_variant(impl, x, init=None, out=None, *, stream=None):
-    N, L = x.shape
+    N, L = _batched_args(x, init, out, False, "cudanp_batched_loop_scan_variant")
     if out is None:
         import torch
         out = torch.empty_like(x)
@@ -423,12 +519,27 @@ def cudanp_autotune(op_kind: str, a, b, out, *, lda=0, n_outer, n_inner, dtype=F
 def cudanp_launch_info(op_kind: str, n_outer: int, n_inner: int, *, dtype=F32, op=SUM, S=8,
                        dist=CYCLIC, map=AUTO, vec4=True) -> dict:
     kinds = {"tmv": 0, "mv": 1, "reduce": 2, "scan": 3, "tmv_tma": 4, "reduce_tma": 5}
-    b, g, r, s, m = _int(), _i64(), _int(), _int(), _int()
+    b, g, r, s, m, su, du = _int(), _i64(), _int(), _int(), _int(), _int(), _int()
     _check(load().cudanp_launch_info(kinds[op_kind], n_outer, n_inner, dtype, op, S, dist, map,
                                      int(vec4), ctypes.byref(b), ctypes.byref(g), ctypes.byref(r),
-                                     ctypes.byref(s), ctypes.byref(m)), "cudanp_launch_info")
+                                     ctypes.byref(s), ctypes.byref(m), ctypes.byref(su),
+                                     ctypes.byref(du)), "cudanp_launch_info")
     return {"block_threads": b.value, "grid_ctas": g.value, "regs_per_thread": r.value,
-            "smem_bytes": s.value, "map": {1: "intra_warp", 2: "inter_warp", 3: "inter_warp_tma", 4: "intra_warp_tma"}.get(m.value, "?")}
+            "smem_bytes": s.value, "map": MAP_NAMES.get(m.value, "?"), "S": su.value,
+            "dist": "cyclic" if du.value == CYCLIC else "block"}
+
+
+MAP_NAMES = {1: "intra_warp", 2: "inter_warp", 3: "inter_warp_tma", 4: "intra_warp_tma"}
+
+
+def cudanp_choose_version(op_kind: str, n_outer: int, n_inner: int, *, vec4=True,
+                          map=AUTO) -> tuple[int, int, int]:
+    """(S, dist, map) the library runs for S = S_AUTO on this shape (host-only rule)."""
+    S, d, m = _int(), _int(), _int()
+    _check(load().cudanp_choose_version(OP_KINDS[op_kind], n_outer, n_inner, int(vec4), map,
+                                        ctypes.byref(S), ctypes.byref(d), ctypes.byref(m)),
+           "cudanp_choose_version")
+    return S.value, d.value, m.value
 
 
 def cudanp_ipc_get_handle(t) -> tuple[bytes, int]:
@@ -476,7 +587,12 @@ def cudanp_group_gather(group: int, local, root_buf, n_total: int, stream=None) 
 
 def cudanp_sharded_tmv(group: int, A_shard, x, y_shard, y_root, n_outer_total: int, *, S=32,
                        dist=CYCLIC, map=AUTO, stream=None) -> None:
-    h, lda = A_shard.shape
+    import torch
+    h, w, lda = _mat(A_shard, "cudanp_sharded_tmv")
+    _buf(x, h, torch.float32, "cudanp_sharded_tmv: x")
+    _buf(y_shard, w, torch.float32, "cudanp_sharded_tmv: y_shard")
+    _buf(y_root, n_outer_total if y_root is not None and not isinstance(y_root, int) else 0,
+         torch.float32, "cudanp_sharded_tmv: y_root")
     _check(load().cudanp_sharded_tmv(group, _ptr(A_shard), lda, _ptr(x), _ptr(y_shard), _ptr(y_root),
                                      n_outer_total, h, S, dist, map, _stream(stream)),
            "cudanp_sharded_tmv")
@@ -485,7 +601,9 @@ def cudanp_sharded_tmv(group: int, A_shard, x, y_shard, y_root, n_outer_total: i
 def cudanp_sharded_batched_loop_reduce(group: int, in_shard, init_shard, out_shard, out_root,
                                        n_outer_total: int, *, op=SUM, S=8, dist=CYCLIC, map=AUTO,
                                        stream=None) -> None:
-    L = in_shard.shape[1]
+    N, L = _items(in_shard, "cudanp_sharded_batched_loop_reduce")
+    _buf(init_shard, N, in_shard.dtype, "cudanp_sharded_batched_loop_reduce: init")
+    _buf(out_shard, N, in_shard.dtype, "cudanp_sharded_batched_loop_reduce: out_shard")
     _check(load().cudanp_sharded_batched_loop_reduce(group, _ptr(in_shard), _ptr(init_shard),
                                                      _ptr(out_shard), _ptr(out_root), n_outer_total, L,
                                                      _dtype_code(in_shard), op, S, dist, map,
