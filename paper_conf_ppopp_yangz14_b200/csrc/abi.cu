@@ -45,6 +45,8 @@ int le_np(const float*, float*, float*, float*, float*, int64_t, int64_t, float,
           bool, cudaStream_t);
 int le_tma(const float*, float*, float*, float*, float*, int64_t, int64_t, float, int, int,
            cudaStream_t);
+int mv_s1_tiled(const float*, int64_t, const float*, float*, int64_t, int64_t, cudaStream_t);
+int scan_s1_tiled(const void*, const void*, void*, int64_t, int64_t, int, cudaStream_t);
 int le_literal(const float*, float*, float*, float*, float*, int64_t, int64_t, float, int,
                cudaStream_t);
 
@@ -597,9 +599,19 @@ int cudanp_le_gicov_literal(const float* in, float* gicov, float* ave, float* va
 
 // ---------------------------------------------------------------- variants
 static int check_impl(int impl) {
-  if (impl != CUDANP_IMPL_S1_LITERAL && impl != CUDANP_IMPL_DP_THREAD && impl != CUDANP_IMPL_DP_BLOCK)
+  if (impl != CUDANP_IMPL_S1_LITERAL && impl != CUDANP_IMPL_DP_THREAD && impl != CUDANP_IMPL_DP_BLOCK &&
+      impl != CUDANP_IMPL_S1_TILED)
     return fail_invalid("impl");
   return CUDANP_OK;
+}
+static int tiled_unsupported() {
+  set_error("the TMA-tiled S=1 baseline needs 16-byte aligned operands, rows a multiple of 4 "
+            "elements and sizes < 2^31");
+  return CUDANP_ERR_UNSUPPORTED;
+}
+static bool tiled_ok(const void* a, int64_t ld, const void* b, int64_t rows, int64_t cols) {
+  return aligned16(a) && (!b || aligned16(b)) && ld % 4 == 0 && rows < (int64_t(1) << 31) &&
+         cols < (int64_t(1) << 31);
 }
 
 int cudanp_tmv_variant(int impl, const float* A, int64_t lda, const float* x, float* y,
@@ -608,6 +620,12 @@ int cudanp_tmv_variant(int impl, const float* A, int64_t lda, const float* x, fl
   if (!rc) rc = check_tmv_args(A, lda, x, y, n_outer, n_inner, 1, 0, 0);
   if (rc) return rc;
   if (impl == CUDANP_IMPL_S1_LITERAL) return tmv_literal(A, lda, x, y, n_outer, n_inner, as_stream(stream));
+  if (impl == CUDANP_IMPL_S1_TILED) {
+    if (n_outer == 0) return CUDANP_OK;
+    if (n_inner == 0) return tmv_np(A, lda, x, y, n_outer, 0, 1, 0, MAP_INTER, false, as_stream(stream), nullptr);
+    if (!tma_ok(A, lda, n_outer, n_inner)) return tiled_unsupported();
+    return tmv_tma(A, lda, x, y, n_outer, n_inner, 1, 0, 0, -1, 0, as_stream(stream), nullptr);
+  }
   return dp_tmv(impl == CUDANP_IMPL_DP_BLOCK, A, lda, x, y, n_outer, n_inner, as_stream(stream));
 }
 
@@ -617,6 +635,10 @@ int cudanp_mv_variant(int impl, const float* A, int64_t lda, const float* x, flo
   if (!rc) rc = check_mv_args(A, lda, x, y, n_outer, n_inner, 1, 0, 0);
   if (rc) return rc;
   if (impl == CUDANP_IMPL_S1_LITERAL) return mv_literal(A, lda, x, y, n_outer, n_inner, as_stream(stream));
+  if (impl == CUDANP_IMPL_S1_TILED) {
+    if (n_outer > 0 && n_inner > 0 && !tiled_ok(A, lda, nullptr, n_outer, n_inner)) return tiled_unsupported();
+    return mv_s1_tiled(A, lda, x, y, n_outer, n_inner, as_stream(stream));
+  }
   return dp_mv(impl == CUDANP_IMPL_DP_BLOCK, A, lda, x, y, n_outer, n_inner, as_stream(stream));
 }
 
@@ -628,6 +650,8 @@ int cudanp_batched_loop_reduce_variant(int impl, const void* in, const void* ini
   if (rc) return rc;
   if (impl == CUDANP_IMPL_S1_LITERAL)
     return reduce_literal(in, init, out, n_outer, n_inner, dtype, op, as_stream(stream));
+  if (impl == CUDANP_IMPL_S1_TILED)
+    return cudanp_batched_loop_reduce_tma(in, init, out, n_outer, n_inner, dtype, op, 1, 0, 0, 0, stream);
   return dp_reduce(impl == CUDANP_IMPL_DP_BLOCK, in, init, out, n_outer, n_inner, dtype, op,
                    as_stream(stream));
 }
@@ -639,6 +663,10 @@ int cudanp_batched_loop_scan_variant(int impl, const void* in, const void* init,
   if (rc) return rc;
   if (impl == CUDANP_IMPL_S1_LITERAL)
     return scan_literal(in, init, out, n_outer, n_inner, dtype, as_stream(stream));
+  if (impl == CUDANP_IMPL_S1_TILED) {
+    if (n_outer > 0 && n_inner > 0 && !tiled_ok(in, n_inner, out, n_outer, n_inner)) return tiled_unsupported();
+    return scan_s1_tiled(in, init, out, n_outer, n_inner, dtype, as_stream(stream));
+  }
   return dp_scan(impl == CUDANP_IMPL_DP_BLOCK, in, init, out, n_outer, n_inner, dtype,
                  as_stream(stream));
 }

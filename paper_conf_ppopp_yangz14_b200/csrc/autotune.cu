@@ -25,6 +25,8 @@ static std::vector<Candidate> candidates(int op_kind) {
   for (int S : small)
     for (int d = 0; d < 2; ++d)
       for (int m = CUDANP_MAP_INTRA_WARP; m <= CUDANP_MAP_INTER_WARP; ++m) c.push_back({S, d, m});
+  for (int S : {3, 5, 10, 15})  // non-power-of-two inter-warp teams (Fig 12)
+    for (int d = 0; d < 2; ++d) c.push_back({S, d, CUDANP_MAP_INTER_WARP});
   if (op_kind == 0) {  // TMV: TMA-staged inter-warp, and inter-warp teams up to 128
     for (int S : small)
       for (int d = 0; d < 2; ++d) c.push_back({S, d, CUDANP_MAP_INTER_WARP_TMA});

@@ -26,7 +26,7 @@ CYCLIC, BLOCK = 0, 1
 AUTO, INTRA_WARP, INTER_WARP, INTER_WARP_TMA, INTRA_WARP_TMA = 0, 1, 2, 3, 4
 F32, I32 = 0, 1
 SUM, MAX = 0, 1
-S1_LITERAL, DP_THREAD, DP_BLOCK = 1, 2, 3
+S1_LITERAL, DP_THREAD, DP_BLOCK, S1_TILED = 1, 2, 3, 4
 GRAD_REGISTERS, GRAD_SHARED, GRAD_GLOBAL = 0, 1, 2   # LE: home of Grad (Fig 6c / 6b / 6a)
 S_AUTO = 0                                            # S argument: the library picks (S, dist, map)
 SLAVE_SIZES = (1, 2, 4, 8, 16, 32)                    # one warp (intra) or S warps (inter)

@@ -108,9 +108,9 @@ int main(void) {
         if (hout[n] != L - 1) { fprintf(stderr, "max S=%d n=%ld: %d\n", S, (long)n, hout[n]); ++fails; break; }
     }
   }
-  /* validation before launch: S = 3 intra-warp is not a team size */
-  if (cudanp_batched_loop_reduce(in, NULL, out, N, L, CUDANP_I32, CUDANP_SUM, 3, 0, 0, st) != CUDANP_ERR_INVALID) {
-    fprintf(stderr, "S=3 was not rejected\n");
+  /* validation before launch: S = 6 is not a team size (3, 5, 10, 15 are, inter-warp) */
+  if (cudanp_batched_loop_reduce(in, NULL, out, N, L, CUDANP_I32, CUDANP_SUM, 6, 0, 0, st) != CUDANP_ERR_INVALID) {
+    fprintf(stderr, "S=6 was not rejected\n");
     ++fails;
   }
   CK(cudaStreamSynchronize(st));

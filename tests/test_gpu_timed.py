@@ -393,3 +393,64 @@ def test_binding_passes_row_stride_as_lda():
     for S, m in ((1, C.AUTO), (8, C.INTER_WARP), (8, C.INTRA_WARP), (C.S_AUTO, C.AUTO)):
         assert_exact(host(C.cudanp_tmv(Ad, dev(xt), S=S, map=m)), O.tmv(full, xt, w), f"tmv view S={S}")
         assert_exact(host(C.cudanp_mv(Ad, dev(xm), S=S, map=m)), O.mv(full, xm, w), f"mv view S={S}")
+
+
+# ------------------------------------------------------------------ tiled S = 1 baselines
+def test_s1_tiled_baselines_parity():
+    """CUDANP_IMPL_S1_TILED: one thread per item, rows through TMA-staged
+    shared-memory tiles (the SMM-style no-NP baseline) -- the
+    denominator of the NP speedups must compute the same thing.  Ragged row
+    groups (h, N not multiples of the 64/128-row tiles), widths not multiples
+    of the 32-column tile, multi-tile rows, init."""
+    for h, w in ((1, 4), (37, 132), (300, 260), (129, 512), (1000, 1004), (4100, 68)):
+        A = synth.matrix(h, w, "f32_int4", seed=w)
+        xt, xm = synth.vector(h, "f32_int4"), synth.vector(w, "f32_int4")
+        assert_exact(host(C.cudanp_mv_variant(C.S1_TILED, dev(A), dev(xm))), O.mv(A, xm), f"mv tiled {h}x{w}")
+        assert_exact(host(C.cudanp_tmv_variant(C.S1_TILED, dev(A), dev(xt))), O.tmv(A, xt), f"tmv tiled {h}x{w}")
+    Au, xu = synth.matrix(513, 2048, "f32_unit"), synth.vector(2048, "f32_unit")
+    assert_rel(host(C.cudanp_mv_variant(C.S1_TILED, dev(Au), dev(xu))), O.mv(Au, xu), 2048, "mv tiled unit")
+    # a padded row pitch (lda > w) through the binding's stride
+    full = synth.matrix(200, 132, "f32_int4")
+    xm = synth.vector(100, "f32_int4")
+    assert_exact(host(C.cudanp_mv_variant(C.S1_TILED, dev(full)[:, :100], dev(xm))), O.mv(full, xm, 100),
+                 "mv tiled lda")
+    for N, L in ((1, 4), (33, 8), (129, 64), (1000, 100), (300, 1024), (5000, 36)):
+        for kind, exact in (("i32_small", True), ("f32_int4", True), ("f32_unit", False)):
+            x = synth.items(N, L, kind, B=1 << 15, seed=L)
+            ini = synth.init(N, kind, B=1 << 15, seed=L)
+            got = host(C.cudanp_batched_loop_scan_variant(C.S1_TILED, dev(x), dev(ini)))
+            ref = O.scan(x, init=ini)
+            what = f"scan tiled {kind} {N}x{L}"
+            assert_exact(got, ref, what) if exact else assert_rel(got, ref, L, what)
+            got = host(C.cudanp_batched_loop_scan_variant(C.S1_TILED, dev(x)))
+            assert_exact(got, O.scan(x), what) if exact else assert_rel(got, O.scan(x), L, what)
+        x = synth.items(N, L, "i32_full")
+        assert_exact(host(C.cudanp_batched_loop_reduce_variant(C.S1_TILED, dev(x))), O.reduce(x), f"reduce tiled {N}x{L}")
+    # preconditions: rows not a multiple of 4 elements -> unsupported, not wrong
+    with pytest.raises(C.CudanpError) as ei:
+        C.cudanp_batched_loop_scan_variant(C.S1_TILED, dev(synth.items(10, 7, "i32_small")))
+    assert ei.value.status == C.ERR_UNSUPPORTED
+
+
+def test_s1_tiled_full_size_C2_C4_sampled():
+    """The tiled S = 1 kernels at the sizes the bench / sweep time them."""
+    n = 16384
+    A = torch.empty(n, n, dtype=torch.float32, device="cuda")
+    C.cudanp_generate(A, "f32_unit", stream_id=1)
+    x = torch.empty(n, dtype=torch.float32, device="cuda")
+    C.cudanp_generate(x, "f32_unit", stream_id=2)
+    idx = _sample_idx(n, 11)
+    assert_rel(host(C.cudanp_mv_variant(C.S1_TILED, A, x))[idx], O.mv_gen(n, n, idx), n, "C2 mv tiled")
+    assert_rel(host(C.cudanp_tmv_variant(C.S1_TILED, A, x))[idx], O.tmv_gen(n, n, idx), n, "C2 tmv tiled")
+    del A
+    torch.cuda.empty_cache()
+    N = 1 << 21
+    items = _sample_idx(N, 12, 256)
+    sel = torch.from_numpy(items).cuda()
+    for L in (64, 1024):
+        xi = torch.empty(N, L, dtype=torch.int32, device="cuda")
+        C.cudanp_generate(xi, "i32_small", stream_id=1, B=1 << 15)
+        out = C.cudanp_batched_loop_scan_variant(C.S1_TILED, xi)
+        assert_exact(host(out[sel]), O.scan_gen(L, items, O.I32, "i32_small", B=1 << 15), f"C4 tiled L={L}")
+        del xi, out
+        torch.cuda.empty_cache()
