@@ -696,12 +696,20 @@ def test_cluster_teams_parity():
 
 def test_launch_info_and_auto_map():
     """cudanp_launch_info reports the instantiation a call would launch; MAP_AUTO
-    resolves per P:340-342 (TMV -> inter-warp, MV/reduce/scan -> intra-warp)."""
-    for op, auto in (("tmv", "inter_warp"), ("mv", "intra_warp"), ("reduce", "intra_warp"),
+    resolves per P:340-342 (TMV -> inter-warp, MV/reduce/scan -> intra-warp),
+    TMV taking the TMA-staged inter-warp kernel on wide 16-byte aligned
+    matrices and the LDG one on narrow or unaligned ones."""
+    for op, auto in (("tmv", "inter_warp_tma"), ("mv", "intra_warp"), ("reduce", "intra_warp"),
                      ("scan", "intra_warp")):
         for S in SS:
             i = C.cudanp_launch_info(op, 1 << 14, 1 << 10, dtype=C.F32 if op != "scan" else C.I32, S=S)
             assert i["map"] == auto, (op, S, i)
+    for S in SS:
+        assert C.cudanp_launch_info("tmv", 1 << 10, 1 << 10, S=S)["map"] == "inter_warp"
+        assert C.cudanp_launch_info("tmv", 1 << 14, 1 << 10, S=S, vec4=False)["map"] == "inter_warp"
+    for op in ("tmv", "mv", "reduce", "scan"):
+        for S in SS:
+            i = C.cudanp_launch_info(op, 1 << 14, 1 << 10, dtype=C.F32 if op != "scan" else C.I32, S=S)
             assert i["block_threads"] > 0 and i["grid_ctas"] > 0 and i["regs_per_thread"] > 0
             assert i["block_threads"] <= 1024
         for m in (C.INTRA_WARP, C.INTER_WARP):
