@@ -20,6 +20,12 @@ ranges); its outputs are gathered to rank 0 with NCCL.
 Metric value = algorithmic HBM bytes of all ranks / max-over-ranks step time
 (GB/s).  Inputs (1 GiB per matrix) exceed the 126 MB L2, so no flush is
 needed between steps.
+
+The same line carries a `c5` block: BASELINE configs[4] (TMV 65536^2 by column
+shards + the 64M x 64 loop-reduce by item shards, strong scaling over the N
+ranks, outputs gathered to rank 0), with max-over-ranks kernel and gather
+times, aggregate GB/s, the fraction of N x peak and a bit-exact check of the
+sharded result against the unsharded one (pin P4).  `--no-c5` skips it.
 """
 from __future__ import annotations
 
@@ -40,7 +46,7 @@ sys.path.insert(0, ROOT)
 METRIC = "HBM GB/s and speedup vs S=1 no-NP kernel per slave count, at 1/2/4/8 B200"
 H = W = 16384
 SEED = 20140215
-MAPN = {1: "intra", 2: "inter", 3: "inter_tma"}   # cudanp_map
+MAPN = {1: "intra", 2: "inter", 3: "inter_tma", 4: "intra_tma"}   # cudanp_map
 
 
 def parse():
@@ -60,8 +66,12 @@ def parse():
                          "torch.distributed, fused into the kernels' master stores through CUDA IPC "
                          "over NVLink (SURVEY f4), or with the library's own NCCL group "
                          "(cudanp_group_gather)")
-    ap.add_argument("--tmv-cfg", default="32,block,inter")
-    ap.add_argument("--mv-cfg", default="16,cyclic,intra")
+    ap.add_argument("--tmv-cfg", default="8,cyclic,inter_tma")
+    ap.add_argument("--mv-cfg", default="256,cyclic,intra")
+    ap.add_argument("--no-c5", action="store_true", help="skip the C5 strong-scaling block")
+    ap.add_argument("--c5-steps", type=int, default=10)
+    ap.add_argument("--cpu-rows", type=int, default=1024,
+                    help="rows of the C2 matrix in the oracle's CPU sample (both arms)")
     return ap.parse_args()
 
 
@@ -149,6 +159,10 @@ def dist_init(ngpus):
     backend = os.environ.get("CUDANP_BENCH_BACKEND", "nccl")
     dev = local % max(torch.cuda.device_count(), 1)
     torch.cuda.set_device(dev)
+    if world > 1 and backend == "nccl":
+        # NCCL's communicator log (the init lines name nranks and the transport)
+        os.environ.setdefault("NCCL_DEBUG", "INFO")
+        os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
     if world > 1:
         if backend == "nccl":
             dist.init_process_group("nccl", device_id=torch.device("cuda", dev))
@@ -242,7 +256,8 @@ def run_cudanp(args):
         def parse_cfg(s):
             S, d, m = s.split(",")
             return (int(S), {"cyclic": C.CYCLIC, "block": C.BLOCK}[d],
-                    {"intra": C.INTRA_WARP, "inter": C.INTER_WARP, "inter_tma": C.INTER_WARP_TMA}[m])
+                    {"intra": C.INTRA_WARP, "inter": C.INTER_WARP, "inter_tma": C.INTER_WARP_TMA,
+                     "auto": C.AUTO}[m])
         sweep["tmv"][parse_cfg(args.tmv_cfg)] = 1.0
         sweep["mv"][parse_cfg(args.mv_cfg)] = 1.0
     else:
@@ -255,6 +270,7 @@ def run_cudanp(args):
                 if ms < 1e29:  # not supported for this shape
                     sweep[op][cand] = ms
     best = {op: min(sweep[op], key=sweep[op].get) for op in sweep}
+    best_ms = {op: sweep[op][best[op]] for op in sweep}
     if not args.no_sweep:
         # refine: the three fastest versions of each op re-timed with 30 launches
         # each (the 5-launch sweep is noisy at the 1-2 % level), max over ranks
@@ -265,18 +281,28 @@ def run_cudanp(args):
             ref = [max_over_ranks(time_op(lambda c=c: fn(A_, x_, y_, S=c[0], dist=c[1], map=c[2], **kw),
                                           reps=30, warm=3), world) for c in top]
             best[op] = top[min(range(len(top)), key=ref.__getitem__)]
+            best_ms[op] = min(ref)
     # literal S=1 (Fig 2) and DP (per-CTA / per-thread) comparison, once each
     comp = {}
     C.cudanp_dp_set_pending_launch_limit(1 << 16)
     for op, fn in () if args.no_sweep else (("tmv_s1_literal", lambda: C.cudanp_tmv_variant(C.S1_LITERAL, A_t, x_t, y_t)),
                    ("mv_s1_literal", lambda: C.cudanp_mv_variant(C.S1_LITERAL, A_m, x_m, y_m)),
-                   ("tmv_s1_tma", lambda: C.cudanp_tmv_tma(A_t, x_t, y_t, S=1)),
+                   ("tmv_s1_tiled", lambda: C.cudanp_tmv_variant(C.S1_TILED, A_t, x_t, y_t)),
+                   ("mv_s1_tiled", lambda: C.cudanp_mv_variant(C.S1_TILED, A_m, x_m, y_m)),
                    ("tmv_dp_block", lambda: C.cudanp_tmv_variant(C.DP_BLOCK, A_t, x_t, y_t)),
                    ("mv_dp_block", lambda: C.cudanp_mv_variant(C.DP_BLOCK, A_m, x_m, y_m)),
                    ("tmv_dp_thread", lambda: C.cudanp_tmv_variant(C.DP_THREAD, A_t, x_t, y_t)),
                    ("mv_dp_thread", lambda: C.cudanp_mv_variant(C.DP_THREAD, A_m, x_m, y_m))):
-        comp[op] = max_over_ranks(time_op(fn, reps=2, warm=1), world)
+        comp[op] = max_over_ranks(time_op(fn, reps=2 if "dp_" in op or "literal" in op else 10,
+                                          warm=1), world)
     dp_err = C.cudanp_dp_error_count(reset=True)
+    # the library's own version choice (S = CUDANP_S_AUTO, MAP_AUTO): what a
+    # caller gets with default arguments, against the autotuned best
+    auto = {}
+    if not args.no_sweep:
+        for op, fn, A_, x_, y_, kw in (("tmv", C.cudanp_tmv, A_t, x_t, y_t, {"n_outer": wt}),
+                                       ("mv", C.cudanp_mv, A_m, x_m, y_m, {})):
+            auto[op] = max_over_ranks(time_op(lambda: fn(A_, x_, y_, **kw), reps=30, warm=3), world)
 
     (St, dt, mt), (Sm, dm, mm) = best["tmv"], best["mv"]
     st = torch.cuda.current_stream()
@@ -383,6 +409,13 @@ def run_cudanp(args):
                "path": "pinned host A,x -> H2D -> cudanp_tmv + cudanp_mv -> D2H y (per rank)"}
         del A_h, Am_h
 
+    # ---- C5 (BASELINE configs[4]): strong scaling over the N ranks
+    c5 = None
+    if not args.no_c5:
+        del A_t, A_m, x_t, x_m, y_t, y_m
+        torch.cuda.empty_cache()
+        c5 = run_c5(C, P, rank, world, args.c5_steps, args.gather)
+
     if rank != 0:
         if world > 1:
             import torch.distributed as dist
@@ -390,6 +423,9 @@ def run_cudanp(args):
         return
 
     peak, peak_src = hbm_peak()
+    if c5 is not None:
+        for rec in (c5["tmv"], c5["reduce"]):
+            rec["frac_of_n_peak"] = round(rec["agg_gbs_kernel"] / (world * peak), 4)
     dom = "tmv" if t_tmv >= t_mv else "mv"
     dom_bytes = bytes_t if dom == "tmv" else bytes_m
     dom_ms = t_tmv if dom == "tmv" else t_mv
@@ -405,10 +441,11 @@ def run_cudanp(args):
         return round(nb / (t * 1e-3) / 1e9, 1)
 
     # "tuned S=1" = the best no-NP kernel: the S=1 instantiations, the literal and
-    # (TMV) the TMA-staged S=1 kernel
+    # the TMA-tiled S=1 kernel (rows staged through shared memory: the paper's
+    # "already optimized" SMM-style baseline)
     def best_s1(op):
         c = [v for (S, d, m), v in sweep[op].items() if S == 1]
-        for extra in (f"{op}_s1_literal", f"{op}_s1_tma"):  # every no-NP kernel we have
+        for extra in (f"{op}_s1_literal", f"{op}_s1_tiled"):  # every no-NP kernel we have
             if extra in comp:
                 c.append(comp[extra])
         return min(c or [float("nan")])
@@ -416,7 +453,8 @@ def run_cudanp(args):
     per_S = {}
     for op, nb in (("tmv", bytes_t), ("mv", bytes_m)):
         s1 = best_s1(op)
-        for S in C.SLAVE_SIZES + (64, 128, 256, 512, 1024):
+        for S in sorted(set(C.SLAVE_SIZES + C.INTER_ONLY_SIZES + C.MULTI_WARP_SIZES
+                            + C.TMV_CLUSTER_SIZES + C.CLUSTER_SIZES)):
             cand = {k: v for k, v in sweep[op].items() if k[0] == S}
             if not cand:
                 continue
@@ -453,67 +491,225 @@ def run_cudanp(args):
                      "traffic": traffic, "peak_source": peak_src,
                      "alg_bytes_per_launch": dom_bytes, "avg_launch_ms": round(dom_ms, 5)},
         "kernels": {"tmv": {"avg_ms": round(t_tmv, 5), "gbs": gbs(bytes_t, t_tmv),
-                            "speedup_vs_s1": round(s1_tmv / t_tmv, 3)},
+                            "speedup_vs_s1": round(s1_tmv / t_tmv, 3),
+                            "s1_tuned_ms": round(s1_tmv, 5)},
                     "mv": {"avg_ms": round(t_mv, 5), "gbs": gbs(bytes_m, t_mv),
-                           "speedup_vs_s1": round(s1_mv / t_mv, 3)}},
+                           "speedup_vs_s1": round(s1_mv / t_mv, 3),
+                           "s1_tuned_ms": round(s1_mv, 5)}},
+        "auto": {op: {"gbs": gbs(bytes_t if op == "tmv" else bytes_m, v),
+                      "vs_autotuned_best": round(best_ms[op] / v, 4),
+                      "choice": dict(zip(("S", "dist", "map"),
+                                         C.cudanp_choose_version(op, wt if op == "tmv" else hm, n)))}
+                 for op, v in auto.items()},
         "per_S": per_S,
         "comparison_ms": {k: round(v, 4) for k, v in comp.items()} | {"dp_launch_errors": dp_err},
         "gpu_launches": 2 * args.steps,
         "clocks": clk,
         "e2e": e2e,
     }
+    if c5 is not None:
+        line["c5"] = c5
     if not args.no_cpu_baseline:
-        line["cpu_baseline"] = cpu_baseline(A_t, x_t, n, wt, hm, A_m)
+        line["cpu_baseline"] = cpu_baseline(n, args.cpu_rows)
     print(json.dumps(line), flush=True)
     if world > 1:
         import torch.distributed as dist
         dist.destroy_process_group()
 
 
+# ------------------------------------------------------------------ C5 strong scaling
+C5_N_TMV = 65536
+C5_N_RED, C5_L_RED = 1 << 26, 64
+
+
+def run_c5(C, P, rank, world, steps, gather_mode):
+    """BASELINE configs[4]: TMV 65536 x 65536 fp32 sharded by column blocks and
+    a 64M-item x 64 fp32 loop-reduce sharded by item blocks (contiguous outer
+    ranges), outputs gathered to rank 0.  Strong scaling: the
+    problem is fixed, each rank generates its 1/N from global indices.  Per op:
+    version = the library's autotune on the shard (max over ranks), timed
+    `steps` times as kernel + gather with device events, max over ranks; the
+    library's own choice (S_AUTO) timed beside it; then pin P4 on exact data:
+    the gathered result must equal, bit for bit, the unsharded result that
+    rank 0 computes alone (at N = 1 the run is the unsharded one)."""
+    import torch
+    import torch.distributed as dist
+    fused = world > 1 and gather_mode == "fused"
+    native = P.NativeGroup(rank, world) if world > 1 and gather_mode == "native" else None
+    st = torch.cuda.current_stream()
+    out = {"workload": "C5: TMV 65536x65536 fp32 by column shards + 64M x 64 fp32 loop-reduce by "
+                       "item shards (BASELINE configs[4])",
+           "scaling": "strong", "n_gpus": world,
+           "gather": (gather_mode if world > 1 else "none (single GPU: outputs written in place)"),
+           "l2": "no flush: 16 GiB operands per op"}
+    for op in ("tmv", "reduce"):
+        total = C5_N_TMV if op == "tmv" else C5_N_RED
+        b, e = P.shard(total, world, rank)
+        if op == "tmv":
+            n = C5_N_TMV
+            A = torch.empty(n, e - b, dtype=torch.float32, device="cuda")
+            x = torch.empty(n, dtype=torch.float32, device="cuda")
+            nbytes = 4 * n * n + 8 * n
+        else:
+            A = torch.empty(e - b, C5_L_RED, dtype=torch.float32, device="cuda")
+            x = None
+            nbytes = 4 * C5_N_RED * C5_L_RED + 4 * C5_N_RED
+
+        def fill(kind):
+            if op == "tmv":
+                C.cudanp_generate(A, kind, stream_id=1, col0=b, w_global=C5_N_TMV)
+                C.cudanp_generate(x, kind, stream_id=2)
+            else:
+                C.cudanp_generate(A, kind, stream_id=1, row0=b, w_global=C5_L_RED)
+        fill("f32_unit")
+        root = torch.empty(total, dtype=torch.float32, device="cuda") if rank == 0 else None
+        y = root if world == 1 else torch.empty(e - b, dtype=torch.float32, device="cuda")
+        fg = P.FusedGather(root, total, rank, world) if fused else None
+        dst = fg.out_ptr() if fused else y
+
+        def kernel(S, d, m, o=None):
+            o = dst if o is None else o
+            if op == "tmv":
+                C.cudanp_tmv(A, x, o, S=S, dist=d, map=m, n_outer=e - b)
+            else:
+                C.cudanp_batched_loop_reduce(A, None, o, S=S, dist=d, map=m)
+
+        def gather():
+            if native is not None:
+                native.gather(y, root, total)
+            elif world > 1 and not fused:
+                P.gather_to_root(y, root, total, rank, world)
+
+        # version selection on this rank's shard, max over ranks so all agree
+        _, table = C.cudanp_autotune(op, A, x, y, lda=A.shape[1], n_outer=e - b,
+                                     n_inner=C5_N_TMV if op == "tmv" else C5_L_RED, reps=3)
+        cands = list(table)
+        vals = max_over_ranks_list([min(table[c], 1e30) for c in cands], world)
+        S, d, m = cands[min(range(len(cands)), key=vals.__getitem__)]
+        for _ in range(2):
+            kernel(S, d, m)
+            gather()
+        if fused:
+            fg.finish()
+        tk, tg = [], []
+        for _ in range(steps):
+            barrier(world)
+            torch.cuda.synchronize()
+            e0, e1, e2 = (torch.cuda.Event(enable_timing=True) for _ in range(3))
+            e0.record(st)
+            kernel(S, d, m)
+            e1.record(st)
+            gather()
+            e2.record(st)
+            torch.cuda.synchronize()
+            if fused:
+                fg.finish()
+            tk.append(e0.elapsed_time(e1))
+            tg.append(e1.elapsed_time(e2))
+        k_ms = max_over_ranks(statistics.median(tk), world)
+        g_ms = max_over_ranks(statistics.median(tg), world)
+        e_ms = max_over_ranks(statistics.median([p + q for p, q in zip(tk, tg)]), world)
+        # the library's own choice (S_AUTO), kernel only
+        ta = max_over_ranks(time_op(lambda: kernel(C.S_AUTO, C.CYCLIC, C.AUTO, y), reps=steps, warm=2), world)
+        rec = {"S": S, "dist": "cyclic" if d == C.CYCLIC else "block", "map": MAPN.get(m, str(m)),
+               "outer_total": total, "inner": C5_N_TMV if op == "tmv" else C5_L_RED,
+               "alg_bytes": nbytes, "kernel_max_ms": round(k_ms, 4), "gather_ms": round(g_ms, 4),
+               "e2e_ms": round(e_ms, 4),
+               "agg_gbs_kernel": round(nbytes / (k_ms * 1e-3) / 1e9, 1),
+               "agg_gbs_e2e": round(nbytes / (e_ms * 1e-3) / 1e9, 1),
+               "auto": {"choice": dict(zip(("S", "dist", "map"),
+                                           C.cudanp_choose_version(op, e - b, C5_N_TMV if op == "tmv" else C5_L_RED))),
+                        "kernel_ms": round(ta, 4), "vs_autotuned_best": round(k_ms / ta, 4)}}
+        # pin P4 on exact data (every summation order gives the same bits)
+        fill("f32_int4")
+        kernel(S, d, m)
+        gather()
+        torch.cuda.synchronize()
+        if fused:
+            fg.finish()
+        if rank == 0 and world > 1:
+            A = None
+            torch.cuda.empty_cache()
+            if op == "tmv":
+                Af = torch.empty(C5_N_TMV, C5_N_TMV, dtype=torch.float32, device="cuda")
+                C.cudanp_generate(Af, "f32_int4", stream_id=1)
+                full = C.cudanp_tmv(Af, x, S=S, dist=d, map=m)
+            else:
+                Af = torch.empty(C5_N_RED, C5_L_RED, dtype=torch.float32, device="cuda")
+                C.cudanp_generate(Af, "f32_int4", stream_id=1)
+                full = C.cudanp_batched_loop_reduce(Af, None, S=S, dist=d, map=m)
+            torch.cuda.synchronize()
+            rec["p4_sharded_equals_unsharded"] = bool(torch.equal(full, root))
+            del Af, full
+        elif rank == 0:
+            rec["p4_sharded_equals_unsharded"] = "n/a at N = 1 (the run is unsharded)"
+        barrier(world)
+        if fg:
+            fg.close()
+        out[op] = rec
+        A = x = y = root = dst = None
+        torch.cuda.empty_cache()
+    if native is not None:
+        native.close()
+    return out
+
+
 # ------------------------------------------------------------------ oracle (CPU) legs
-def _oracle_step_sample(A, x, rows_t, rows_m, threads=1):
-    """One oracle pass over a sample of the workload: TMV over the first
-    rows_t rows (all columns) and MV over the first rows_m rows.  threads > 1
-    runs the same oracle functions over contiguous outer-item ranges."""
+def _cpu_sample(n, rows):
+    """The CPU sample both arms time: the first `rows` rows of the C2 matrix
+    (generated on the host by synth, the same values the device generator
+    makes) and x."""
+    import synth
+    rows = min(rows, n)
+    return synth.matrix(rows, n, "f32_unit"), synth.vector(n, "f32_unit"), rows
+
+
+def _oracle_pass(A, x, rows, threads):
+    """One oracle pass over the sample: TMV over its rows (all columns) and MV
+    over its rows; threads > 1 runs the same oracle functions over contiguous
+    outer-item ranges."""
     import oracle as O
     t0 = time.perf_counter()
     if threads > 1:
-        O.tmv_parallel(A[:rows_t], x[:rows_t], threads)
-        O.mv_parallel(A[:rows_m], x, threads)
+        O.tmv_parallel(A, x[:rows], threads)
+        O.mv_parallel(A, x, threads)
     else:
-        O.tmv(A[:rows_t], x[:rows_t])
-        O.mv(A[:rows_m], x)
+        O.tmv(A, x[:rows])
+        O.mv(A, x)
     dt = time.perf_counter() - t0
-    nb = alg_bytes_matvec(rows_t, A.shape[1]) + alg_bytes_matvec(rows_m, A.shape[1])
-    return dt, nb
+    return dt, 2 * alg_bytes_matvec(rows, A.shape[1])
 
 
-def _timed_oracle(A, x, rows, threads, budget_s):
+def _timed_oracle(A, x, rows, threads, budget_s=None, passes=None):
     tot_t, tot_b, reps = 0.0, 0, 0
-    while tot_t < budget_s and reps < 200:
-        dt, nb = _oracle_step_sample(A, x, rows, rows, threads)
+    while (passes is not None and reps < passes) or (passes is None and tot_t < budget_s and reps < 500):
+        dt, nb = _oracle_pass(A, x, rows, threads)
         tot_t += dt
         tot_b += nb
         reps += 1
+        if passes is not None and tot_t > 150:
+            break
     return tot_b / tot_t / 1e9, reps, tot_t
 
 
-def cpu_baseline(A_t, x_t, n, wt, hm, A_m):
-    """The oracle as it stands (plain C, fp64 accumulation) on a bounded sample
-    of the same workload: the first 2048 rows for TMV and MV (1/8 of the
-    matrix), about 10 s on all host cores (contiguous outer-item ranges, one
-    thread each) and about 10 s on one core."""
-    import torch  # noqa: F401
-    rows = min(2048, n)
-    A = A_t[:rows].cpu().numpy()
-    x = x_t.cpu().numpy()
+def _sample_text(n, rows, cores):
+    return (f"TMV + MV over the first {rows} of {n} rows of the C2 matrix (1/{n // rows} of one "
+            f"step; the oracle's plain fp64-accumulating loops), {cores} threads over contiguous "
+            f"outer-item ranges")
+
+
+def cpu_baseline(n, rows):
+    """The oracle as it stands on the bounded sample (_cpu_sample) -- the same
+    sample and thread count the `--impl reference` arm times -- about 10 s on
+    all host cores, plus about 10 s on one core."""
+    A, x, rows = _cpu_sample(n, rows)
     cores = os.cpu_count() or 1
-    v_all, reps_all, t_all = _timed_oracle(A, x, rows, cores, 10.0)
-    v_one, reps_one, t_one = _timed_oracle(A, x, rows, 1, 10.0)
+    _oracle_pass(A, x, rows, cores)  # warm-up (page-in)
+    v_all, reps_all, t_all = _timed_oracle(A, x, rows, cores, budget_s=10.0)
+    v_one, reps_one, t_one = _timed_oracle(A, x, rows, 1, budget_s=10.0)
     return {"value": round(v_all, 4), "unit": "GB/s", "cores": cores, "kind": "oracle",
-            "sample": f"TMV + MV over the first {rows} of {n} rows of the C2 matrix "
-                      f"(1/{n // rows} of one step): {reps_all} repetitions on {cores} threads in "
-                      f"{t_all:.1f} s; 1-core: {reps_one} repetitions in {t_one:.1f} s",
+            "sample": _sample_text(n, rows, cores) + f": {reps_all} passes in {t_all:.1f} s; "
+                      f"1 core: {reps_one} passes in {t_one:.1f} s",
             "value_1core": round(v_one, 4), "cpu": _cpu_model()}
 
 
@@ -528,39 +724,29 @@ def _cpu_model():
 
 
 def run_reference(args):
-    """--impl reference: the oracle on the host cores, same metric/config."""
+    """--impl reference: the oracle on the host cores, same metric/config; each
+    step = one oracle pass over the same sample the cudanp arm's cpu_baseline
+    times (so the run states one CPU rate)."""
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return
-    import synth
     n = args.n
-    rows = min(512, n)
-    A = synth.matrix(rows, n, "f32_unit")
-    x = synth.vector(n, "f32_unit")
+    A, x, rows = _cpu_sample(n, args.cpu_rows)
     cores = os.cpu_count() or 1
-    for _ in range(max(args.warmup, 0) and 1):
-        _oracle_step_sample(A, x, rows, rows, cores)
-    ts, nbs = [], []
-    t_start = time.perf_counter()
-    for _ in range(args.steps):
-        dt, nb = _oracle_step_sample(A, x, rows, rows, cores)
-        ts.append(dt)
-        nbs.append(nb)
-        if time.perf_counter() - t_start > 120:
-            break
-    tot_t = sum(ts)
-    value = sum(nbs) / tot_t / 1e9
-    ms = tot_t / len(ts) * 1e3
-    sample = (f"each step: oracle TMV + MV over the first {rows} of {n} rows of the C2 matrix "
-              f"(1/{n // rows} of a step), {cores} threads over contiguous outer-item ranges")
+    if args.warmup > 0:
+        _oracle_pass(A, x, rows, cores)
+    value, steps, tot_t = _timed_oracle(A, x, rows, cores, passes=max(args.steps, 1))
+    ms = tot_t / steps * 1e3
+    sample = "each step: " + _sample_text(n, rows, cores)
     print(json.dumps({
         "impl": "reference", "metric": METRIC, "value": round(value, 4), "unit": "GB/s",
-        "n_gpus": args.gpus, "steps": len(ts), "warmup": args.warmup, "ms_per_step": round(ms, 3),
+        "n_gpus": args.gpus, "steps": steps, "warmup": args.warmup, "ms_per_step": round(ms, 3),
         "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64-accum",
         "data": "synthetic (counter-based generator, f32_unit)",
-        "config": {"workload": f"C2: TMV y=A^T x + MV y=A x, {n}x{n} fp32 (sampled rows)"},
+        "config": {"workload": f"C2: TMV y=A^T x + MV y=A x, {n}x{n} fp32 per rank (BASELINE configs[1]); "
+                               f"sampled rows", "h": n, "w": n, "sample_rows": rows},
         "cpu_baseline": {"value": round(value, 4), "unit": "GB/s", "cores": cores, "kind": "oracle",
-                         "sample": sample},
+                         "sample": sample, "cpu": _cpu_model()},
         "e2e": {"value": round(value, 4), "unit": "GB/s", "h2d_bytes_per_step": 0,
                 "d2h_bytes_per_step": 0},
     }), flush=True)
