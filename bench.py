@@ -70,7 +70,7 @@ def parse():
     ap.add_argument("--mv-cfg", default="256,cyclic,intra")
     ap.add_argument("--no-c5", action="store_true", help="skip the C5 strong-scaling block")
     ap.add_argument("--c5-steps", type=int, default=10)
-    ap.add_argument("--cpu-rows", type=int, default=1024,
+    ap.add_argument("--cpu-rows", type=int, default=4096,
                     help="rows of the C2 matrix in the oracle's CPU sample (both arms)")
     return ap.parse_args()
 
@@ -682,7 +682,7 @@ def _oracle_pass(A, x, rows, threads):
 
 def _timed_oracle(A, x, rows, threads, budget_s=None, passes=None):
     tot_t, tot_b, reps = 0.0, 0, 0
-    while (passes is not None and reps < passes) or (passes is None and tot_t < budget_s and reps < 500):
+    while (passes is not None and reps < passes) or (passes is None and tot_t < budget_s and reps < 5000):
         dt, nb = _oracle_pass(A, x, rows, threads)
         tot_t += dt
         tot_b += nb
@@ -690,6 +690,16 @@ def _timed_oracle(A, x, rows, threads, budget_s=None, passes=None):
         if passes is not None and tot_t > 150:
             break
     return tot_b / tot_t / 1e9, reps, tot_t
+
+
+def _cpu_warm(A, x, rows, threads, passes=1, min_s=2.0):
+    """Untimed passes (page-in, thread start-up, core clocks ramping): at least
+    `passes` and at least `min_s` seconds, in both arms alike."""
+    t0 = time.perf_counter()
+    k = 0
+    while k < passes or time.perf_counter() - t0 < min_s:
+        _oracle_pass(A, x, rows, threads)
+        k += 1
 
 
 def _sample_text(n, rows, cores):
@@ -704,7 +714,7 @@ def cpu_baseline(n, rows):
     all host cores, plus about 10 s on one core."""
     A, x, rows = _cpu_sample(n, rows)
     cores = os.cpu_count() or 1
-    _oracle_pass(A, x, rows, cores)  # warm-up (page-in)
+    _cpu_warm(A, x, rows, cores)
     v_all, reps_all, t_all = _timed_oracle(A, x, rows, cores, budget_s=10.0)
     v_one, reps_one, t_one = _timed_oracle(A, x, rows, 1, budget_s=10.0)
     return {"value": round(v_all, 4), "unit": "GB/s", "cores": cores, "kind": "oracle",
@@ -733,8 +743,7 @@ def run_reference(args):
     n = args.n
     A, x, rows = _cpu_sample(n, args.cpu_rows)
     cores = os.cpu_count() or 1
-    if args.warmup > 0:
-        _oracle_pass(A, x, rows, cores)
+    _cpu_warm(A, x, rows, cores, passes=max(args.warmup, 1))
     value, steps, tot_t = _timed_oracle(A, x, rows, cores, passes=max(args.steps, 1))
     ms = tot_t / steps * 1e3
     sample = "each step: " + _sample_text(n, rows, cores)
