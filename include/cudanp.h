@@ -102,9 +102,10 @@ typedef enum { CUDANP_SUM = 0, CUDANP_MAX = 1 } cudanp_op;
  * runs the TMA-staged kernel (cudanp_tmv_tma) when S is a power of two <= 32
  * and its preconditions hold, else the LDG inter-warp kernel (same result
  * contract; never CUDANP_ERR_UNSUPPORTED for alignment).  CUDANP_MAP_AUTO
- * takes the TMA-staged kernel under the same conditions when the matrix is
- * wide (2 x ceil(n_outer/128) >= SM count), else the LDG inter-warp kernel
- * (adjacent masters read adjacent columns). */
+ * takes the TMA-staged kernel under the same conditions when the 128-column
+ * strips give 0.3 .. 1.1 CTAs per SM (one resident strip per SM with a deep
+ * ring), else the LDG inter-warp kernel (adjacent
+ * masters read adjacent columns). */
 int cudanp_tmv(const float* A, int64_t lda, const float* x, float* y,
                int64_t n_outer, int64_t n_inner, int S, int dist, int map, void* stream);
 
@@ -335,7 +336,9 @@ int cudanp_launch_info(int op_kind, int64_t n_outer, int64_t n_inner, int dtype,
 /* The (S, dist, map) that S = CUDANP_S_AUTO selects for op_kind (0 tmv, 1 mv,
  * 2 reduce, 3 scan) on N = n_outer items of L = n_inner iterations, given
  * `map` (AUTO, or a map to keep) and vec4 as above.  Rule:
- * TMV wide -> TMA S = 8 cyclic, else inter-warp S = clamp(SMs*1024/N, 8, 64);
+ * TMV with 0.3..1.1 128-column strips per SM -> TMA S = 8 cyclic; wider ->
+ * inter-warp S = 32 block; narrower -> inter-warp S = clamp(2*SMs*1024/N,
+ * 8, 64), block when L/S <= 32;
  * MV intra S = clamp(L/64, 1, 256); reduce intra S = clamp(L/8, 1, 32);
  * scan intra S = clamp(L/4, 1, 16); reduce/scan/MV teams grow (up to S/32
  * warps, slaves keeping >= 8 elements) while N*S < SMs*1024. */

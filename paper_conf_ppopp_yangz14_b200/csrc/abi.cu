@@ -136,12 +136,19 @@ static int floor_pow2(int64_t v) {
 }
 static int clampi(int v, int lo, int hi) { return v < lo ? lo : (v > hi ? hi : v); }
 
-// TMA staging of TMV pays when the 128-column strips give at least half the
-// SMs a CTA each (the regime where the 4-wide LDG kernel is also used); on
-// narrower matrices (C1, 1024 columns: TMA S = 32 5.1 us vs LDG inter-warp
-// 3.2 us, profiles/sweep_r01n.jsonl) the LDG inter-warp kernel with more
-// slaves per column spreads the few columns better.
-static bool tmv_wide(int64_t w) { return 2 * ((w + 127) / 128) >= sm_count(); }
+// TMA staging of TMV pays while the 128-column strips give between ~0.3 and
+// ~1.1 CTAs per SM: one resident strip per SM with a deep ring of 32-64 KB
+// stages (profiles/tmv_width_r02d.jsonl: w = 8192..20480 at h = 16384/65536,
+// TMA 6.3-7.2 TB/s vs LDG 6.0-7.2).  Narrower (C1, 1024 columns: TMA S = 32
+// 5.1 us vs LDG inter-warp 3.2 us, profiles/sweep_r01n.jsonl; w = 4096: 4.1 vs
+// 4.7 TB/s) the LDG kernel with more slaves per column spreads the few
+// columns better; wider (w >= 24576: several strips per SM, smaller stages)
+// the LDG inter-warp kernel with S = 32 holds 6.8-7.3 TB/s where the TMA
+// ring's shape swings from 4.1 to 7.2.
+static bool tmv_wide(int64_t w) {
+  const int64_t strips = (w + 127) / 128, sms = sm_count();
+  return 10 * strips >= 3 * sms && 10 * strips <= 11 * sms;
+}
 // TMA preconditions: A 16-byte aligned, row pitch a multiple of 16 bytes,
 // coordinates in int32, something to stream.  y is stored with scalar stores
 // and x with ordinary loads, so neither needs alignment.
@@ -157,8 +164,10 @@ static bool tma_ok(const float* A, int64_t lda, int64_t w, int64_t h) {
 // anything.  T = SMs x 1024 threads is "enough threads to fill the GPU":
 // when N x S falls short, the team grows (NP pays when outer
 // TLP is short), up to a team whose slaves still get >= 8 elements each.
-//   TMV: wide + TMA-able -> TMA, S = 8 cyclic (C2 best); else inter-warp LDG
-//        with S = clamp(T / w, 8, 64), block when S >= 64 (C1 best: 64 block).
+//   TMV: tmv_wide + TMA-able -> TMA, S = 8 cyclic (C2 best); wider than that
+//        -> LDG inter-warp S = 32 block; narrower -> LDG inter-warp with
+//        S = clamp(2T / w, 8, 64), block when each slave's share is <= 32
+//        rows (C1: 64 block), cyclic otherwise (w = 4096: 64 cyclic).
 //   MV:  intra, S = clamp(L / 64, 1, 256) cyclic (C2 best: S = 256), grown.
 //   reduce: intra, S = clamp(L / 8, 1, 32) (C3: 4/8/16/32 at L = 32..256),
 //        block above L = 32 (L % 4 != 0: L / 16), grown.
@@ -182,12 +191,16 @@ int choose_version(int op_kind, int64_t N, int64_t L, bool vec, bool tma, int ma
       if (m == CUDANP_MAP_INTER_WARP_TMA) m = CUDANP_MAP_INTER_WARP;  // fallback (not TMA-able)
       if (m == CUDANP_MAP_INTRA_WARP) {
         s = clampi(floor_pow2(N > 0 ? T / N : 32), 1, 32);
+      } else if (10 * ((N + 127) / 128) > 11 * (int64_t)sm_count()) {
+        m = CUDANP_MAP_INTER_WARP;  // wide: several strips per SM
+        s = 32;
+        d = CUDANP_DIST_BLOCK;
       } else {
         m = CUDANP_MAP_INTER_WARP;
-        s = clampi(floor_pow2(N > 0 ? T / N : 64), 8, 64);
-        d = s >= 64 ? CUDANP_DIST_BLOCK : CUDANP_DIST_CYCLIC;
+        s = clampi(floor_pow2(N > 0 ? 2 * T / N : 64), 8, 64);
       }
       s = clampi(s, 1, clampi(floor_pow2(L / 4), 1, 64));
+      if (m == CUDANP_MAP_INTER_WARP && s != 32) d = L / s <= 32 ? CUDANP_DIST_BLOCK : CUDANP_DIST_CYCLIC;
       break;
     case 1:  // MV
       if (m == CUDANP_MAP_INTER_WARP) {

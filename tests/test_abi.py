@@ -94,6 +94,9 @@ def test_auto_team_size_rule(lib):
     # not 16-byte aligned -> LDG inter-warp
     assert ch("tmv", 16384, 16384) == (8, C.CYCLIC, C.INTER_WARP_TMA)
     assert ch("tmv", 1024, 1024) == (64, C.BLOCK, C.INTER_WARP)
+    assert ch("tmv", 4096, 16384) == (64, C.CYCLIC, C.INTER_WARP)
+    assert ch("tmv", 8192, 65536) == (8, C.CYCLIC, C.INTER_WARP_TMA)   # C5 shard at G = 8
+    assert ch("tmv", 65536, 65536) == (32, C.BLOCK, C.INTER_WARP)     # C5 at G = 1
     S, d, m = ch("tmv", 16384, 16384, vec4=False)
     assert m == C.INTER_WARP and 8 <= S <= 64
     # MV: C2 rows -> a 256-thread team (the bench's fastest); short rows stay small

@@ -110,6 +110,37 @@ def main():
         C.cudanp_group_destroy(g)
     for S in (3, 5, 10, 15):
         C.cudanp_le_gicov(le, 0.01, S=S, map=C.INTER_WARP, layout=0)
+        for d in (C.CYCLIC, C.BLOCK):  # non-power-of-two inter-warp teams
+            C.cudanp_tmv(A, xt, S=S, dist=d, map=C.INTER_WARP, n_outer=70)
+            C.cudanp_mv(A4, xm4, S=S, dist=d, map=C.INTER_WARP)
+            for X, ini in ((Xf, inif), (Xi, inii)):
+                C.cudanp_batched_loop_reduce(X, ini, S=S, dist=d, map=C.INTER_WARP)
+                C.cudanp_batched_loop_scan(X, ini, S=S, dist=d, map=C.INTER_WARP)
+    # more items than one persistent wave of the multi-warp kernels (their
+    # grid-stride loops), S = 64 reduce/scan and S = 256 MV
+    Xw = dev(synth.items(5003, 16, "i32_small"))
+    Xwf = dev(synth.items(5003, 16, "f32_unit"))
+    Aw = dev(synth.matrix(2500, 64, "f32_unit"))
+    xw = dev(synth.vector(64))
+    for d in (C.CYCLIC, C.BLOCK):
+        C.cudanp_batched_loop_reduce(Xw, None, S=64, dist=d)
+        C.cudanp_batched_loop_scan(Xwf, None, S=64, dist=d)
+        C.cudanp_mv(Aw, xw, S=256, dist=d)
+    # the library's own version choice (S = S_AUTO) and the TMA fallbacks
+    C.cudanp_tmv(A4, xt)
+    C.cudanp_mv(A4, xm4)
+    C.cudanp_batched_loop_reduce(Xi4)
+    C.cudanp_batched_loop_scan(Xf)
+    yb = torch.empty(69, device="cuda")
+    C.cudanp_tmv(A4, xt, yb[1:], S=8, map=C.INTER_WARP_TMA)  # y off 16-byte alignment
+    # tiled S = 1 baselines (TMA rings that wrap; TMA stores for the scan)
+    Am = dev(synth.matrix(300, 1000, "f32_unit"))
+    xmm = dev(synth.vector(1000))
+    C.cudanp_mv_variant(C.S1_TILED, Am, xmm)
+    C.cudanp_mv_variant(C.S1_TILED, A4, xm4)
+    Xs = dev(synth.items(300, 1000, "i32_small"))
+    C.cudanp_batched_loop_scan_variant(C.S1_TILED, Xs, dev(synth.init(300, "i32_small")))
+    C.cudanp_batched_loop_scan_variant(C.S1_TILED, Xf)
     if not quick:
         C.cudanp_dp_set_pending_launch_limit(1 << 12)
         for impl in (C.S1_LITERAL,) if no_dp else (C.S1_LITERAL, C.DP_THREAD, C.DP_BLOCK):
