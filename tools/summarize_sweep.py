@@ -39,7 +39,7 @@ def main(path, out=None):
             b = max(np_, key=lambda r: r["gbs"])
         else:
             continue
-        comp = {r["impl"]: r for r in rs if r["impl"] not in ("np", "best_np")}
+        comp = {r["impl"]: r for r in rs if r["impl"] not in ("np", "best_np", "fig12", "auto")}
 
         def vs(name):
             c = comp.get(name)
@@ -61,6 +61,20 @@ def main(path, out=None):
                          f"{r['L']} | {r['S']},{r['dist']},{r['map']} | {r['gbs']:.0f} | {r['gbs_steady']:.0f} | "
                          f"{100 * r['gbs_steady'] / PEAK:.1f} | {r['s1_steady']} | {r['gbs_s1_steady']:.0f} | "
                          f"{r['speedup_vs_s1_steady']:.2f}x |")
+    au = [r for r in recs if r["impl"] == "auto" and "vs_best_np" in r]
+    if au:
+        lines += ["", "Library's own choice (S = S_AUTO, MAP_AUTO) against the swept best NP version", "",
+                  "| config | op | dtype | L | auto GB/s | auto / best NP | auto / tuned S=1 |", "|---|---|---|---|---|---|---|"]
+        lines += [f"| {r['config']} | {r['op']}{(' ' + r['opname']) if r.get('opname') else ''} | {r['dtype']} | "
+                  f"{r['L']} | {r['gbs']:.0f} | {r['vs_best_np']:.3f} | {r['vs_s1_tuned']:.2f}x |" for r in au]
+    f12 = [r for r in recs if r["impl"] == "fig12"]
+    if f12:
+        lines += ["", "Fig 12 analog: non-power-of-two inter-warp S vs the power of two it pads to (GB/s)", "",
+                  "| config | op | dtype | L | S | dist | GB/s | padded S | padded GB/s | S / padded |",
+                  "|---|---|---|---|---|---|---|---|---|---|"]
+        lines += [f"| {r['config']} | {r['op']}{(' ' + r['opname']) if r.get('opname') else ''} | {r['dtype']} | "
+                  f"{r['L']} | {r['S']} | {r['dist']} | {r['gbs']:.0f} | {r['S_padded']} | {r['gbs_padded']:.0f} | "
+                  f"{r['speedup_vs_padded']:.2f}x |" for r in f12]
     f3 = [r for r in special if r["config"] == "F3"]
     if f3:
         lines += ["", "F3 — Fig 1 memcopy (64M floats): impl, m parents x n children, GB/s", "",

@@ -121,7 +121,7 @@ def graph_time_ms(fns, reps=5):
 
 
 def sweep_np(cfg, op, nbytes, run, extra, s1_ref=None, literal=None, comps=(), maps=None, call=None,
-             big=()):
+             big=(), auto=None):
     """run(S, dist, map) -> (median_ms, min_ms).  s1_ref: extra no-NP kernel
     times (e.g. the TMA-staged S=1 TMV) that count toward "tuned S=1".
     call(S, dist, map) -> a one-launch callable: the best NP and the best S=1
@@ -132,6 +132,9 @@ def sweep_np(cfg, op, nbytes, run, extra, s1_ref=None, literal=None, comps=(), m
                                                "reduce": (C.INTRA_WARP_TMA,)}.get(op, ())
     cands = list(itertools.product(C.SLAVE_SIZES, (C.CYCLIC, C.BLOCK), maps)) + \
         [(S, d, m) for S, m in big for d in (C.CYCLIC, C.BLOCK)]
+    if C.INTER_WARP in maps and op in ("tmv", "mv", "reduce", "scan"):
+        # non-power-of-two inter-warp teams (Fig 12)
+        cands += list(itertools.product(C.INTER_ONLY_SIZES, (C.CYCLIC, C.BLOCK), (C.INTER_WARP,)))
     for S, d, m in cands:
         try:
             res[(S, d, m)] = run(S, d, m)
@@ -157,6 +160,24 @@ def sweep_np(cfg, op, nbytes, run, extra, s1_ref=None, literal=None, comps=(), m
               "alg_bytes": nbytes, "gbs": round(nbytes / (t * 1e-3) / 1e9, 1),
               "speedup_of_best_np": round(t / res[best][0], 3)})
     bS, bd, bm = best
+    # Fig 12 analog: each non-power-of-two inter-warp S against the power of two
+    # it would be padded to under intra-warp NP's limit
+    for S in C.INTER_ONLY_SIZES:
+        P2 = 1 << (S - 1).bit_length()
+        for d in (C.CYCLIC, C.BLOCK):
+            k, kp = (S, d, C.INTER_WARP), (P2, d, C.INTER_WARP)
+            if k in res and kp in res:
+                emit({"config": cfg, "op": op, **extra, "impl": "fig12", "S": S, "S_padded": P2,
+                      "dist": DN[d], "map": "inter", "t_median_us": round(res[k][0] * 1e3, 2),
+                      "t_padded_us": round(res[kp][0] * 1e3, 2), "alg_bytes": nbytes,
+                      "gbs": round(nbytes / (res[k][0] * 1e-3) / 1e9, 1),
+                      "gbs_padded": round(nbytes / (res[kp][0] * 1e-3) / 1e9, 1),
+                      "speedup_vs_padded": round(res[kp][0] / res[k][0], 3)})
+    if auto is not None:  # the library's own choice (S = S_AUTO, MAP_AUTO)
+        ta = auto()[0]
+        emit({"config": cfg, "op": op, **extra, "impl": "auto", "t_median_us": round(ta * 1e3, 2),
+              "alg_bytes": nbytes, "gbs": round(nbytes / (ta * 1e-3) / 1e9, 1),
+              "vs_best_np": round(res[best][0] / ta, 3), "vs_s1_tuned": round(s1 / ta, 3)})
     steady = {}
     if call is not None:
         best1 = min((k for k in res if k[0] == 1), key=lambda k: res[k][0])
@@ -190,10 +211,12 @@ def c1():
         return graph_time_ms([lambda i=i: C.cudanp_tmv(As[i], x, ys[i], S=S, dist=d, map=m)
                               for i in range(copies)])
     lit = graph_time_ms([lambda i=i: C.cudanp_tmv_variant(C.S1_LITERAL, As[i], x, ys[i]) for i in range(copies)])[0]
-    comps = [("s1_literal", lit)]
+    tiled = graph_time_ms([lambda i=i: C.cudanp_tmv_variant(C.S1_TILED, As[i], x, ys[i]) for i in range(copies)])[0]
+    comps = [("s1_literal", lit), ("s1_tiled", tiled)]
     for impl, name in ((C.DP_BLOCK, "dp_block"), (C.DP_THREAD, "dp_thread")):
         comps.append((name, time_ms(lambda: C.cudanp_tmv_variant(impl, As[0], x, ys[0]), reps=5)[0]))
-    sweep_np("C1", "tmv", nb, run, {"dtype": "f32", "N": n, "L": n}, literal=lit, comps=comps)
+    sweep_np("C1", "tmv", nb, run, {"dtype": "f32", "N": n, "L": n}, literal=lit, comps=comps, s1_ref=[tiled],
+             auto=lambda: graph_time_ms([lambda i=i: C.cudanp_tmv(As[i], x, ys[i]) for i in range(copies)]))
     for S in (64, 128):  # teams larger than a warp (inter-warp, 8 masters per CTA)
         for d in (C.CYCLIC, C.BLOCK):
             med, mn = run(S, d, C.INTER_WARP)
@@ -210,12 +233,12 @@ def c2():
     nb = 4 * n * n + 8 * n
     for op, fnp, fv in (("tmv", C.cudanp_tmv, C.cudanp_tmv_variant), ("mv", C.cudanp_mv, C.cudanp_mv_variant)):
         lit = time_ms(lambda: fv(C.S1_LITERAL, A, x, y), reps=3)[0]
-        comps = [("s1_literal", lit)]
-        s1_ref = []
-        if op == "tmv":  # the no-NP kernel with TMA staging is part of the tuned S=1 baseline
-            t_tma1 = min(time_ms(lambda: C.cudanp_tmv_tma(A, x, y, S=1, dist=d))[0] for d in (C.CYCLIC, C.BLOCK))
-            comps.append(("s1_tma", t_tma1))
-            s1_ref.append(t_tma1)
+        # the no-NP kernel with rows staged through shared memory by TMA (the
+        # paper's SMM-style "already optimized" baseline) is part of the
+        # tuned S=1 baseline
+        t_tiled = time_ms(lambda: fv(C.S1_TILED, A, x, y))[0]
+        comps = [("s1_literal", lit), ("s1_tiled", t_tiled)]
+        s1_ref = [t_tiled]
         for impl, name in ((C.DP_BLOCK, "dp_block"), (C.DP_THREAD, "dp_thread")):
             comps.append((name, time_ms(lambda: fv(impl, A, x, y), reps=3, warm=1)[0]))
         # vendor-library context (the paper's CUBLAS comparison, Figs 13/14; not
@@ -228,7 +251,8 @@ def c2():
                [(S, C.INTER_WARP) for S in (64, 128) + C.TMV_CLUSTER_SIZES])
         sweep_np("C2", op, nb, lambda S, d, m: time_ms(lambda: fnp(A, x, y, S=S, dist=d, map=m)),
                  {"dtype": "f32", "N": n, "L": n}, s1_ref=s1_ref, literal=lit, comps=comps, big=big,
-                 call=lambda S, d, m: (lambda: fnp(A, x, y, S=S, dist=d, map=m)))
+                 call=lambda S, d, m: (lambda: fnp(A, x, y, S=S, dist=d, map=m)),
+                 auto=lambda: time_ms(lambda: fnp(A, x, y)))
     tma_sweep("C2", A, x, y, n)
     del A
 
@@ -266,6 +290,10 @@ def c3(Ls=(32, 64, 128, 256, 80, 150)):
             lit = time_ms(lambda: C.cudanp_batched_loop_reduce_variant(C.S1_LITERAL, x, None, out, op=op))[0]
             comps = [("s1_literal", lit),
                      ("dp_block", time_ms(lambda: C.cudanp_batched_loop_reduce_variant(C.DP_BLOCK, x, None, out, op=op), reps=3, warm=1)[0])]
+            s1_ref = []
+            if L % 4 == 0:  # one thread per item, rows staged by TMA (S1_TILED)
+                s1_ref.append(time_ms(lambda: C.cudanp_batched_loop_reduce_variant(C.S1_TILED, x, None, out, op=op))[0])
+                comps.append(("s1_tiled", s1_ref[-1]))
             # DP per thread: one device launch per item (full size if the runtime takes it)
             Np = 65536
             xp, op_ = x[:Np], out[:Np]
@@ -275,8 +303,9 @@ def c3(Ls=(32, 64, 128, 256, 80, 150)):
             sweep_np("C3", "reduce", nb,
                      lambda S, d, m: time_ms(lambda: C.cudanp_batched_loop_reduce(x, None, out, op=op, S=S, dist=d, map=m)),
                      {"dtype": "f32" if dtype == C.F32 else "i32", "opname": "sum" if op == C.SUM else "max",
-                      "N": N, "L": L}, literal=lit, comps=comps,
-                     call=lambda S, d, m: (lambda: C.cudanp_batched_loop_reduce(x, None, out, op=op, S=S, dist=d, map=m)))
+                      "N": N, "L": L}, literal=lit, comps=comps, s1_ref=s1_ref,
+                     call=lambda S, d, m: (lambda: C.cudanp_batched_loop_reduce(x, None, out, op=op, S=S, dist=d, map=m)),
+                     auto=lambda: time_ms(lambda: C.cudanp_batched_loop_reduce(x, None, out, op=op)))
             del x, out
             torch.cuda.empty_cache()
 
@@ -289,7 +318,8 @@ def c4(Ls=(64, 128, 256, 512, 1024)):
             out = torch.empty_like(x)
             nb = 8 * N * L
             lit = time_ms(lambda: C.cudanp_batched_loop_scan_variant(C.S1_LITERAL, x, None, out), reps=3)[0]
-            comps = [("s1_literal", lit),
+            t_tiled = time_ms(lambda: C.cudanp_batched_loop_scan_variant(C.S1_TILED, x, None, out), reps=3)[0]
+            comps = [("s1_literal", lit), ("s1_tiled", t_tiled),
                      ("dp_block", time_ms(lambda: C.cudanp_batched_loop_scan_variant(C.DP_BLOCK, x, None, out), reps=3, warm=1)[0])]
             Np = 65536
             xp, op_ = x[:Np], out[:Np]
@@ -299,7 +329,9 @@ def c4(Ls=(64, 128, 256, 512, 1024)):
             sweep_np("C4", "scan", nb,
                      lambda S, d, m: time_ms(lambda: C.cudanp_batched_loop_scan(x, None, out, S=S, dist=d, map=m), reps=3),
                      {"dtype": "f32" if dtype == C.F32 else "i32", "N": N, "L": L}, literal=lit, comps=comps,
-                     call=lambda S, d, m: (lambda: C.cudanp_batched_loop_scan(x, None, out, S=S, dist=d, map=m)))
+                     s1_ref=[t_tiled],
+                     call=lambda S, d, m: (lambda: C.cudanp_batched_loop_scan(x, None, out, S=S, dist=d, map=m)),
+                     auto=lambda: time_ms(lambda: C.cudanp_batched_loop_scan(x, None, out), reps=3))
             del x, out
             torch.cuda.empty_cache()
 
@@ -316,6 +348,10 @@ def c5():
         emit({"config": "C5", "op": "tmv", "dtype": "f32", "N": n, "L": n, "G": 1, "S": S, "dist": DN[d],
               "map": "inter", "impl": "np", "t_median_us": round(med * 1e3, 1), "alg_bytes": nb,
               "gbs": round(nb / (med * 1e-3) / 1e9, 1)})
+    med, _ = time_ms(lambda: C.cudanp_tmv(A, x, y), reps=3)
+    emit({"config": "C5", "op": "tmv", "dtype": "f32", "N": n, "L": n, "G": 1, "impl": "auto",
+          "choice": C.cudanp_choose_version("tmv", n, n), "t_median_us": round(med * 1e3, 1),
+          "alg_bytes": nb, "gbs": round(nb / (med * 1e-3) / 1e9, 1)})
     del A
     torch.cuda.empty_cache()
     N, L = 1 << 26, 64
@@ -327,6 +363,10 @@ def c5():
         emit({"config": "C5", "op": "reduce", "dtype": "f32", "N": N, "L": L, "G": 1, "S": S, "dist": DN[d],
               "map": "intra", "impl": "np", "t_median_us": round(med * 1e3, 1), "alg_bytes": nb,
               "gbs": round(nb / (med * 1e-3) / 1e9, 1)})
+    med, _ = time_ms(lambda: C.cudanp_batched_loop_reduce(xr, None, out), reps=3)
+    emit({"config": "C5", "op": "reduce", "dtype": "f32", "N": N, "L": L, "G": 1, "impl": "auto",
+          "choice": C.cudanp_choose_version("reduce", N, L), "t_median_us": round(med * 1e3, 1),
+          "alg_bytes": nb, "gbs": round(nb / (med * 1e-3) / 1e9, 1)})
     del xr, out
     torch.cuda.empty_cache()
 
