@@ -70,6 +70,11 @@ def parse():
     ap.add_argument("--mv-cfg", default="256,cyclic,intra")
     ap.add_argument("--no-c5", action="store_true", help="skip the C5 strong-scaling block")
     ap.add_argument("--c5-steps", type=int, default=10)
+    ap.add_argument("--oracle-timing", default=None, metavar="JSONL",
+                    help="time the CPU oracle on C1-C5 (1 core / all cores / generation only; "
+                         "SURVEY §8(d)) into JSONL and exit (no GPU work)")
+    ap.add_argument("--oracle-cap-s", type=float, default=12.0,
+                    help="--oracle-timing: seconds per (config, op, cores) before extrapolating")
     ap.add_argument("--cpu-rows", type=int, default=4096,
                     help="rows of the C2 matrix in the oracle's CPU sample (both arms)")
     return ap.parse_args()
@@ -761,8 +766,112 @@ def run_reference(args):
     }), flush=True)
 
 
+def oracle_timing(path, cap_s):
+    """SURVEY §8(d) "Oracle timing": the oracle's on-the-fly-generating forms
+    (orc_*_gen: inputs recomputed from the counter-based generator, no
+    multi-GiB host copies) timed on C1-C5 on 1 core and on all host cores
+    (contiguous outer-item ranges, one thread each), plus a generation-only
+    pass over the same input elements.  A run that would exceed `cap_s` is
+    stopped after whole chunks and extrapolated (the record says the fraction
+    done).  The oracle as it stands -- never tuned for this."""
+    import ctypes
+    from concurrent.futures import ThreadPoolExecutor
+
+    import oracle as O
+    L = O.lib()
+    cores = os.cpu_count() or 1
+    seed = O.SEED
+    K = O.KIND
+
+    def tmv_chunk(h, w):
+        def f(lo, hi):
+            cols = np.arange(lo, hi, dtype=np.int64)
+            y = np.empty(hi - lo, np.float32)
+            L.orc_tmv_gen(seed, K["f32_unit"], K["f32_unit"], h, w, cols.ctypes.data, hi - lo, y.ctypes.data)
+        return f
+
+    def mv_chunk(h, w):
+        def f(lo, hi):
+            rows = np.arange(lo, hi, dtype=np.int64)
+            y = np.empty(hi - lo, np.float32)
+            L.orc_mv_gen(seed, K["f32_unit"], K["f32_unit"], h, w, rows.ctypes.data, hi - lo, y.ctypes.data)
+        return f
+
+    def reduce_chunk(Lc):
+        def f(lo, hi):
+            it = np.arange(lo, hi, dtype=np.int64)
+            o = np.empty(hi - lo, np.float32)
+            L.orc_reduce_gen(seed, O.F32, K["f32_unit"], 1 << 20, -1, Lc, O.SUM, it.ctypes.data, hi - lo,
+                             o.ctypes.data)
+        return f
+
+    def scan_chunk(Lc):
+        def f(lo, hi):
+            it = np.arange(lo, hi, dtype=np.int64)
+            o = np.empty((hi - lo) * Lc, np.int32)
+            L.orc_scan_gen(seed, O.I32, K["i32_small"], 1 << 15, -1, Lc, it.ctypes.data, hi - lo, o.ctypes.data)
+        return f
+
+    def gen_chunk():
+        buf = {}
+
+        def f(lo, hi):  # generation only: the same input elements, materialized in a scratch buffer
+            b = buf.setdefault(threading.get_ident(), np.empty(1 << 22, np.float32))
+            i = lo
+            while i < hi:
+                n = min(hi - i, b.size)
+                L.orc_gen_f32(seed, 1, K["f32_unit"], i, n, b.ctypes.data)
+                i += n
+        return f
+
+    def timed(fn, n_outer, chunk, threads):
+        """Run fn over [0, n_outer) in chunks of `chunk`, on `threads` threads,
+        until done or cap_s; return (seconds extrapolated to all, fraction done)."""
+        bounds = [(lo, min(lo + chunk, n_outer)) for lo in range(0, n_outer, chunk)]
+        done, t0 = 0, time.perf_counter()
+        with ThreadPoolExecutor(threads) as ex:
+            for k in range(0, len(bounds), threads):
+                list(ex.map(lambda b: fn(*b), bounds[k:k + threads]))
+                done += sum(b[1] - b[0] for b in bounds[k:k + threads])
+                if time.perf_counter() - t0 > cap_s:
+                    break
+        dt = time.perf_counter() - t0
+        return dt * n_outer / done, done / n_outer
+
+    cases = [("C1", "tmv", 1024, 1024, tmv_chunk(1024, 1024), 4 * 1024 * 1024 + 8 * 1024, 1024 * 1024),
+             ("C2", "tmv", 16384, 16384, tmv_chunk(16384, 16384), 4 * 16384 ** 2 + 8 * 16384, 16384 ** 2),
+             ("C2", "mv", 16384, 16384, mv_chunk(16384, 16384), 4 * 16384 ** 2 + 8 * 16384, 16384 ** 2)]
+    cases += [("C3", "reduce", 1 << 22, Lc, reduce_chunk(Lc), 4 * (1 << 22) * Lc + 4 * (1 << 22), (1 << 22) * Lc)
+              for Lc in (32, 64, 128, 256)]
+    cases += [("C4", "scan", 1 << 21, Lc, scan_chunk(Lc), 8 * (1 << 21) * Lc, (1 << 21) * Lc)
+              for Lc in (64, 128, 256, 512, 1024)]
+    cases += [("C5", "tmv", 65536, 65536, tmv_chunk(65536, 65536), 4 * 65536 ** 2 + 8 * 65536, 65536 ** 2),
+              ("C5", "reduce", 1 << 26, 64, reduce_chunk(64), 4 * (1 << 26) * 64 + 4 * (1 << 26), (1 << 26) * 64)]
+    with open(path, "w") as f:
+        for cfg, op, N, Lc, fn, nbytes, elems in cases:
+            chunk = max(1, N // (64 * cores))
+            rec = {"config": cfg, "op": op, "N": N, "L": Lc, "alg_bytes": nbytes, "elements": elems,
+                   "cpu": _cpu_model(), "cores": cores, "kind": "oracle (on-the-fly generation)"}
+            for name, threads in (("1core", 1), ("allcore", cores)):
+                t, frac = timed(fn, N, chunk, threads)
+                rec[f"s_{name}"] = round(t, 3)
+                rec[f"gbs_{name}"] = round(nbytes / t / 1e9, 4)
+                rec[f"frac_done_{name}"] = round(frac, 4)
+            tg, fg = timed(gen_chunk(), elems, max(1, elems // (64 * cores)), cores)
+            rec["s_gen_only_allcore"] = round(tg, 3)
+            rec["frac_done_gen_only"] = round(fg, 4)
+            rec["s_compute_allcore"] = round(max(rec["s_allcore"] - tg, 0.0), 3)
+            f.write(json.dumps(rec) + "\n")
+            f.flush()
+            print(json.dumps(rec), flush=True)
+    del ctypes
+
+
 def main():
     args = parse()
+    if args.oracle_timing:
+        oracle_timing(args.oracle_timing, args.oracle_cap_s)
+        return
     if args.impl == "reference":
         run_reference(args)
     else:

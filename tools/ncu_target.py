@@ -20,7 +20,8 @@ def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--op", required=True, choices=["tmv", "mv", "reduce", "scan", "tmv_literal",
                                                     "mv_literal", "reduce_literal", "scan_literal",
-                                                    "ragged", "le", "le_literal", "tmv_tma"])
+                                                    "ragged", "le", "le_literal", "tmv_tma",
+                                                    "mv_tiled", "tmv_tiled", "scan_tiled", "reduce_tiled"])
     ap.add_argument("--lens", default="uniform", help="ragged: length distribution")
     ap.add_argument("--layout", type=int, default=0, help="le: 0 item-major, 1 point-major")
     ap.add_argument("--S", type=int, default=8)
@@ -33,7 +34,8 @@ def main():
     ap.add_argument("--reps", type=int, default=3)
     a = ap.parse_args()
     d = {"cyclic": C.CYCLIC, "block": C.BLOCK}[a.dist]
-    m = {"auto": C.AUTO, "intra": C.INTRA_WARP, "inter": C.INTER_WARP, "inter_tma": C.INTER_WARP_TMA}[a.map]
+    m = {"auto": C.AUTO, "intra": C.INTRA_WARP, "inter": C.INTER_WARP, "inter_tma": C.INTER_WARP_TMA,
+         "intra_tma": C.INTRA_WARP_TMA}[a.map]
     C.load()
     if a.op == "ragged":
         import synth
@@ -57,7 +59,9 @@ def main():
                "tmv_tma": lambda: C.cudanp_tmv_tma(A, x, y, S=a.S, dist=d),
                "mv": lambda: C.cudanp_mv(A, x, y, S=a.S, dist=d, map=m),
                "tmv_literal": lambda: C.cudanp_tmv_variant(C.S1_LITERAL, A, x, y),
-               "mv_literal": lambda: C.cudanp_mv_variant(C.S1_LITERAL, A, x, y)}
+               "mv_literal": lambda: C.cudanp_mv_variant(C.S1_LITERAL, A, x, y),
+               "mv_tiled": lambda: C.cudanp_mv_variant(C.S1_TILED, A, x, y),
+               "tmv_tiled": lambda: C.cudanp_tmv_variant(C.S1_TILED, A, x, y)}
     else:
         dt = torch.float32 if a.dtype == "f32" else torch.int32
         X = torch.empty(a.N, a.L, dtype=dt, device="cuda")
@@ -67,7 +71,9 @@ def main():
         fns = {"reduce": lambda: C.cudanp_batched_loop_reduce(X, None, o1, S=a.S, dist=d, map=m),
                "scan": lambda: C.cudanp_batched_loop_scan(X, None, o2, S=a.S, dist=d, map=m),
                "reduce_literal": lambda: C.cudanp_batched_loop_reduce_variant(C.S1_LITERAL, X, None, o1),
-               "scan_literal": lambda: C.cudanp_batched_loop_scan_variant(C.S1_LITERAL, X, None, o2)}
+               "scan_literal": lambda: C.cudanp_batched_loop_scan_variant(C.S1_LITERAL, X, None, o2),
+               "reduce_tiled": lambda: C.cudanp_batched_loop_reduce_variant(C.S1_TILED, X, None, o1),
+               "scan_tiled": lambda: C.cudanp_batched_loop_scan_variant(C.S1_TILED, X, None, o2)}
     for _ in range(a.reps):
         fns[a.op]()
     torch.cuda.synchronize()
