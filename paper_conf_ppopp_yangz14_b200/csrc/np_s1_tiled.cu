@@ -15,9 +15,11 @@
 // the NP speedups (CUDANP_IMPL_S1_TILED); the method (one master, no slaves)
 // is the literal Fig 2 loop.
 //
-//  MV:   a CTA owns R rows; a producer warp streams the column tiles into the
-//        ring; each consumer thread accumulates its row (acc += A[r][j]*x[j],
-//        x read through L1, broadcast across the warp) and stores y[r].
+//  MV:   a CTA owns R rows; a producer warp streams the column tiles -- and
+//        the matching 128-byte chunk of x (a 1-D bulk copy on the same
+//        barrier) -- into the ring; each consumer thread accumulates its row
+//        (acc += A[r][j]*x[j], x read from shared memory as a broadcast) and
+//        stores y[r].
 //  scan: a persistent CTA walks (row group, column tile) tiles; each thread
 //        scans its row's 32 elements in place in shared memory with its
 //        running carry (init[n] at the row's first tile), the CTA stores the
@@ -67,6 +69,7 @@ mv_s1_tiled_kernel(const __grid_constant__ CUtensorMap mapA, const float* __rest
   uint64_t* full = reinterpret_cast<uint64_t*>(base);
   uint64_t* empty = full + stages;
   float* tiles = reinterpret_cast<float*>(base + kS1Header);
+  float* xs = tiles + stages * (R * kS1Cols);  // [stages][32]: the x chunk of each stage
   constexpr int kWarps = R / 32;
   constexpr uint32_t kStageBytes = R * kS1Cols * 4;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -87,8 +90,11 @@ mv_s1_tiled_kernel(const __grid_constant__ CUtensorMap mapA, const float* __rest
       for (int t = 0; t < ntiles; ++t) {
         const int st = t % stages;
         if (t >= stages) mbar_wait(&empty[st], ((t / stages) - 1) & 1);
-        mbar_expect_tx(&full[st], kStageBytes);
+        const int64_t j0 = (int64_t)t * kS1Cols;
+        const uint32_t xb = (uint32_t)((w - j0 < kS1Cols ? w - j0 : kS1Cols) * 4);  // w % 4 == 0
+        mbar_expect_tx(&full[st], kStageBytes + xb);
         tma_load_2d(tiles + st * (R * kS1Cols), &mapA, t * kS1Cols, row0, &full[st]);
+        bulk_load_1d(xs + st * kS1Cols, x + j0, xb, &full[st]);
       }
     }
     return;
@@ -97,19 +103,17 @@ mv_s1_tiled_kernel(const __grid_constant__ CUtensorMap mapA, const float* __rest
   V4<float> acc = {0.f, 0.f, 0.f, 0.f};
   for (int t = 0; t < ntiles; ++t) {
     const int st = t % stages;
-    // x does not depend on the tile: its (broadcast) loads go out before the wait
-    V4<float> xv[8];
     const int64_t j0 = (int64_t)t * kS1Cols;
-#pragma unroll
-    for (int c = 0; c < 8; ++c)
-      xv[c] = j0 + 4 * c < w ? ldg4(x + j0 + 4 * c) : V4<float>{0.f, 0.f, 0.f, 0.f};
     mbar_wait(&full[st], (t / stages) & 1);
     const float* tile = tiles + st * (R * kS1Cols);
+    const float* xt = xs + st * kS1Cols;
 #pragma unroll
     for (int c = 0; c < 8; ++c) {
+      if (j0 + 4 * c >= w) break;  // past the row (the tile is zero there; x's slot is stale)
       const float4 a = *reinterpret_cast<const float4*>(tile + swz128(r, c));
-      acc.x = fmaf(a.x, xv[c].x, acc.x); acc.y = fmaf(a.y, xv[c].y, acc.y);
-      acc.z = fmaf(a.z, xv[c].z, acc.z); acc.w = fmaf(a.w, xv[c].w, acc.w);
+      const float4 xv = *reinterpret_cast<const float4*>(xt + 4 * c);  // broadcast
+      acc.x = fmaf(a.x, xv.x, acc.x); acc.y = fmaf(a.y, xv.y, acc.y);
+      acc.z = fmaf(a.z, xv.z, acc.z); acc.w = fmaf(a.w, xv.w, acc.w);
     }
     __syncwarp();
     if (lane == 0) mbar_arrive(&empty[st]);
@@ -247,8 +251,8 @@ static int launch_mv_s1(const float* A, int64_t lda, const float* x, float* y, i
   const int64_t grid = (h + R - 1) / R;
   const int sms = sm_count();
   const int per_sm = (int)((grid + sms - 1) / sms) < 2 ? 1 : 2;
-  const int stages = s1_stages(per_sm, (size_t)R * kS1Cols * 4);
-  const size_t smem = kS1Header + 1024 + (size_t)stages * R * kS1Cols * 4;
+  const int stages = s1_stages(per_sm, (size_t)R * kS1Cols * 4 + kS1Cols * 4);
+  const size_t smem = kS1Header + 1024 + (size_t)stages * (R * kS1Cols * 4 + kS1Cols * 4);
   auto kern = mv_s1_tiled_kernel<R>;
   if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess)
     return check_launch("mv S=1 tiled smem attribute");

@@ -426,9 +426,18 @@ def test_s1_tiled_baselines_parity():
             assert_exact(got, O.scan(x), what) if exact else assert_rel(got, O.scan(x), L, what)
         x = synth.items(N, L, "i32_full")
         assert_exact(host(C.cudanp_batched_loop_reduce_variant(C.S1_TILED, dev(x))), O.reduce(x), f"reduce tiled {N}x{L}")
-    # preconditions: rows not a multiple of 4 elements -> unsupported, not wrong
+    # preconditions: rows not a multiple of 4 elements, or x off 16-byte
+    # alignment -> unsupported, not wrong
     with pytest.raises(C.CudanpError) as ei:
         C.cudanp_batched_loop_scan_variant(C.S1_TILED, dev(synth.items(10, 7, "i32_small")))
+    assert ei.value.status == C.ERR_UNSUPPORTED
+    A = dev(synth.matrix(40, 104, "f32_int4"))
+    with pytest.raises(C.CudanpError) as ei:
+        C.cudanp_mv_variant(C.S1_TILED, A[:, :101], dev(synth.vector(101, "f32_int4")))
+    assert ei.value.status == C.ERR_UNSUPPORTED
+    xb = torch.zeros(105, device="cuda")
+    with pytest.raises(C.CudanpError) as ei:
+        C.cudanp_mv_variant(C.S1_TILED, A, xb[1:])
     assert ei.value.status == C.ERR_UNSUPPORTED
 
 
