@@ -5,7 +5,8 @@ GPU suite (BASELINE.json north_star):
     (C2, 16384^2 fp32; the measured copy peak of MEASURED_PEAKS.json);
   * it beats both the S=1 (no-NP) kernel and the dynamic-parallelism variant
     at every inner trip count <= 1024 (C3 reduce L = 32..256, C4 scan
-    L = 64..1024, C1 TMV L = 1024).
+    L = 64..1024, C1 TMV L = 1024) -- the S=1 kernels being the LDG ones, the
+    literal and the TMA-tiled one-thread-per-item kernels (CUDANP_IMPL_S1_TILED).
 
 Times are CUDA events on the launching stream, median of several launches,
 inputs > L2 (C1 is timed as a graph of launches over 64 cold copies).  The
@@ -77,12 +78,18 @@ def test_tmv_best_np_reaches_70pct_of_hbm():
     assert gbs >= 0.70 * peak_gbs(), f"TMV {gbs:.0f} GB/s < 70 % of {peak_gbs():.0f}"
 
 
-def _np_vs_s1_dp(run_np, run_s1s, run_dp_block, run_dp_thread_prefix, N, Np, what):
+def _np_vs_s1_dp(run_np, run_s1s, run_dp_block, run_dp_thread_prefix, N, Np, what, run_tiled=None):
+    """NP against the LDG S=1 kernels (>= 1.1x), the TMA-tiled S=1 kernel
+    (the SMM-style "already optimized" baseline: NP must still win) and
+    both DP variants (>= 2x)."""
     t_np = min(t_ms(f) for f in run_np)
     t_s1 = min(t_ms(f) for f in run_s1s)
     t_dpb = t_ms(run_dp_block, reps=3, warm=1)
     t_dpt = t_ms(run_dp_thread_prefix, reps=3, warm=1) * N / Np
     assert t_s1 / t_np >= 1.1, f"{what}: NP {t_np:.3f} ms vs S=1 {t_s1:.3f} ms"
+    if run_tiled is not None:
+        t_t = t_ms(run_tiled)
+        assert t_t / t_np >= 1.0, f"{what}: NP {t_np:.3f} ms vs tiled S=1 {t_t:.3f} ms"
     assert t_dpb / t_np >= 2.0, f"{what}: NP {t_np:.3f} ms vs DP per CTA {t_dpb:.3f} ms"
     assert t_dpt / t_np >= 2.0, f"{what}: NP {t_np:.3f} ms vs DP per thread {t_dpt:.3f} ms (scaled)"
 
@@ -98,7 +105,8 @@ def test_reduce_np_beats_s1_and_dp(L):
     s1.append(lambda: C.cudanp_batched_loop_reduce_variant(C.S1_LITERAL, x, None, out))
     _np_vs_s1_dp(np_, s1, lambda: C.cudanp_batched_loop_reduce_variant(C.DP_BLOCK, x, None, out),
                  lambda: C.cudanp_batched_loop_reduce_variant(C.DP_THREAD, x[:Np], None, out[:Np]),
-                 N, Np, f"C3 reduce L={L}")
+                 N, Np, f"C3 reduce L={L}",
+                 run_tiled=lambda: C.cudanp_batched_loop_reduce_variant(C.S1_TILED, x, None, out))
 
 
 @pytest.mark.parametrize("L", [64, 1024])
@@ -112,7 +120,8 @@ def test_scan_np_beats_s1_and_dp(L):
     s1.append(lambda: C.cudanp_batched_loop_scan_variant(C.S1_LITERAL, x, None, out))
     _np_vs_s1_dp(np_, s1, lambda: C.cudanp_batched_loop_scan_variant(C.DP_BLOCK, x, None, out),
                  lambda: C.cudanp_batched_loop_scan_variant(C.DP_THREAD, x[:Np], None, out[:Np]),
-                 N, Np, f"C4 scan L={L}")
+                 N, Np, f"C4 scan L={L}",
+                 run_tiled=lambda: C.cudanp_batched_loop_scan_variant(C.S1_TILED, x, None, out))
     del x, out
     torch.cuda.empty_cache()
 
