@@ -39,18 +39,24 @@ METRICS = [
 CASES = [
     ("C1 TMV 1024²", "S=1 inter (no NP)", "--op tmv --n 1024 --S 1 --dist cyclic --map inter", "tmv_"),
     ("C1 TMV 1024²", "literal Fig 2", "--op tmv_literal --n 1024", "tmv_"),
+    ("C1 TMV 1024²", "S=1 TMA (no NP)", "--op tmv --n 1024 --S 1 --dist cyclic --map inter_tma", "tmv_"),
     ("C1 TMV 1024²", "NP S=32 cyclic inter", "--op tmv --n 1024 --S 32 --dist cyclic --map inter", "tmv_"),
+    ("C1 TMV 1024²", "NP S=64 block inter", "--op tmv --n 1024 --S 64 --dist block --map inter", "tmv_"),
     ("C2 MV 16384²", "S=1 inter (no NP)", "--op mv --S 1 --dist cyclic --map inter", "mv_"),
     ("C2 MV 16384²", "literal", "--op mv_literal", "mv_"),
+    ("C2 MV 16384²", "S=1 TMA-tiled (no NP; SMM-style)", "--op mv_tiled", "mv_"),
     ("C2 MV 16384²", "NP S=32 cyclic intra", "--op mv --S 32 --dist cyclic --map intra", "mv_"),
+    ("C2 MV 16384²", "NP S=256 cyclic (multi-warp)", "--op mv --S 256 --dist cyclic --map intra", "mv_"),
     ("C2 TMV 16384²", "S=1 inter LDG (no NP)", "--op tmv --S 1 --dist cyclic --map inter", "tmv_"),
     ("C2 TMV 16384²", "S=1 TMA (no NP)", "--op tmv --S 1 --dist cyclic --map inter_tma", "tmv_"),
     ("C2 TMV 16384²", "NP S=8 block TMA", "--op tmv --S 8 --dist block --map inter_tma", "tmv_"),
     ("C3 reduce 4M×256", "S=1 inter (no NP)", "--op reduce --L 256 --S 1 --dist block --map inter", "reduce_"),
     ("C3 reduce 4M×256", "literal", "--op reduce_literal --L 256", "reduce_"),
+    ("C3 reduce 4M×256", "S=1 TMA-tiled (no NP)", "--op reduce_tiled --L 256", "reduce_"),
     ("C3 reduce 4M×256", "NP S=32 block intra", "--op reduce --L 256 --S 32 --dist block --map intra", "reduce_"),
     ("C4 scan 2M×256 i32", "S=1 inter (no NP)", "--op scan --N 2097152 --L 256 --dtype i32 --S 1 --dist block --map inter", "scan_"),
     ("C4 scan 2M×256 i32", "literal", "--op scan_literal --N 2097152 --L 256 --dtype i32", "scan_"),
+    ("C4 scan 2M×256 i32", "S=1 TMA-tiled (no NP)", "--op scan_tiled --N 2097152 --L 256 --dtype i32", "scan_"),
     ("C4 scan 2M×256 i32", "NP S=16 cyclic intra", "--op scan --N 2097152 --L 256 --dtype i32 --S 16 --dist cyclic --map intra", "scan_"),
     ("F2 LE 2M×150 item-major", "literal Fig 5", "--op le_literal --N 2097152 --L 150 --layout 0", "le_"),
     ("F2 LE 2M×150 item-major", "S=1 intra (no NP)", "--op le --N 2097152 --L 150 --layout 0 --S 1 --dist cyclic --map intra", "le_"),
