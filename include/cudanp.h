@@ -258,9 +258,8 @@ int cudanp_le_gicov_literal(const float* in, float* gicov, float* ave, float* va
  *   CUDANP_IMPL_S1_TILED  : the tuned no-NP baseline -- one thread per item
  *       (S = 1) whose rows reach it through shared-memory tiles copied by TMA
  *       (the "already optimized" SMM-style baseline of P:411 / Table 1):
- *       MV and scan (np_s1_tiled.cu; scan tiles are stored back by TMA), TMV
- *       (= cudanp_tmv_tma with S = 1), reduce (= cudanp_batched_loop_reduce_tma
- *       with S = 1).  Needs 16-byte aligned operands with rows a multiple of
+ *       MV, reduce and scan (np_s1_tiled.cu; scan tiles are stored back by
+ *       TMA), TMV (= cudanp_tmv_tma with S = 1).  Needs 16-byte aligned operands with rows a multiple of
  *       4 elements (and sizes < 2^31), else CUDANP_ERR_UNSUPPORTED.
  * DP variants need enough device-runtime launch slots: see
  * cudanp_dp_set_pending_launch_limit.  A DP launch that the device runtime

@@ -47,6 +47,7 @@ int le_tma(const float*, float*, float*, float*, float*, int64_t, int64_t, float
            cudaStream_t);
 int mv_s1_tiled(const float*, int64_t, const float*, float*, int64_t, int64_t, cudaStream_t);
 int scan_s1_tiled(const void*, const void*, void*, int64_t, int64_t, int, cudaStream_t);
+int reduce_s1_tiled(const void*, const void*, void*, int64_t, int64_t, int, int, cudaStream_t);
 int le_literal(const float*, float*, float*, float*, float*, int64_t, int64_t, float, int,
                cudaStream_t);
 
@@ -664,8 +665,12 @@ int cudanp_batched_loop_reduce_variant(int impl, const void* in, const void* ini
   if (rc) return rc;
   if (impl == CUDANP_IMPL_S1_LITERAL)
     return reduce_literal(in, init, out, n_outer, n_inner, dtype, op, as_stream(stream));
-  if (impl == CUDANP_IMPL_S1_TILED)
-    return cudanp_batched_loop_reduce_tma(in, init, out, n_outer, n_inner, dtype, op, 1, 0, 0, 0, stream);
+  if (impl == CUDANP_IMPL_S1_TILED) {
+    if (n_outer > 0 && n_inner == 0)  // nothing to stream: init / the identity
+      return reduce_np(in, init, out, n_outer, 0, dtype, op, 1, 0, MAP_INTRA, false, as_stream(stream), nullptr);
+    if (n_outer > 0 && !tiled_ok(in, n_inner, nullptr, n_outer, n_inner)) return tiled_unsupported();
+    return reduce_s1_tiled(in, init, out, n_outer, n_inner, dtype, op, as_stream(stream));
+  }
   return dp_reduce(impl == CUDANP_IMPL_DP_BLOCK, in, init, out, n_outer, n_inner, dtype, op,
                    as_stream(stream));
 }

@@ -20,6 +20,9 @@
 //        barrier) -- into the ring; each consumer thread accumulates its row
 //        (acc += A[r][j]*x[j], x read from shared memory as a broadcast) and
 //        stores y[r].
+//  reduce: the same walk; each thread folds its row's elements of every tile
+//        (sum or max) and the master -- the thread itself -- applies init[n]
+//        and stores out[n] at the row's last tile.
 //  scan: a persistent CTA walks (row group, column tile) tiles; each thread
 //        scans its row's 32 elements in place in shared memory with its
 //        running carry (init[n] at the row's first tile), the CTA stores the
@@ -192,6 +195,70 @@ scan_s1_tiled_kernel(const __grid_constant__ CUtensorMap mapIn, const __grid_con
   if (r == 0) bulk_wait_all();  // stores done before the CTA's shared memory goes away
 }
 
+// ---------------------------------------------------------------- reduce, S = 1
+// Stage s is refilled (tile t + stages) once every thread has passed tile t's
+// barrier; columns past L (zero-filled by TMA) are skipped, so max sees only
+// the row's own elements.
+template <class T, class Op, int R>
+__global__ void __launch_bounds__(R, 1)
+reduce_s1_tiled_kernel(const __grid_constant__ CUtensorMap mapIn, const T* __restrict__ init,
+                       T* __restrict__ out, int64_t N, int64_t L, int stages) {
+  pdl_entry();
+  extern __shared__ __align__(1024) unsigned char smem_raw[];
+  unsigned char* base = smem_raw + ((1024 - (smem_u32(smem_raw) & 1023)) & 1023);
+  uint64_t* full = reinterpret_cast<uint64_t*>(base);
+  const T* tiles = reinterpret_cast<const T*>(base + kS1Header);
+  constexpr uint32_t kStageBytes = R * kS1Cols * 4;
+  const int r = threadIdx.x;
+  const int64_t ngroups = (N + R - 1) / R;
+  const int nk = (int)((L + kS1Cols - 1) / kS1Cols);
+  const int64_t mygroups = blockIdx.x < ngroups ? (ngroups - 1 - blockIdx.x) / gridDim.x + 1 : 0;
+  const int64_t ntiles = mygroups * nk;
+  auto coords = [&](int64_t t, int& col, int& row) {
+    const int64_t g = blockIdx.x + (t / nk) * gridDim.x;
+    col = (int)(t % nk) * kS1Cols;
+    row = (int)(g * R);
+  };
+  if (r == 0) {
+    for (int i = 0; i < stages; ++i) mbar_init(&full[i], 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    for (int64_t t = 0; t < stages && t < ntiles; ++t) {
+      int col, row;
+      coords(t, col, row);
+      mbar_expect_tx(&full[t], kStageBytes);
+      tma_load_2d(const_cast<T*>(tiles) + t * (R * kS1Cols), &mapIn, col, row, &full[t]);
+    }
+  }
+  __syncthreads();
+  const T id = Op::template identity<T>();
+  T acc = id;
+  for (int64_t t = 0; t < ntiles; ++t) {
+    const int st = (int)(t % stages);
+    int col, row;
+    coords(t, col, row);
+    mbar_wait(&full[st], (uint32_t)(t / stages) & 1);
+    const T* tile = tiles + st * (R * kS1Cols);
+#pragma unroll
+    for (int c = 0; c < 8; ++c) {
+      if (col + 4 * c >= L) break;
+      const V4<T> v = *reinterpret_cast<const V4<T>*>(tile + swz128(r, c));
+      acc = Op::apply(acc, Op::apply(Op::apply(v.x, v.y), Op::apply(v.z, v.w)));
+    }
+    if (col + kS1Cols >= L) {  // the row's last tile: the master finishes the item
+      const int64_t n = (int64_t)row + r;
+      if (n < N) out[n] = init ? Op::apply(init[n], acc) : acc;
+      acc = id;
+    }
+    __syncthreads();  // every thread is done with stage st
+    if (r == 0 && t + stages < ntiles) {
+      int c2, r2;
+      coords(t + stages, c2, r2);
+      mbar_expect_tx(&full[st], kStageBytes);
+      tma_load_2d(const_cast<T*>(tiles) + st * (R * kS1Cols), &mapIn, c2, r2, &full[st]);
+    }
+  }
+}
+
 // ---------------------------------------------------------------- host side
 typedef CUresult (*EncodeTiledFnS1)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*,
                                     const cuuint64_t*, const cuuint64_t*, const cuuint32_t*,
@@ -290,6 +357,35 @@ static int launch_scan_s1(const T* in, const T* init, T* out, int64_t N, int64_t
   const int64_t grid = persistent_grid(kern, R, smem, groups);
   launch_pdl(kern, dim3((unsigned)grid), dim3(R), smem, st, mi, mo, init, N, L, stages);
   return check_launch("scan S=1 tiled launch");
+}
+
+template <class T, class Op>
+static int launch_reduce_s1(const T* in, const T* init, T* out, int64_t N, int64_t L, cudaStream_t st) {
+  constexpr int R = 128;
+  CUtensorMap mi;
+  if (int rc = encode_s1(&mi, in, N, L, L, R)) return rc;
+  constexpr int kPerSM = 2;
+  const int stages = s1_stages(kPerSM, (size_t)R * kS1Cols * 4);
+  const size_t smem = kS1Header + 1024 + (size_t)stages * R * kS1Cols * 4;
+  auto kern = reduce_s1_tiled_kernel<T, Op, R>;
+  if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess)
+    return check_launch("reduce S=1 tiled smem attribute");
+  const int64_t grid = persistent_grid(kern, R, smem, (N + R - 1) / R);
+  launch_pdl(kern, dim3((unsigned)grid), dim3(R), smem, st, mi, init, out, N, L, stages);
+  return check_launch("reduce S=1 tiled launch");
+}
+
+// Loop-reduce with one thread per item, rows staged by TMA (needs `in`
+// 16-byte aligned, L % 4 == 0, sizes < 2^31; the ABI checks).  L = 0 is the
+// caller's (the NP path writes init / the identity).
+int reduce_s1_tiled(const void* in, const void* init, void* out, int64_t N, int64_t L, int dtype,
+                    int op, cudaStream_t st) {
+  if (N == 0) return CUDANP_OK;
+  if (dtype == CUDANP_F32)
+    return op == CUDANP_SUM ? launch_reduce_s1<float, OpSum>((const float*)in, (const float*)init, (float*)out, N, L, st)
+                            : launch_reduce_s1<float, OpMax>((const float*)in, (const float*)init, (float*)out, N, L, st);
+  return op == CUDANP_SUM ? launch_reduce_s1<int32_t, OpSum>((const int32_t*)in, (const int32_t*)init, (int32_t*)out, N, L, st)
+                          : launch_reduce_s1<int32_t, OpMax>((const int32_t*)in, (const int32_t*)init, (int32_t*)out, N, L, st);
 }
 
 // Inclusive scan with one thread per item, rows staged (and stored) by TMA

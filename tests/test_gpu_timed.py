@@ -424,8 +424,18 @@ def test_s1_tiled_baselines_parity():
             assert_exact(got, ref, what) if exact else assert_rel(got, ref, L, what)
             got = host(C.cudanp_batched_loop_scan_variant(C.S1_TILED, dev(x)))
             assert_exact(got, O.scan(x), what) if exact else assert_rel(got, O.scan(x), L, what)
-        x = synth.items(N, L, "i32_full")
-        assert_exact(host(C.cudanp_batched_loop_reduce_variant(C.S1_TILED, dev(x))), O.reduce(x), f"reduce tiled {N}x{L}")
+        for kind, op in (("i32_full", C.SUM), ("i32_full", C.MAX), ("f32_signed", C.MAX), ("f32_int4", C.SUM)):
+            x = synth.items(N, L, kind, seed=L)
+            ini = synth.init(N, kind, seed=L)
+            # max over all-negative-capable data: the zero-filled columns past L
+            # must not take part
+            assert_exact(host(C.cudanp_batched_loop_reduce_variant(C.S1_TILED, dev(x), op=op)),
+                         O.reduce(x, op=op), f"reduce tiled {kind} op={op} {N}x{L}")
+            assert_exact(host(C.cudanp_batched_loop_reduce_variant(C.S1_TILED, dev(x), dev(ini), op=op)),
+                         O.reduce(x, op=op, init=ini), f"reduce tiled init {kind} op={op} {N}x{L}")
+        xu = synth.items(N, L, "f32_unit", seed=L)
+        assert_rel(host(C.cudanp_batched_loop_reduce_variant(C.S1_TILED, dev(xu))), O.reduce(xu), L,
+                   f"reduce tiled f32_unit {N}x{L}")
     # preconditions: rows not a multiple of 4 elements, or x off 16-byte
     # alignment -> unsupported, not wrong
     with pytest.raises(C.CudanpError) as ei:
