@@ -61,11 +61,12 @@ def parse():
     ap.add_argument("--no-sweep", action="store_true",
                     help="skip the autotune sweep and comparisons (for ncu launch lists); "
                          "use --tmv-cfg / --mv-cfg")
-    ap.add_argument("--gather", choices=["nccl", "fused", "native"], default="nccl",
+    ap.add_argument("--gather", choices=["auto", "nccl", "fused", "native"], default="auto",
                     help="N > 1: gather outputs to rank 0 with NCCL send/recv through "
                          "torch.distributed, fused into the kernels' master stores through CUDA IPC "
                          "over NVLink (SURVEY f4), or with the library's own NCCL group "
-                         "(cudanp_group_gather)")
+                         "(cudanp_group_gather); auto = fused when every rank can map rank 0's "
+                         "buffers, else nccl")
     ap.add_argument("--tmv-cfg", default="8,cyclic,inter_tma")
     ap.add_argument("--mv-cfg", default="256,cyclic,intra")
     ap.add_argument("--no-c5", action="store_true", help="skip the C5 strong-scaling block")
@@ -314,14 +315,22 @@ def run_cudanp(args):
     y_root = torch.empty(n * world, dtype=torch.float32, device="cuda") if rank == 0 else None
     ym_root = torch.empty(n * world, dtype=torch.float32, device="cuda") if rank == 0 else None
 
-    fused = world > 1 and args.gather == "fused"
+    fused = world > 1 and args.gather in ("fused", "auto")
     native = P.NativeGroup(rank, world) if world > 1 and args.gather == "native" else None
     if fused:
         fg_t = P.FusedGather(y_root, n * world, rank, world)
         fg_m = P.FusedGather(ym_root, n * world, rank, world)
+        if not P.FusedGather.all_ok([fg_t, fg_m], world):
+            if args.gather == "fused":
+                raise SystemExit(f"--gather fused: CUDA IPC unavailable ({fg_t.error or fg_m.error})")
+            fg_t.close()
+            fg_m.close()
+            fused = False   # auto: fall back to the NCCL send/recv gather
+    if fused:
         out_t, out_m = fg_t.out_ptr(), fg_m.out_ptr()
     else:
         out_t, out_m = y_t, y_m
+    gather_used = ("fused" if fused else ("native" if native else "nccl")) if world > 1 else "none"
 
     def step(evs=None):
         if evs:
@@ -419,7 +428,7 @@ def run_cudanp(args):
     if not args.no_c5:
         del A_t, A_m, x_t, x_m, y_t, y_m
         torch.cuda.empty_cache()
-        c5 = run_c5(C, P, rank, world, args.c5_steps, args.gather)
+        c5 = run_c5(C, P, rank, world, args.c5_steps, gather_used if world > 1 else "none")
 
     if rank != 0:
         if world > 1:
@@ -484,10 +493,11 @@ def run_cudanp(args):
             "tmv": {"S": St, "dist": "cyclic" if dt == 0 else "block", "map": MAPN[mt]},
             "mv": {"S": Sm, "dist": "cyclic" if dm == 0 else "block", "map": MAPN[mm]},
             "parallelism": (f"dp{world}: contiguous outer-item shards + "
-                            + ("gather fused into the master stores (CUDA IPC over NVLink)"
-                               if fused else "NCCL send/recv gather to rank 0"
+                            + ("gather fused into the master stores (CUDA IPC over NVLink; no "
+                               "collective kernel)" if fused else "NCCL send/recv gather to rank 0"
                                + (" (library group, cudanp_group_gather)" if native else "")))
                            if world > 1 else "single GPU",
+            "gather": gather_used,
             "l2": "no flush: each matrix is 1 GiB > 126 MB L2",
             "step": "cudanp_tmv + cudanp_mv (+ gather when n_gpus > 1)",
         },
@@ -570,6 +580,10 @@ def run_c5(C, P, rank, world, steps, gather_mode):
         root = torch.empty(total, dtype=torch.float32, device="cuda") if rank == 0 else None
         y = root if world == 1 else torch.empty(e - b, dtype=torch.float32, device="cuda")
         fg = P.FusedGather(root, total, rank, world) if fused else None
+        if fg is not None and not P.FusedGather.all_ok([fg], world):
+            fg.close()
+            fg, fused = None, False  # fall back to the NCCL send/recv gather
+            out["gather"] = "nccl (CUDA IPC unavailable)"
         dst = fg.out_ptr() if fused else y
 
         def kernel(S, d, m, o=None):

@@ -74,18 +74,44 @@ class FusedGather:
         import torch.distributed as dist
         self.rank, self.world, self.root = rank, world, root
         self.begin, self.end = shard(n_total, world, rank)
+        self.mapped, self.error = None, None
         obj = [None]
         if rank == root:
-            obj = [C.cudanp_ipc_get_handle(root_buf)]
             self.base = root_buf.data_ptr()
+            try:
+                obj = [C.cudanp_ipc_get_handle(root_buf)]
+            except C.CudanpError as e:  # every rank still joins the broadcast
+                self.error = str(e)
         dist.broadcast_object_list(obj, src=root)
-        self.handle, self.offset = obj[0]
-        if rank != root:
-            self.mapped = C.cudanp_ipc_open(self.handle, self.offset)
-            self.base = self.mapped
+        if obj[0] is None:
+            self.error = self.error or "rank 0 could not export its buffer"
+            self.handle, self.offset = None, 0
         else:
-            self.mapped = None
+            self.handle, self.offset = obj[0]
+        if rank != root and self.handle is not None:
+            try:
+                self.mapped = C.cudanp_ipc_open(self.handle, self.offset)
+                self.base = self.mapped
+            except C.CudanpError as e:
+                self.error = str(e)
         self.elem_bytes = elem_bytes
+
+    @property
+    def ok(self) -> bool:
+        """This rank can store into rank 0's buffer (collective agreement is
+        the caller's: see all_ok)."""
+        return self.error is None
+
+    @staticmethod
+    def all_ok(gathers, world: int) -> bool:
+        """True when every rank opened every buffer (an all-reduce MIN)."""
+        import torch
+        import torch.distributed as dist
+        flag = 1.0 if all(g.ok for g in gathers) else 0.0
+        dev = "cuda" if dist.get_backend() == "nccl" else "cpu"
+        t = torch.tensor([flag], device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MIN)
+        return bool(t.item() > 0)
 
     def out_ptr(self) -> int:
         return self.base + self.begin * self.elem_bytes
