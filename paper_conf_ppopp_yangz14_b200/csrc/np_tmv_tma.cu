@@ -188,103 +188,6 @@ tmv_tma_kernel(const __grid_constant__ CUtensorMap mapA, const float* __restrict
   }
 }
 
-// ---------------------------------------------------------------- S = 32, block: per-slave rings
-// With 32 slave warps a CTA has no room for a producer warp, and one thread
-// refilling 32 boxes per stage for everyone serialises the ring (4.9 TB/s
-// on C2).  With the block distribution each slave streams its own contiguous
-// chunk, so each slave warp runs its own ring: lane 0 issues the boxes of its
-// chunk [s*c, (s+1)*c) (RK rows x COLS columns each) into D private stages,
-// the warp consumes a stage and lane 0 refills it with the chunk's next box
-// right away -- no cross-warp barrier until the team reduction.
-template <int COLS, int RK>
-__global__ void __launch_bounds__(1024, 1)
-tmv_tma_slave_ring_kernel(const __grid_constant__ CUtensorMap mapA, const float* __restrict__ x,
-                          float* __restrict__ y, int64_t w, int64_t h, int D) {
-  pdl_entry();
-  constexpr int S = 32;
-  constexpr int V = COLS / 32;
-  constexpr uint32_t kBoxBytes = RK * COLS * 4;
-  extern __shared__ __align__(128) unsigned char smem_raw[];
-  uint64_t* full = reinterpret_cast<uint64_t*>(smem_raw);  // [S][D]
-  float* tiles = reinterpret_cast<float*>(smem_raw + 128 * ((8 * S * D + 127) / 128));  // [S][D][RK][COLS]
-  float* red = tiles;  // [S][COLS], reused after the loop
-  const int lane = threadIdx.x & 31, s = threadIdx.x >> 5;
-  const int col0 = blockIdx.x * COLS;
-  const int64_t c = (h + S - 1) / S;  // rows per slave chunk (R5)
-  const int ntiles = (int)((c + RK - 1) / RK);
-  uint64_t* fb = full + s * D;
-  float* ring = tiles + (size_t)s * D * RK * COLS;
-  if (lane == 0) {
-    for (int i = 0; i < D; ++i) mbar_init(&fb[i], 1);
-    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    for (int t = 0; t < D && t < ntiles; ++t) {
-      mbar_expect_tx(&fb[t], kBoxBytes);
-      tma_load_2d(ring + t * RK * COLS, &mapA, col0, (int)(s * c + (int64_t)t * RK), &fb[t]);
-    }
-  }
-  __syncwarp();
-  V4<float> acc = {0.f, 0.f, 0.f, 0.f};
-  for (int t = 0; t < ntiles; ++t) {
-    const int st = t % D;
-    float xs[RK];
-    const bool whole = (int64_t)(t + 1) * RK <= c && s * c + (int64_t)(t + 1) * RK <= h;
-#pragma unroll
-    for (int kk = 0; kk < RK; ++kk) {
-      const int64_t k = (int64_t)t * RK + kk, row = s * c + k;
-      xs[kk] = (k < c && row < h) ? __ldg(x + row) : 0.f;
-    }
-    mbar_wait(&fb[st], (t / D) & 1);
-    const float* tile = ring + st * RK * COLS;
-#pragma unroll
-    for (int kk = 0; kk < RK; ++kk) {
-      if (!whole) {  // ragged last box: rows past the chunk (next slave's) or past h are skipped
-        const int64_t k = (int64_t)t * RK + kk;
-        if (!(k < c && s * c + k < h)) continue;
-      }
-      const float xv = xs[kk];
-      const float* ap = tile + kk * COLS + lane * V;
-      if constexpr (V == 4) {
-        const float4 a = *reinterpret_cast<const float4*>(ap);
-        acc.x = fmaf(a.x, xv, acc.x); acc.y = fmaf(a.y, xv, acc.y);
-        acc.z = fmaf(a.z, xv, acc.z); acc.w = fmaf(a.w, xv, acc.w);
-      } else if constexpr (V == 2) {
-        const float2 a = *reinterpret_cast<const float2*>(ap);
-        acc.x = fmaf(a.x, xv, acc.x); acc.y = fmaf(a.y, xv, acc.y);
-      } else {
-        acc.x = fmaf(*ap, xv, acc.x);
-      }
-    }
-    __syncwarp();  // the whole warp is done with this stage: refill it
-    if (lane == 0 && t + D < ntiles) {
-      mbar_expect_tx(&fb[st], kBoxBytes);
-      tma_load_2d(ring + st * RK * COLS, &mapA, col0, (int)(s * c + (int64_t)(t + D) * RK), &fb[st]);
-    }
-  }
-  // Team reduction through shared memory (the rings are free once every
-  // slave is past its last box); the master warp folds in slave order.
-  __syncthreads();
-  {
-    float* rr = red + s * COLS + lane * V;
-    const float av[4] = {acc.x, acc.y, acc.z, acc.w};
-#pragma unroll
-    for (int v = 0; v < V; ++v) rr[v] = av[v];
-  }
-  __syncthreads();
-  if (s == 0) {
-    const int64_t col = col0 + lane * V;
-    float sum[4] = {0.f, 0.f, 0.f, 0.f};
-#pragma unroll
-    for (int k = 0; k < S; ++k) {
-      const float* p = red + k * COLS + lane * V;
-#pragma unroll
-      for (int v = 0; v < V; ++v) sum[v] += p[v];
-    }
-#pragma unroll
-    for (int v = 0; v < V; ++v)
-      if (col + v < w) y[col + v] = sum[v];
-  }
-}
-
 // ---------------------------------------------------------------- host side
 typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*,
                                   const cuuint64_t*, const cuuint64_t*, const cuuint32_t*,
@@ -343,56 +246,6 @@ static int launch_tmv_tma_s(const float* A, int64_t lda, const float* x, float* 
     return check_launch("tmv_tma smem attribute");
   launch_pdl(kern, dim3(grid), dim3(TmaThreads<S>::value), smem, st, map, x, y, w, h, stages);
   return check_launch("tmv_tma launch");
-}
-
-// S = 32 block: per-slave rings.  COLS as wide as keeps >= 0.8 x SMs strips
-// (else narrower), RK rows per box and D stages per slave sized to ~200 KB.
-template <int COLS, int RK>
-static int launch_tmv_slave_ring(const float* A, int64_t lda, const float* x, float* y, int64_t w,
-                                 int64_t h, cudaStream_t st, LaunchInfo* info) {
-  constexpr int S = 32;
-  const size_t box = (size_t)RK * COLS * 4;
-  int D = (int)((200 * 1024) / (S * box));
-  if (D > 8) D = 8;
-  const size_t smem = 128 * ((8 * S * (size_t)D + 127) / 128) + (size_t)S * D * box;
-  auto kern = tmv_tma_slave_ring_kernel<COLS, RK>;
-  const unsigned grid = (unsigned)((w + COLS - 1) / COLS);
-  if (info) {
-    info->block_threads = 32 * S; info->grid = grid; info->smem = (int)smem; info->map = MAP_INTER;
-    kernel_attrs(kern, &info->regs, nullptr);
-    return CUDANP_OK;
-  }
-  EncodeTiledFn enc = encode_fn();
-  if (!enc) {
-    set_error("cuTensorMapEncodeTiled entry point unavailable");
-    return CUDANP_ERR_CUDA;
-  }
-  CUtensorMap map;
-  const cuuint64_t dims[2] = {(cuuint64_t)w, (cuuint64_t)h};
-  const cuuint64_t strides[1] = {(cuuint64_t)lda * 4};
-  const cuuint32_t boxd[2] = {(cuuint32_t)COLS, (cuuint32_t)RK};
-  const cuuint32_t estr[2] = {1, 1};
-  CUresult r = enc(&map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, (void*)A, dims, strides, boxd, estr,
-                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
-                   CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
-  if (r != CUDA_SUCCESS) {
-    set_error("cuTensorMapEncodeTiled failed (%d)", (int)r);
-    return CUDANP_ERR_CUDA;
-  }
-  if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess)
-    return check_launch("tmv_tma (per-slave rings) smem attribute");
-  launch_pdl(kern, dim3(grid), dim3(32 * S), smem, st, map, x, y, w, h, D);
-  return check_launch("tmv_tma (per-slave rings) launch");
-}
-
-static int tmv_tma_s32_block(const float* A, int64_t lda, const float* x, float* y, int64_t w,
-                             int64_t h, int cols_req, cudaStream_t st, LaunchInfo* info) {
-  const int64_t sms = sm_count();
-  int cols = cols_req;
-  if (!cols) cols = (w + 127) / 128 * 5 >= sms * 4 ? 128 : ((w + 63) / 64 * 5 >= sms * 4 ? 64 : 32);
-  if (cols == 128) return launch_tmv_slave_ring<128, 4>(A, lda, x, y, w, h, st, info);
-  if (cols == 64) return launch_tmv_slave_ring<64, 8>(A, lda, x, y, w, h, st, info);
-  return launch_tmv_slave_ring<32, 8>(A, lda, x, y, w, h, st, info);
 }
 
 // Shared memory of one SM that resident CTAs can take (B200: 228 KB per SM,
@@ -483,10 +336,6 @@ int tmv_tma(const float* A, int64_t lda, const float* x, float* y, int64_t w, in
   if (!(cols == 0 || cols == 32 || cols == 64 || cols == 128)) return fail_invalid("tma cols");
   if (rk_sel < -1 || rk_sel > 2) return fail_invalid("tma rows-per-slave selector");
   if (stages < 0 || stages > 64) return fail_invalid("tma stages");
-  // S = 32, block, automatic shape: per-slave rings (a pinned rows/stages
-  // shape keeps the shared-ring kernel for the A/B)
-  if (S == 32 && dist == DIST_BLOCK && rk_sel < 0 && stages == 0)
-    return tmv_tma_s32_block(A, lda, x, y, w, h, cols, st, info);
   CUDANP_DISPATCH_S(S, {
     return dist == DIST_CYCLIC
                ? tmv_tma_dispatch<kS, DIST_CYCLIC>(A, lda, x, y, w, h, cols, rk_sel, stages, st, info)
