@@ -15,11 +15,10 @@
 // the NP speedups (CUDANP_IMPL_S1_TILED); the method (one master, no slaves)
 // is the literal Fig 2 loop.
 //
-//  MV:   a CTA owns R rows; a producer warp streams the column tiles -- and
-//        the matching 128-byte chunk of x (a 1-D bulk copy on the same
-//        barrier) -- into the ring; each consumer thread accumulates its row
-//        (acc += A[r][j]*x[j], x read from shared memory as a broadcast) and
-//        stores y[r].
+//  MV:   a CTA owns R rows; a producer warp streams the column tiles into
+//        the ring; each consumer thread accumulates its row (acc += A[r][j] *
+//        x[j]; x's 128-byte chunk is a broadcast load issued one tile ahead,
+//        so its L2 latency hides behind the previous tile) and stores y[r].
 //  reduce: the same walk; each thread folds its row's elements of every tile
 //        (sum or max) and the master -- the thread itself -- applies init[n]
 //        and stores out[n] at the row's last tile.
@@ -72,7 +71,6 @@ mv_s1_tiled_kernel(const __grid_constant__ CUtensorMap mapA, const float* __rest
   uint64_t* full = reinterpret_cast<uint64_t*>(base);
   uint64_t* empty = full + stages;
   float* tiles = reinterpret_cast<float*>(base + kS1Header);
-  float* xs = tiles + stages * (R * kS1Cols);  // [stages][32]: the x chunk of each stage
   constexpr int kWarps = R / 32;
   constexpr uint32_t kStageBytes = R * kS1Cols * 4;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -93,31 +91,35 @@ mv_s1_tiled_kernel(const __grid_constant__ CUtensorMap mapA, const float* __rest
       for (int t = 0; t < ntiles; ++t) {
         const int st = t % stages;
         if (t >= stages) mbar_wait(&empty[st], ((t / stages) - 1) & 1);
-        const int64_t j0 = (int64_t)t * kS1Cols;
-        const uint32_t xb = (uint32_t)((w - j0 < kS1Cols ? w - j0 : kS1Cols) * 4);  // w % 4 == 0
-        mbar_expect_tx(&full[st], kStageBytes + xb);
+        mbar_expect_tx(&full[st], kStageBytes);
         tma_load_2d(tiles + st * (R * kS1Cols), &mapA, t * kS1Cols, row0, &full[st]);
-        bulk_load_1d(xs + st * kS1Cols, x + j0, xb, &full[st]);
       }
     }
     return;
   }
   const int r = threadIdx.x;
   V4<float> acc = {0.f, 0.f, 0.f, 0.f};
+  auto load_x = [&](int t, V4<float>* xv) {  // x chunk of tile t (zeros past w)
+    const int64_t j0 = (int64_t)t * kS1Cols;
+#pragma unroll
+    for (int c = 0; c < 8; ++c)
+      xv[c] = j0 + 4 * c < w ? ldg4(x + j0 + 4 * c) : V4<float>{0.f, 0.f, 0.f, 0.f};
+  };
+  V4<float> xcur[8], xnext[8];
+  load_x(0, xcur);
   for (int t = 0; t < ntiles; ++t) {
     const int st = t % stages;
-    const int64_t j0 = (int64_t)t * kS1Cols;
+    if (t + 1 < ntiles) load_x(t + 1, xnext);
     mbar_wait(&full[st], (t / stages) & 1);
     const float* tile = tiles + st * (R * kS1Cols);
-    const float* xt = xs + st * kS1Cols;
 #pragma unroll
     for (int c = 0; c < 8; ++c) {
-      if (j0 + 4 * c >= w) break;  // past the row (the tile is zero there; x's slot is stale)
-      const float4 a = *reinterpret_cast<const float4*>(tile + swz128(r, c));
-      const float4 xv = *reinterpret_cast<const float4*>(xt + 4 * c);  // broadcast
-      acc.x = fmaf(a.x, xv.x, acc.x); acc.y = fmaf(a.y, xv.y, acc.y);
-      acc.z = fmaf(a.z, xv.z, acc.z); acc.w = fmaf(a.w, xv.w, acc.w);
+      const float4 a = *reinterpret_cast<const float4*>(tile + swz128(r, c));  // zero past w
+      acc.x = fmaf(a.x, xcur[c].x, acc.x); acc.y = fmaf(a.y, xcur[c].y, acc.y);
+      acc.z = fmaf(a.z, xcur[c].z, acc.z); acc.w = fmaf(a.w, xcur[c].w, acc.w);
     }
+#pragma unroll
+    for (int c = 0; c < 8; ++c) xcur[c] = xnext[c];
     __syncwarp();
     if (lane == 0) mbar_arrive(&empty[st]);
   }
@@ -318,8 +320,8 @@ static int launch_mv_s1(const float* A, int64_t lda, const float* x, float* y, i
   const int64_t grid = (h + R - 1) / R;
   const int sms = sm_count();
   const int per_sm = (int)((grid + sms - 1) / sms) < 2 ? 1 : 2;
-  const int stages = s1_stages(per_sm, (size_t)R * kS1Cols * 4 + kS1Cols * 4);
-  const size_t smem = kS1Header + 1024 + (size_t)stages * (R * kS1Cols * 4 + kS1Cols * 4);
+  const int stages = s1_stages(per_sm, (size_t)R * kS1Cols * 4);
+  const size_t smem = kS1Header + 1024 + (size_t)stages * R * kS1Cols * 4;
   auto kern = mv_s1_tiled_kernel<R>;
   if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess)
     return check_launch("mv S=1 tiled smem attribute");
