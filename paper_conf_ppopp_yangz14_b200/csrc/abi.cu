@@ -651,7 +651,7 @@ int cudanp_mv_variant(int impl, const float* A, int64_t lda, const float* x, flo
   if (impl == CUDANP_IMPL_S1_LITERAL) return mv_literal(A, lda, x, y, n_outer, n_inner, as_stream(stream));
   if (impl == CUDANP_IMPL_S1_TILED) {
     if (n_outer > 0 && n_inner > 0 && !(tiled_ok(A, lda, x, n_outer, n_inner) && n_inner % 4 == 0))
-      return tiled_unsupported();  // (x is read with 128-bit loads)
+      return tiled_unsupported();  // (x chunks are 1-D bulk copies: 16-byte aligned, w % 4 == 0)
     return mv_s1_tiled(A, lda, x, y, n_outer, n_inner, as_stream(stream));
   }
   return dp_mv(impl == CUDANP_IMPL_DP_BLOCK, A, lda, x, y, n_outer, n_inner, as_stream(stream));

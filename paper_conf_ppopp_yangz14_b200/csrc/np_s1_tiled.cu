@@ -15,10 +15,11 @@
 // the NP speedups (CUDANP_IMPL_S1_TILED); the method (one master, no slaves)
 // is the literal Fig 2 loop.
 //
-//  MV:   a CTA owns R rows; a producer warp streams the column tiles into
-//        the ring; each consumer thread accumulates its row (acc += A[r][j] *
-//        x[j]; x's 128-byte chunk is a broadcast load issued one tile ahead,
-//        so its L2 latency hides behind the previous tile) and stores y[r].
+//  MV:   a CTA owns R rows; a producer warp streams the column tiles -- and
+//        the matching 128-byte chunk of x, a 1-D tensor box on the same
+//        barrier (zero-filled past w) -- into the ring; each consumer thread
+//        accumulates its row (acc += A[r][j]*x[j], x read from shared memory
+//        as a broadcast) and stores y[r].
 //  reduce: the same walk; each thread folds its row's elements of every tile
 //        (sum or max) and the master -- the thread itself -- applies init[n]
 //        and stores out[n] at the row's last tile.
@@ -40,6 +41,13 @@ constexpr int kS1Cols = 32;  // tile width: 32 x 4 B = one 128-byte swizzle row
 // Element offset of float4 chunk c (0..7) of row r in a SWIZZLE_128B tile.
 __device__ __forceinline__ int swz128(int r, int c) { return r * kS1Cols + ((c ^ (r & 7)) << 2); }
 
+__device__ __forceinline__ void tma_load_1d(void* dst, const CUtensorMap* map, int c0, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.tensor.1d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
+      " [%0], [%1, {%2}], [%3];" ::"r"(smem_u32(dst)),
+      "l"((uint64_t)map), "r"(c0), "r"(smem_u32(bar))
+      : "memory");
+}
 __device__ __forceinline__ void tma_store_2d(const CUtensorMap* map, int c0, int c1, const void* src) {
   asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%1, %2}], [%3];" ::"l"(
                    (uint64_t)map),
@@ -63,14 +71,15 @@ constexpr size_t kS1Header = 1024;
 // ---------------------------------------------------------------- MV, S = 1
 template <int R>
 __global__ void __launch_bounds__(R + 32, 1)
-mv_s1_tiled_kernel(const __grid_constant__ CUtensorMap mapA, const float* __restrict__ x,
+mv_s1_tiled_kernel(const __grid_constant__ CUtensorMap mapA, const __grid_constant__ CUtensorMap mapX,
                    float* __restrict__ y, int64_t h, int64_t w, int stages) {
   pdl_entry();
   extern __shared__ __align__(1024) unsigned char smem_raw[];
   unsigned char* base = smem_raw + ((1024 - (smem_u32(smem_raw) & 1023)) & 1023);
-  uint64_t* full = reinterpret_cast<uint64_t*>(base);
-  uint64_t* empty = full + stages;
+  uint64_t* full = reinterpret_cast<uint64_t*>(base);   // A tile and x chunk landed
+  uint64_t* empty = full + stages;                         // consumers done with the stage
   float* tiles = reinterpret_cast<float*>(base + kS1Header);
+  float* xs = tiles + stages * (R * kS1Cols);              // [stages][32]
   constexpr int kWarps = R / 32;
   constexpr uint32_t kStageBytes = R * kS1Cols * 4;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -91,35 +100,27 @@ mv_s1_tiled_kernel(const __grid_constant__ CUtensorMap mapA, const float* __rest
       for (int t = 0; t < ntiles; ++t) {
         const int st = t % stages;
         if (t >= stages) mbar_wait(&empty[st], ((t / stages) - 1) & 1);
-        mbar_expect_tx(&full[st], kStageBytes);
+        mbar_expect_tx(&full[st], kStageBytes + kS1Cols * 4);
         tma_load_2d(tiles + st * (R * kS1Cols), &mapA, t * kS1Cols, row0, &full[st]);
+        tma_load_1d(xs + st * kS1Cols, &mapX, t * kS1Cols, &full[st]);
       }
     }
     return;
   }
   const int r = threadIdx.x;
   V4<float> acc = {0.f, 0.f, 0.f, 0.f};
-  auto load_x = [&](int t, V4<float>* xv) {  // x chunk of tile t (zeros past w)
-    const int64_t j0 = (int64_t)t * kS1Cols;
-#pragma unroll
-    for (int c = 0; c < 8; ++c)
-      xv[c] = j0 + 4 * c < w ? ldg4(x + j0 + 4 * c) : V4<float>{0.f, 0.f, 0.f, 0.f};
-  };
-  V4<float> xcur[8], xnext[8];
-  load_x(0, xcur);
   for (int t = 0; t < ntiles; ++t) {
     const int st = t % stages;
-    if (t + 1 < ntiles) load_x(t + 1, xnext);
     mbar_wait(&full[st], (t / stages) & 1);
     const float* tile = tiles + st * (R * kS1Cols);
+    const float* xt = xs + st * kS1Cols;
 #pragma unroll
-    for (int c = 0; c < 8; ++c) {
-      const float4 a = *reinterpret_cast<const float4*>(tile + swz128(r, c));  // zero past w
-      acc.x = fmaf(a.x, xcur[c].x, acc.x); acc.y = fmaf(a.y, xcur[c].y, acc.y);
-      acc.z = fmaf(a.z, xcur[c].z, acc.z); acc.w = fmaf(a.w, xcur[c].w, acc.w);
+    for (int c = 0; c < 8; ++c) {  // (past w both the tile and the x chunk are zero-filled)
+      const float4 a = *reinterpret_cast<const float4*>(tile + swz128(r, c));
+      const float4 xv = *reinterpret_cast<const float4*>(xt + 4 * c);  // broadcast
+      acc.x = fmaf(a.x, xv.x, acc.x); acc.y = fmaf(a.y, xv.y, acc.y);
+      acc.z = fmaf(a.z, xv.z, acc.z); acc.w = fmaf(a.w, xv.w, acc.w);
     }
-#pragma unroll
-    for (int c = 0; c < 8; ++c) xcur[c] = xnext[c];
     __syncwarp();
     if (lane == 0) mbar_arrive(&empty[st]);
   }
@@ -302,6 +303,27 @@ static int encode_s1(CUtensorMap* map, const void* p, int64_t rows, int64_t cols
   return CUDANP_OK;
 }
 
+// x as a 1-D tensor of w floats, box of 32 (one 128-byte chunk per stage).
+static int encode_x1(CUtensorMap* map, const float* x, int64_t w) {
+  EncodeTiledFnS1 enc = encode_fn_s1();
+  if (!enc) {
+    set_error("cuTensorMapEncodeTiled entry point unavailable");
+    return CUDANP_ERR_CUDA;
+  }
+  const cuuint64_t dims[1] = {(cuuint64_t)w};
+  const cuuint64_t strides[1] = {0};
+  const cuuint32_t box[1] = {(cuuint32_t)kS1Cols};
+  const cuuint32_t estr[1] = {1};
+  CUresult r = enc(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 1, const_cast<float*>(x), dims, strides, box, estr,
+                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                   CU_TENSOR_MAP_L2_PROMOTION_NONE, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) {
+    set_error("cuTensorMapEncodeTiled (x) failed (%d)", (int)r);
+    return CUDANP_ERR_CUDA;
+  }
+  return CUDANP_OK;
+}
+
 // Ring depth for `per_sm` resident CTAs of `stage` bytes (<= 227 KB per CTA,
 // 228 KB per SM, 1 KB reserved per CTA), at most 12 stages.
 static int s1_stages(int per_sm, size_t stage) {
@@ -315,17 +337,18 @@ static int s1_stages(int per_sm, size_t stage) {
 template <int R>
 static int launch_mv_s1(const float* A, int64_t lda, const float* x, float* y, int64_t h, int64_t w,
                         cudaStream_t st) {
-  CUtensorMap map;
+  CUtensorMap map, mapx;
   if (int rc = encode_s1(&map, A, h, w, lda, R)) return rc;
+  if (int rc = encode_x1(&mapx, x, w)) return rc;
   const int64_t grid = (h + R - 1) / R;
   const int sms = sm_count();
   const int per_sm = (int)((grid + sms - 1) / sms) < 2 ? 1 : 2;
-  const int stages = s1_stages(per_sm, (size_t)R * kS1Cols * 4);
-  const size_t smem = kS1Header + 1024 + (size_t)stages * R * kS1Cols * 4;
+  const int stages = s1_stages(per_sm, (size_t)R * kS1Cols * 4 + kS1Cols * 4);
+  const size_t smem = kS1Header + 1024 + (size_t)stages * (R * kS1Cols * 4 + kS1Cols * 4);
   auto kern = mv_s1_tiled_kernel<R>;
   if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess)
     return check_launch("mv S=1 tiled smem attribute");
-  launch_pdl(kern, dim3((unsigned)grid), dim3(R + 32), smem, st, map, x, y, h, w, stages);
+  launch_pdl(kern, dim3((unsigned)grid), dim3(R + 32), smem, st, map, mapx, y, h, w, stages);
   return check_launch("mv S=1 tiled launch");
 }
 
