@@ -48,6 +48,8 @@ int le_tma(const float*, float*, float*, float*, float*, int64_t, int64_t, float
 int mv_s1_tiled(const float*, int64_t, const float*, float*, int64_t, int64_t, cudaStream_t);
 int scan_s1_tiled(const void*, const void*, void*, int64_t, int64_t, int, cudaStream_t);
 int reduce_s1_tiled(const void*, const void*, void*, int64_t, int64_t, int, int, cudaStream_t);
+int le_tma_pm(const float*, float*, float*, float*, float*, int64_t, int64_t, float, int, int,
+              cudaStream_t);
 int le_literal(const float*, float*, float*, float*, float*, int64_t, int64_t, float, int,
                cudaStream_t);
 
@@ -595,6 +597,14 @@ int cudanp_le_gicov_placement(const float* in, float* gicov, float* ave, float* 
     return le_np(in, gicov, ave, var, ep, n_outer, n_inner, threshold, layout, S, dist, m, true,
                  as_stream(stream));
   if (placement != CUDANP_GRAD_SHARED) return fail_invalid("placement");
+  if (layout == 1) {  // point-major: inter-warp teams, one TMA box of [32 items x L points] per group
+    if (m != MAP_INTER || S > 16 || n_inner > 256 || n_outer % 4 != 0 || !aligned16(in)) {
+      set_error("shared-memory Grad (point-major) is built for the inter-warp map, S <= 16, "
+                "n_inner <= 256, n_outer %% 4 == 0 and a 16-byte aligned input");
+      return CUDANP_ERR_UNSUPPORTED;
+    }
+    return le_tma_pm(in, gicov, ave, var, ep, n_outer, n_inner, threshold, S, dist, as_stream(stream));
+  }
   if (layout != 0 || m != MAP_INTRA || !valid_S(S) || !aligned16(in)) {
     set_error("shared-memory Grad is built for item-major data, the intra-warp map, S = 2^k <= 32 "
               "and a 16-byte aligned input");

@@ -105,7 +105,9 @@ def test_le_grad_placements_bit_identical():
                 for gv, bv, name in zip(got, base, ("gicov", "ave", "var", "ep")):
                     assert np.array_equal(gv.view(np.uint32), bv.view(np.uint32)), \
                         f"placement {pl} N={N} L={L} S={S} d={d} {name}"
-    # point-major: the global placement for both maps; shared is item-major only
+    # point-major: the global placement for both maps; the shared placement
+    # (a TMA box of [32 items x L points] per group, Fig 6b) for inter-warp
+    # teams of S <= 16, non-powers of two included
     x = np.ascontiguousarray(synth.items(200, 150, "f32_unit").T)
     xd = dev(x)
     for m in (C.INTRA_WARP, C.INTER_WARP):
@@ -113,6 +115,28 @@ def test_le_grad_placements_bit_identical():
         got = [host(t) for t in C.cudanp_le_gicov(xd, 0.02, layout=1, S=8, map=m, placement=C.GRAD_GLOBAL)]
         for gv, bv in zip(got, base):
             assert np.array_equal(gv.view(np.uint32), bv.view(np.uint32))
-    with pytest.raises(C.CudanpError) as ei:
-        C.cudanp_le_gicov(xd, 0.02, layout=1, S=8, placement=C.GRAD_SHARED)
+    for N, L in [(4, 1), (36, 5), (200, 150), (1000, 150), (4100, 150), (64, 256)]:
+        xi = synth.items(N, L, "f32_unit", seed=L)
+        x = np.ascontiguousarray(xi.T)
+        _, ra, rv, _ = O.le_gicov(xi, 0.0, 0)
+        with np.errstate(divide="ignore"):
+            thr = float(np.median(ra.astype(np.float64) ** 2 / rv))
+        ref = O.le_gicov(xi, thr, 0)
+        xd = dev(x)
+        for S, d in itertools.product((1, 2, 3, 4, 5, 8, 10, 15, 16), (C.CYCLIC, C.BLOCK)):
+            base = [host(t) for t in C.cudanp_le_gicov(xd, thr, layout=1, S=S, dist=d, map=C.INTER_WARP)]
+            got = [host(t) for t in C.cudanp_le_gicov(xd, thr, layout=1, S=S, dist=d, map=C.INTER_WARP,
+                                                        placement=C.GRAD_SHARED)]
+            check([torch.from_numpy(t) for t in got], ref, xi, L, thr, f"le pm shared N={N} L={L} S={S}")
+            for gv, bv, name in zip(got, base, ("gicov", "ave", "var", "ep")):
+                assert np.array_equal(gv.view(np.uint32), bv.view(np.uint32)), \
+                    f"pm shared placement N={N} L={L} S={S} d={d} {name}"
+    for kw in ({"map": C.INTRA_WARP, "S": 8}, {"map": C.INTER_WARP, "S": 32}):
+        with pytest.raises(C.CudanpError) as ei:
+            C.cudanp_le_gicov(dev(np.ascontiguousarray(synth.items(200, 150, "f32_unit").T)), 0.02,
+                              layout=1, placement=C.GRAD_SHARED, **kw)
+        assert ei.value.status == C.ERR_UNSUPPORTED
+    with pytest.raises(C.CudanpError) as ei:  # N % 4 != 0: the TMA row pitch
+        C.cudanp_le_gicov(dev(np.ascontiguousarray(synth.items(203, 150, "f32_unit").T)), 0.02,
+                          layout=1, S=8, map=C.INTER_WARP, placement=C.GRAD_SHARED)
     assert ei.value.status == C.ERR_UNSUPPORTED

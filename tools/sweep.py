@@ -446,16 +446,18 @@ def f2(L=150):
         # Fig 15 analog: the home of Grad (6c registers = above, 6b shared memory
         # staged by TMA, 6a global = loop 3 re-reads the input), intra-warp teams
         for pl, name in ((C.GRAD_SHARED, "grad_shared"), (C.GRAD_GLOBAL, "grad_global")):
-            if pl == C.GRAD_SHARED and layout == 1:
-                continue
-            for S in C.SLAVE_SIZES:
+            # item-major: intra-warp teams; point-major: the shared placement is
+            # built for inter-warp teams (S <= 16, any of the Fig 12 sizes)
+            pm_shared = pl == C.GRAD_SHARED and layout == 1
+            mp = C.INTER_WARP if pm_shared else C.INTRA_WARP
+            for S in ((1, 2, 3, 4, 5, 8, 10, 15, 16) if pm_shared else C.SLAVE_SIZES):
                 for d in (C.CYCLIC, C.BLOCK):
                     med, _ = time_ms(lambda: C.load().cudanp_le_gicov_placement(
                         x.data_ptr(), g.data_ptr(), *(t.data_ptr() for t in st), N, L, 0.02, layout, S,
-                        d, C.INTRA_WARP, pl, None))
+                        d, mp, pl, None))
                     emit({"config": "F2", "op": "le_gicov", "dtype": "f32", "N": N, "L": L,
                           "layout": "point-major" if layout else "item-major", "placement": name,
-                          "S": S, "dist": DN[d], "map": "intra", "impl": "np_" + name,
+                          "S": S, "dist": DN[d], "map": MN[mp], "impl": "np_" + name,
                           "t_median_us": round(med * 1e3, 2), "alg_bytes": nb,
                           "gbs": round(nb / (med * 1e-3) / 1e9, 1),
                           "speedup_vs_s1_literal": round(lit / med, 3)})
