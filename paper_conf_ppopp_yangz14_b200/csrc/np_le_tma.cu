@@ -138,10 +138,11 @@ le_tma_kernel(const float* __restrict__ in, float* gicov, float* ave_out, float*
 // box [32 items x L points] -- 128 bytes per point, coalesced -- that a
 // producer warp streams into the ring with one 2-D TMA copy; slave s runs
 // loops 1+2 over its points (cyclic P:166 / block R5) reading
-// ring[point][lane], the S partial sums meet in shared memory and the
-// master folds them (in slave order) into ave, which the team reads
-// back (read_from_master); loop 3 re-reads the points from shared
-// memory and var / ep are folded the same way before the master stores.  The
+// ring[point][lane], the S partial sums meet in shared memory and
+// every slave folds them (in slave order) into ave itself -- a uniform value
+// recomputed rather than broadcast, which saves a barrier; loop 3
+// re-reads the points from shared memory and var / ep are folded by the
+// master before it stores.  The
 // producer runs up to `stages` groups ahead, so the next groups' bytes are
 // in flight while the slaves reduce (the register version idles its loads
 // during each group's reductions and barriers).  The slaves sync among
@@ -153,7 +154,7 @@ __global__ void __launch_bounds__(32 * (S + 1), 1)
 le_tma_pm_kernel(const __grid_constant__ CUtensorMap map, float* gicov, float* ave_out,
                  float* var_out, float* ep_out, int64_t N, int64_t L, float thr, int stages) {
   extern __shared__ __align__(128) unsigned char smem_raw[];
-  __shared__ float red[2][S][33], red2[2][S][33], slot[2][32];  // double-buffered by group parity
+  __shared__ float red[2][S][33], red2[2][S][33];  // double-buffered by group parity
   uint64_t* full = reinterpret_cast<uint64_t*>(smem_raw);
   uint64_t* empty = full + stages;
   float* ring = reinterpret_cast<float*>(smem_raw + lt_header_bytes(stages));  // [stages][L][32]
@@ -198,13 +199,10 @@ le_tma_pm_kernel(const __grid_constant__ CUtensorMap map, float* gicov, float* a
     if (c < cnt) s2.x += p0[c * pstep];
     red[par][warp][lane] = s2.x + s2.y;
     team_sync();
-    if (warp == 0) {  // sum = reduction(sum) in slave order; ave
-      float sm = red[par][0][lane];
-      for (int k = 1; k < S; ++k) sm += red[par][k][lane];
-      slot[par][lane] = sm / (float)L;
-    }
-    team_sync();
-    const float ave = slot[par][lane];  // read_from_master
+    float sm = red[par][0][lane];  // sum = reduction(sum) in slave order
+#pragma unroll
+    for (int k = 1; k < S; ++k) sm += red[par][k][lane];
+    const float ave = sm / (float)L;  // P:309, recomputed by every slave
     // loop 3, pairs as LeSlave::loop3
     const float2 na = make_float2(-ave, -ave);
     float2 v2 = make_float2(0.f, 0.f), e2 = make_float2(0.f, 0.f);
@@ -288,14 +286,16 @@ static int launch_le_tma_pm(const float* in, float* g, float* a, float* v, float
   const cuuint32_t estr[2] = {1, 1};
   CUresult r = enc(&map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float*>(in), dims, strides, box,
                    estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
-                   CU_TENSOR_MAP_L2_PROMOTION_L2_128B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+                   CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) {
     set_error("cuTensorMapEncodeTiled failed (%d)", (int)r);
     return CUDANP_ERR_CUDA;
   }
-  // two CTAs per SM, each with as many group stages as half an SM holds (<= 8)
+  // three CTAs per SM (the slaves' reductions and barriers need the extra
+  // warps; ncu saw one 9-warp CTA per SM consumer-bound), each with as many
+  // group stages as a third of the SM's shared memory holds (<= 8)
   const size_t stage = (size_t)L * 32 * 4;
-  int nst = (int)((113 * 1024 - lt_header_bytes(8)) / stage);
+  int nst = (int)((72 * 1024 - lt_header_bytes(8)) / stage);
   if (nst > 8) nst = 8;
   if (nst < 2) {
     set_error("shared-memory Grad (point-major): %lld points leave no room for a 2-stage ring", (long long)L);
@@ -303,8 +303,9 @@ static int launch_le_tma_pm(const float* in, float* g, float* a, float* v, float
   }
   const size_t smem = lt_header_bytes(nst) + (size_t)nst * stage;
   auto kern = le_tma_pm_kernel<S, DIST>;
-  if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess)
-    return check_launch("le_tma (point-major) smem attribute");
+  if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess ||
+      cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, 100) != cudaSuccess)
+    return check_launch("le_tma (point-major) smem attributes");
   const int64_t grid = persistent_grid(kern, 32 * (S + 1), smem, (N + 31) / 32);
   kern<<<(unsigned)grid, 32 * (S + 1), smem, st>>>(map, g, a, v, p, N, L, thr, nst);
   return check_launch("le_gicov (shared-memory Grad, point-major) launch");
