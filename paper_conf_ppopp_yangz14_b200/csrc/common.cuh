@@ -57,9 +57,12 @@ bool pdl_enabled();
 
 // Launch `kern` with programmatic stream serialization allowed (when enabled):
 // the kernel must begin with pdl_entry() (np_team.cuh).
+// `allow` = false launches without the attribute (the kernel's
+// griddepcontrol instructions are then no-ops and it starts after its
+// predecessor completes, as an ordinary stream launch).
 template <typename... KArgs, typename... Args>
-inline cudaError_t launch_pdl(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem,
-                              cudaStream_t st, Args... args) {
+inline cudaError_t launch_pdl_if(bool allow, void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem,
+                                 cudaStream_t st, Args... args) {
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = grid;
   cfg.blockDim = block;
@@ -67,11 +70,17 @@ inline cudaError_t launch_pdl(void (*kern)(KArgs...), dim3 grid, dim3 block, siz
   cfg.stream = st;
   cudaLaunchAttribute attr[1];
   attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-  attr[0].val.programmaticStreamSerializationAllowed = pdl_enabled() ? 1 : 0;
+  attr[0].val.programmaticStreamSerializationAllowed = (allow && pdl_enabled()) ? 1 : 0;
   cfg.attrs = attr;
   cfg.numAttrs = 1;
   return cudaLaunchKernelEx(&cfg, kern, static_cast<KArgs>(args)...);
 }
+template <typename... KArgs, typename... Args>
+inline cudaError_t launch_pdl(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem,
+                              cudaStream_t st, Args... args) {
+  return launch_pdl_if(true, kern, grid, block, smem, st, args...);
+}
+
 
 // Grid for a persistent grid-stride kernel: enough CTAs to cover `work_ctas`
 // units of CTA work, capped at (resident CTAs per SM) x (SM count), so the

@@ -287,7 +287,12 @@ int mv_multi(const float* A, int64_t lda, const float* x, float* y, int64_t h, i
       return CUDANP_OK;
     }
     if (h == 0) return CUDANP_OK;
-    launch_pdl(kern, dim3((unsigned)grid), dim3(Sh::CTA), 0, st, A, lda, x, y, h, w);
+    // Launched WITHOUT programmatic dependent launch: its CTAs launched early
+    // would co-reside with a preceding TMA TMV's CTAs (which leave registers
+    // free on every SM) and the C2 step (TMV then MV, repeated) loses 3-4 %;
+    // launched plainly they start on SMs the TMV has left (A/B,
+    // tools/exp_pdl_ab.py: step 7.07 -> 7.33 TB/s; MV repeated alone -1 %).
+    launch_pdl_if(false, kern, dim3((unsigned)grid), dim3(Sh::CTA), 0, st, A, lda, x, y, h, w);
     return check_launch("mv (multi-warp team) launch");
   });
   return CUDANP_OK;
