@@ -438,7 +438,11 @@ def run_cudanp(args):
     if not args.no_c5:
         del A_t, A_m, x_t, x_m, y_t, y_m
         torch.cuda.empty_cache()
-        c5 = run_c5(C, P, rank, world, args.c5_steps, gather_used if world > 1 else "none")
+        # C5's outputs are bulk (64M floats for the reduce): "auto" gathers them
+        # with NCCL's bulk send/recv rather than as 16-byte remote stores from
+        # the kernel's masters; --gather fused / native force those paths.
+        c5_gather = "nccl" if args.gather == "auto" else gather_used
+        c5 = run_c5(C, P, rank, world, args.c5_steps, c5_gather if world > 1 else "none")
 
     if rank != 0:
         if world > 1:
