@@ -9,8 +9,11 @@
  *   MV  with A = all ones        -> y[i] = sum_j x[j]
  *   reduce of ones (int32, sum)  -> L; of 0..L-1 (max) -> L-1
  *   scan of ones (int32)         -> 1..L
- * with small-integer x so every fp32 sum is exact.  It also checks that a bad
- * argument is rejected before any launch with CUDANP_ERR_INVALID.
+ * with small-integer x so every fp32 sum is exact -- for S = CUDANP_S_AUTO
+ * (the library's choice), S = 1, 4, 32, 256 and the inter-warp-only S = 5,
+ * and for the TMA-tiled S=1 baselines (CUDANP_IMPL_S1_TILED).  It also checks
+ * that a bad argument is rejected before any launch with CUDANP_ERR_INVALID
+ * and an unbuilt combination with CUDANP_ERR_UNSUPPORTED.
  * Exit code 0 = all checks passed.  Test infrastructure, not product code. */
 #include <stdio.h>
 #include <stdlib.h>
@@ -40,7 +43,7 @@
 
 int main(void) {
   const int64_t h = 777, w = 1030, N = 5000, L = 150;
-  const int Ss[] = {1, 4, 32, 256};
+  const int Ss[] = {CUDANP_S_AUTO, 1, 4, 5, 32, 256};
   int fails = 0;
   cudaStream_t st;
   CK(cudaStreamCreate(&st));
@@ -64,7 +67,7 @@ int main(void) {
   for (int64_t i = 0; i < (h > w ? h : w); ++i) hx[i] = (float)(i % 7);
   CK(cudaMemcpy(x, hx, sizeof(float) * (h > w ? h : w), cudaMemcpyHostToDevice));
 
-  for (int k = 0; k < 4; ++k) {
+  for (int k = 0; k < 6; ++k) {
     for (int dist = 0; dist < 2; ++dist) {
       const int S = Ss[k];
       /* TMV: y[j] = sum_{i<h} x[i] */
@@ -107,6 +110,35 @@ int main(void) {
       for (int64_t n = 0; n < N; ++n)
         if (hout[n] != L - 1) { fprintf(stderr, "max S=%d n=%ld: %d\n", S, (long)n, hout[n]); ++fails; break; }
     }
+  }
+  /* tiled S=1 baselines on rows of 148 elements (a multiple of 4): scan of ones -> 1..148,
+   * reduce of ones -> 148 */
+  {
+    const int64_t L4 = 148;
+    for (int64_t i = 0; i < N * L4; ++i) hin[i] = 1;
+    CK(cudaMemcpy(in, hin, sizeof(int32_t) * N * L4, cudaMemcpyHostToDevice));
+    NP(cudanp_batched_loop_scan_variant(CUDANP_IMPL_S1_TILED, in, NULL, out, N, L4, CUDANP_I32, st));
+    CK(cudaMemcpyAsync(hout, out, sizeof(int32_t) * N * L4, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    for (int64_t i = 0; i < N * L4; ++i)
+      if (hout[i] != (int32_t)(i % L4) + 1) { fprintf(stderr, "tiled scan i=%ld: %d\n", (long)i, hout[i]); ++fails; break; }
+    NP(cudanp_batched_loop_reduce_variant(CUDANP_IMPL_S1_TILED, in, NULL, out, N, L4, CUDANP_I32, CUDANP_SUM, st));
+    CK(cudaMemcpyAsync(hout, out, sizeof(int32_t) * N, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    for (int64_t n = 0; n < N; ++n)
+      if (hout[n] != L4) { fprintf(stderr, "tiled reduce n=%ld: %d\n", (long)n, hout[n]); ++fails; break; }
+    /* rows of 150 elements cannot be described to TMA: unsupported, not wrong */
+    if (cudanp_batched_loop_scan_variant(CUDANP_IMPL_S1_TILED, in, NULL, out, N, L, CUDANP_I32, st) !=
+        CUDANP_ERR_UNSUPPORTED) {
+      fprintf(stderr, "tiled scan with L %% 4 != 0 was not refused\n");
+      ++fails;
+    }
+  }
+  /* intra-warp teams need S = 2^k: S = 5 intra-warp is unsupported */
+  if (cudanp_batched_loop_reduce(in, NULL, out, N, L, CUDANP_I32, CUDANP_SUM, 5, 0, CUDANP_MAP_INTRA_WARP, st) !=
+      CUDANP_ERR_UNSUPPORTED) {
+    fprintf(stderr, "S=5 intra-warp was not refused\n");
+    ++fails;
   }
   /* validation before launch: S = 6 is not a team size (3, 5, 10, 15 are, inter-warp) */
   if (cudanp_batched_loop_reduce(in, NULL, out, N, L, CUDANP_I32, CUDANP_SUM, 6, 0, 0, st) != CUDANP_ERR_INVALID) {
