@@ -21,16 +21,24 @@ B.build()
 C.load()
 
 S_ = st.sampled_from(C.SLAVE_SIZES)
+# + the inter-warp-only team sizes and the library's own choice
+S_ALL = st.sampled_from(C.SLAVE_SIZES + C.INTER_ONLY_SIZES + (C.S_AUTO,))
+
+
+def _map_for(S, map_):
+    """A non-power-of-two S exists only as an inter-warp team."""
+    return C.INTER_WARP if S in C.INTER_ONLY_SIZES and map_ == C.INTRA_WARP else map_
 D_ = st.sampled_from([C.CYCLIC, C.BLOCK])
 M_ = st.sampled_from([C.INTRA_WARP, C.INTER_WARP, C.AUTO])
 CFG = settings(max_examples=150, deadline=None, suppress_health_check=list(HealthCheck))
 
 
 @CFG
-@given(N=st.integers(0, 700), L=st.integers(0, 300), S=S_, dist=D_, map_=M_,
+@given(N=st.integers(0, 700), L=st.integers(0, 300), S=S_ALL, dist=D_, map_=M_,
        op=st.sampled_from([C.SUM, C.MAX]), shift=st.integers(0, 3), use_init=st.booleans(),
        seed=st.integers(0, 10**6))
 def test_reduce_random(N, L, S, dist, map_, op, shift, use_init, seed):
+    map_ = _map_for(S, map_)
     x = synth.gen(1, "i32_full", 0, N * L + shift, seed=seed)
     xd = dev(x)[shift:].view(N, L) if N * L else dev(x)[: 0].view(N, L)
     ini = synth.init(N, "i32_full", seed=seed)
@@ -41,9 +49,10 @@ def test_reduce_random(N, L, S, dist, map_, op, shift, use_init, seed):
 
 
 @CFG
-@given(N=st.integers(0, 400), L=st.integers(0, 300), S=S_, dist=D_, map_=M_,
+@given(N=st.integers(0, 400), L=st.integers(0, 300), S=S_ALL, dist=D_, map_=M_,
        shift=st.integers(0, 3), use_init=st.booleans(), seed=st.integers(0, 10**6))
 def test_scan_random(N, L, S, dist, map_, shift, use_init, seed):
+    map_ = _map_for(S, map_)
     x = synth.gen(1, "i32_small", 0, N * L + shift, B=1 << 15, seed=seed)
     xd = dev(x)[shift:].view(N, L) if N * L else dev(x)[: 0].view(N, L)
     ini = synth.init(N, "i32_small", B=1 << 15, seed=seed)
@@ -54,9 +63,10 @@ def test_scan_random(N, L, S, dist, map_, shift, use_init, seed):
 
 
 @CFG
-@given(h=st.integers(0, 300), w=st.integers(1, 300), pad=st.integers(0, 5), S=S_, dist=D_,
+@given(h=st.integers(0, 300), w=st.integers(1, 300), pad=st.integers(0, 5), S=S_ALL, dist=D_,
        map_=M_, seed=st.integers(0, 10**6))
 def test_matvec_random(h, w, pad, S, dist, map_, seed):
+    map_ = _map_for(S, map_)
     lda = w + pad
     A = synth.matrix(h, lda, "f32_int4", seed=seed)
     xt, xm = synth.vector(h, "f32_int4", seed=seed), synth.vector(w, "f32_int4", seed=seed)
