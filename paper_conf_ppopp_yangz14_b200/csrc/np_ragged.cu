@@ -289,42 +289,17 @@ static int launch_ragged_multi(const T* in, const int64_t* off, const T* init, T
 // turns (ballot of the long ones, bounds broadcast by shfl from their
 // master), with a butterfly team reduction; the master stores
 // (P:327).  Every segment is still reduced by exactly one team.
-//
-// STAGED: when the 32 segments of a tile are short enough that their whole
-// span [off[first], off[last+1]) fits kStageCap elements (mean-16 segments:
-// ~512), the warp first copies the span into its shared-memory buffer with
-// coalesced 128-bit loads (every lane a slice of the contiguous span), and
-// each master then reduces its own segment out of shared memory.  Without
-// it each master walks its ~64-byte segment alone, so a warp's load touches
-// 32 separate segments (the short-segment mixes ran at 50-66 % of the copy
-// peak).  The master alone still runs its loop (a team of one); the warp only
-// moves the bytes, as the TMA does for the tiled S = 1 kernels.
-constexpr int kStageCap = 1024;  // elements of one tile's span a warp stages
-
-// cp.async (LDGSTS): a global -> shared copy that needs no register.
-__device__ __forceinline__ void cp_async16(void* s, const void* g) {
-  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"((uint32_t)__cvta_generic_to_shared(s)),
-               "l"(g) : "memory");
-}
-__device__ __forceinline__ void cp_async4(void* s, const void* g) {
-  asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"((uint32_t)__cvta_generic_to_shared(s)),
-               "l"(g) : "memory");
-}
-
-template <class T, class Op, bool STAGED>
+template <class T, class Op>
 __global__ void __launch_bounds__(kRaggedBlock)
 ragged_adaptive_kernel(const T* __restrict__ in, const int64_t* __restrict__ off,
                        const T* __restrict__ init, T* __restrict__ out, int64_t N, int64_t thresh) {
   pdl_entry();
   constexpr int K = 2;  // tiles of 32 segments per warp step: their bound loads overlap
-  constexpr int kBuf = kStageCap + 4;  // + up to 3 leading pad elements (16-byte alignment)
-  extern __shared__ __align__(16) unsigned char ragged_smem[];
   const int lane = threadIdx.x & 31;
   const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
   const int64_t ntiles = (N + 31) / 32;
   const T id = Op::template identity<T>();
-  T* wbuf = reinterpret_cast<T*>(ragged_smem) + (threadIdx.x >> 5) * (K * kBuf);
   for (int64_t t0 = warp * K; t0 < ntiles; t0 += nwarps * K) {
     int64_t item[K], b[K], len[K];
 #pragma unroll
@@ -336,62 +311,6 @@ ragged_adaptive_kernel(const T* __restrict__ in, const int64_t* __restrict__ off
         len[k] = off[item[k] + 1] - b[k];
         if (len[k] < 0) len[k] = 0;
       }
-    }
-    T sp[K];       // staged segments' results
-    bool stg[K];   // warp-uniform: tile k went through the staged path
-    if constexpr (STAGED) {
-      int64_t b0[K], e0[K];
-#pragma unroll
-      for (int k = 0; k < K; ++k) {
-        // the tile's span: from the first master's start to the last valid master's end
-        const int last = (int)((N - (t0 + k) * 32 - 1 < 31) ? N - (t0 + k) * 32 - 1 : 31);
-        b0[k] = __shfl_sync(kFull, b[k], 0);
-        e0[k] = __shfl_sync(kFull, b[k] + len[k], last < 0 ? 0 : last);
-        const bool inside = item[k] >= N || (b[k] >= b0[k] && b[k] + len[k] <= e0[k]);
-        stg[k] = last >= 0 && __all_sync(kFull, inside) && e0[k] - b0[k] <= kStageCap;
-      }
-      // copy every staged span with cp.async (global -> shared without
-      // registers, every copy of both tiles in flight): head scalars, 16-byte
-      // body units, tail scalars; element g lands at g - b0 + pad, pad = b0's
-      // offset in its 16-byte line, so body units stay aligned
-      int pad[K];
-#pragma unroll
-      for (int k = 0; k < K; ++k) {
-        pad[k] = (int)(((uintptr_t)(in + b0[k]) >> 2) & 3);
-        if (!stg[k]) continue;
-        const int64_t sp_len = e0[k] - b0[k];
-        const int hn = (int)(((4 - pad[k]) & 3) < sp_len ? ((4 - pad[k]) & 3) : sp_len);
-        const int nu = (int)((sp_len - hn) >> 2);
-        const int done = hn + 4 * nu;
-        const T* g = in + b0[k];
-        T* buf = wbuf + k * kBuf + pad[k];
-        if (lane < hn) cp_async4(buf + lane, g + lane);
-        for (int u = lane; u < nu; u += 32) cp_async16(buf + hn + 4 * u, g + hn + 4 * u);
-        if (lane < (int)(sp_len - done)) cp_async4(buf + done + lane, g + done + lane);
-      }
-      asm volatile("cp.async.commit_group;\n\tcp.async.wait_group 0;" ::: "memory");
-      __syncwarp();
-#pragma unroll
-      for (int k = 0; k < K; ++k) {
-        sp[k] = id;
-        if (!stg[k]) continue;
-        // the master's own loop over its segment, out of shared memory
-        const T* p = wbuf + k * kBuf + pad[k] + (b[k] - b0[k]);
-        const int n = item[k] < N ? (int)len[k] : 0;
-        T a0 = id, a1 = id, a2 = id, a3 = id;
-        int i = 0;
-        for (; i + 3 < n; i += 4) {
-          a0 = Op::apply(a0, p[i]); a1 = Op::apply(a1, p[i + 1]);
-          a2 = Op::apply(a2, p[i + 2]); a3 = Op::apply(a3, p[i + 3]);
-        }
-        for (; i < n; ++i) a0 = Op::apply(a0, p[i]);
-        sp[k] = Op::apply(Op::apply(a0, a1), Op::apply(a2, a3));
-        len[k] = 0;  // nothing left for the direct paths below
-      }
-      __syncwarp();  // the buffer is rewritten next step
-    } else {
-#pragma unroll
-      for (int k = 0; k < K; ++k) { sp[k] = id; stg[k] = false; }
     }
     T part[K];
     // short segments: each master alone (a team of one); all K items' loads in flight
@@ -464,7 +383,6 @@ ragged_adaptive_kernel(const T* __restrict__ in, const int64_t* __restrict__ off
         for (int o = 16; o > 0; o >>= 1) pv = Op::apply(pv, __shfl_xor_sync(kFull, pv, o));
         if (lane == src) part[k] = pv;
       }
-      if (stg[k]) part[k] = sp[k];
       if (item[k] < N) out[item[k]] = init ? Op::apply(init[item[k]], part[k]) : part[k];
     }
   }
@@ -474,12 +392,9 @@ template <class T, class Op>
 static int launch_ragged_adaptive(const T* in, const int64_t* off, const T* init, T* out, int64_t N,
                                   int64_t thresh, cudaStream_t st) {
   if (N == 0) return CUDANP_OK;
-  auto kern = ragged_adaptive_kernel<T, Op, true>;
-  const size_t smem = (size_t)(kRaggedBlock / 32) * 2 * (kStageCap + 4) * sizeof(T);
-  if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess)
-    return check_launch("ragged_loop_reduce (adaptive teams) smem attribute");
-  const int64_t grid = persistent_grid(kern, kRaggedBlock, smem, (N + 2 * kRaggedBlock - 1) / (2 * kRaggedBlock));
-  launch_pdl(kern, dim3((unsigned)grid), dim3(kRaggedBlock), smem, st, in, off, init, out, N, thresh);
+  auto kern = ragged_adaptive_kernel<T, Op>;
+  const int64_t grid = persistent_grid(kern, kRaggedBlock, 0, (N + 2 * kRaggedBlock - 1) / (2 * kRaggedBlock));
+  launch_pdl(kern, dim3((unsigned)grid), dim3(kRaggedBlock), 0, st, in, off, init, out, N, thresh);
   return check_launch("ragged_loop_reduce (adaptive teams) launch");
 }
 
