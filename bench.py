@@ -76,6 +76,7 @@ def parse():
                          "SURVEY §8(d)) into JSONL and exit (no GPU work)")
     ap.add_argument("--oracle-cap-s", type=float, default=12.0,
                     help="--oracle-timing: seconds per (config, op, cores) before extrapolating")
+    ap.add_argument("--cpu-sample-json", action="store_true", help=argparse.SUPPRESS)
     ap.add_argument("--cpu-rows", type=int, default=4096,
                     help="rows of the C2 matrix in the oracle's CPU sample (both arms)")
     return ap.parse_args()
@@ -541,7 +542,7 @@ def run_cudanp(args):
     if c5 is not None:
         line["c5"] = c5
     if not args.no_cpu_baseline:
-        line["cpu_baseline"] = cpu_baseline(n, args.cpu_rows)
+        line["cpu_baseline"] = cpu_baseline_subprocess(n, args.cpu_rows)
     print(json.dumps(line), flush=True)
     if world > 1:
         import torch.distributed as dist
@@ -758,6 +759,19 @@ def cpu_baseline(n, rows):
             "value_1core": round(v_one, 4), "cpu": _cpu_model()}
 
 
+def cpu_baseline_subprocess(n, rows):
+    """cpu_baseline in a fresh process with no CUDA context (the same
+    function the --impl reference arm runs): this process's GPU state --
+    pinned host buffers, driver threads -- slowed the oracle by up to 40 %
+    when it ran in-process (bench r02t: 3.8 vs 5.3 GB/s)."""
+    r = subprocess.run([sys.executable, os.path.abspath(__file__), "--cpu-sample-json", "--n", str(n),
+                        "--cpu-rows", str(rows)], capture_output=True, text=True, timeout=600)
+    try:
+        return json.loads(r.stdout.strip().splitlines()[-1])
+    except Exception:
+        return {"value": None, "unit": "GB/s", "kind": "oracle", "error": (r.stderr or r.stdout)[-300:]}
+
+
 def _cpu_model():
     try:
         for line in open("/proc/cpuinfo"):
@@ -901,6 +915,9 @@ def main():
     args = parse()
     if args.oracle_timing:
         oracle_timing(args.oracle_timing, args.oracle_cap_s)
+        return
+    if args.cpu_sample_json:
+        print(json.dumps(cpu_baseline(args.n, args.cpu_rows)), flush=True)
         return
     if args.impl == "reference":
         run_reference(args)
