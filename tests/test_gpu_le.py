@@ -140,3 +140,26 @@ def test_le_grad_placements_bit_identical():
         C.cudanp_le_gicov(dev(np.ascontiguousarray(synth.items(203, 150, "f32_unit").T)), 0.02,
                           layout=1, S=8, map=C.INTER_WARP, placement=C.GRAD_SHARED)
     assert ei.value.status == C.ERR_UNSUPPORTED
+
+
+def test_le_point_major_inter_many_groups_per_cta():
+    # Point-major inter-warp with Grad in registers double-buffers loop 1
+    # across groups (np_le.cu, DB): with N well past one persistent wave each
+    # CTA alternates between its two register copies many times, an odd or
+    # even number of groups, with a ragged last group.  Oracle parity, and
+    # bit-identical to the re-read placement (Fig 6a, no double buffering).
+    for N, L in [(300013, 40), (100003, 150)]:
+        xi = synth.items(N, L, "f32_unit", seed=N)
+        _, ra, rv, _ = O.le_gicov(xi, 0.0, 0)
+        with np.errstate(divide="ignore"):
+            thr = float(np.median(ra.astype(np.float64) ** 2 / rv))
+        ref = O.le_gicov(xi, thr, 0)
+        xd = dev(np.ascontiguousarray(xi.T))
+        for S, d in itertools.product((3, 5, 8, 10, 16, 32), (C.CYCLIC, C.BLOCK)):
+            got = [host(t) for t in C.cudanp_le_gicov(xd, thr, layout=1, S=S, dist=d, map=C.INTER_WARP)]
+            check([torch.from_numpy(t) for t in got], ref, xi, L, thr, f"le pm many N={N} L={L} S={S} d={d}")
+            rr = [host(t) for t in C.cudanp_le_gicov(xd, thr, layout=1, S=S, dist=d, map=C.INTER_WARP,
+                                                       placement=C.GRAD_GLOBAL)]
+            for gv, bv, name in zip(got, rr, ("gicov", "ave", "var", "ep")):
+                assert np.array_equal(gv.view(np.uint32), bv.view(np.uint32)), \
+                    f"pm regs vs reread N={N} L={L} S={S} d={d} {name}"

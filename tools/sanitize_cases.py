@@ -126,6 +126,12 @@ def main():
         C.cudanp_batched_loop_reduce(Xw, None, S=64, dist=d)
         C.cudanp_batched_loop_scan(Xwf, None, S=64, dist=d)
         C.cudanp_mv(Aw, xw, S=256, dist=d)
+    # point-major LE, inter-warp: several groups per CTA through the
+    # double-buffered loop 1 (np_le.cu DB), and the S = 32 single-buffer path
+    lpm = dev(synth.items(30, 40003, "f32_unit"))  # (L, N) point-major
+    for S in (5, 8, 16, 32):
+        for d in (C.CYCLIC, C.BLOCK):
+            C.cudanp_le_gicov(lpm, 0.01, S=S, dist=d, map=C.INTER_WARP, layout=1)
     # the library's own version choice (S = S_AUTO) and the TMA fallbacks
     C.cudanp_tmv(A4, xt)
     C.cudanp_mv(A4, xm4)
