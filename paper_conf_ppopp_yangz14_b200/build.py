@@ -27,7 +27,7 @@ LIB = os.path.join(PKG, "libcudanp.so")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 NVFLAGS = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC", "--expt-relaxed-constexpr",
            "-Xptxas", "-warn-spills", "-I" + os.path.join(ROOT, "include")]
-SOURCES = ["abi.cu", "np_reduce.cu", "np_scan.cu", "np_matvec.cu", "np_ragged.cu", "np_le.cu", "np_tmv_tma.cu", "np_reduce_tma.cu", "np_le_tma.cu", "np_multi.cu", "np_cluster.cu", "np_s1_tiled.cu", "autotune.cu", "group.cu"]
+SOURCES = ["abi.cu", "np_reduce.cu", "np_scan.cu", "np_matvec.cu", "np_ragged.cu", "np_le.cu", "np_le_pm.cu", "np_tmv_tma.cu", "np_reduce_tma.cu", "np_le_tma.cu", "np_multi.cu", "np_cluster.cu", "np_s1_tiled.cu", "autotune.cu", "group.cu"]
 RDC_SOURCES = ["np_dp.cu"]
 
 

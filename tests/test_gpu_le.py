@@ -78,7 +78,7 @@ def test_le_full_size_sampled():
     _, ra, rv, _ = O.le_gicov(sub, 0.0, 1)
     thr = float(np.median(ra.astype(np.float64) ** 2 / rv))
     ref = O.le_gicov(sub, thr, 1)
-    for S, d in itertools.product((5, 8, 10, 15, 16), (C.CYCLIC, C.BLOCK)):
+    for S, d in itertools.product((3, 4, 5, 8, 10, 15, 16), (C.CYCLIC, C.BLOCK)):
         g, a, v, e = C.cudanp_le_gicov(x, thr, layout=1, S=S, dist=d, map=C.INTER_WARP)
         idx = torch.from_numpy(items).cuda()
         check((g[idx], a[idx], v[idx], e[idx]), ref, np.ascontiguousarray(sub.T), L, thr,
@@ -155,7 +155,7 @@ def test_le_point_major_inter_many_groups_per_cta():
             thr = float(np.median(ra.astype(np.float64) ** 2 / rv))
         ref = O.le_gicov(xi, thr, 0)
         xd = dev(np.ascontiguousarray(xi.T))
-        for S, d in itertools.product((3, 5, 8, 10, 16, 32), (C.CYCLIC, C.BLOCK)):
+        for S, d in itertools.product((3, 4, 5, 8, 10, 16, 32), (C.CYCLIC, C.BLOCK)):
             got = [host(t) for t in C.cudanp_le_gicov(xd, thr, layout=1, S=S, dist=d, map=C.INTER_WARP)]
             check([torch.from_numpy(t) for t in got], ref, xi, L, thr, f"le pm many N={N} L={L} S={S} d={d}")
             rr = [host(t) for t in C.cudanp_le_gicov(xd, thr, layout=1, S=S, dist=d, map=C.INTER_WARP,
