@@ -39,6 +39,7 @@ __device__ __forceinline__ void pdl_entry() {
   asm volatile("griddepcontrol.wait;" ::: "memory");
   asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
 }
+
 enum Dist : int { DIST_CYCLIC = 0, DIST_BLOCK = 1 };
 
 // ---------------------------------------------------------------- operators
@@ -103,6 +104,46 @@ __device__ __forceinline__ T ldg1(const T* p) { return __ldg(p); }
 // UBLKPF.L2): fire-and-forget, no registers; 16-byte aligned, bytes % 16 == 0.
 __device__ __forceinline__ void prefetch_l2(const void* p, uint32_t bytes) {
   asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(p), "r"(bytes) : "memory");
+}
+
+// L2 prefetch of bytes [p, p + bytes).  It returns no data and the L2 is the
+// device's point of coherence, so it may run BEFORE griddepcontrol.wait: a
+// predecessor's later store to those bytes updates the L2 copy, and every load
+// after the wait still sees it.  Latency-bound kernels use it to start their
+// DRAM round trip while the predecessor drains (C1).  The copy
+// engine does the work (one instruction per contiguous span, no load/store-unit
+// replays); the span is widened to 16-byte boundaries, which never leaves the
+// pages holding its first and last byte.
+__device__ __forceinline__ void prefetch_l2_span(const void* p, int64_t bytes) {
+  if (bytes <= 0) return;
+  uintptr_t a = reinterpret_cast<uintptr_t>(p) & ~uintptr_t(15);
+  const uintptr_t e = (reinterpret_cast<uintptr_t>(p) + (uintptr_t)bytes + 15) & ~uintptr_t(15);
+  for (; a < e; a += 65536) {
+    const uint32_t n = (uint32_t)(e - a < 65536 ? e - a : 65536);
+    prefetch_l2(reinterpret_cast<const void*>(a), n);
+  }
+}
+
+// Grid-wide L2 prefetch of rows [0, h) (each `row_bytes` long, row stride lda
+// floats) of a row-major fp32 matrix and of the vector x[0, nx): CTA b takes
+// its contiguous 1/gridDim of the rows (not the columns it reads itself), one
+// row per lane of warp 0, so the whole grid pulls the operand in while it
+// waits on its predecessor.
+__device__ __forceinline__ void prefetch_l2_grid(const float* A, int64_t lda, int64_t h,
+                                                 int64_t row_bytes, const float* x, int64_t nx) {
+  const int tid = threadIdx.x + blockDim.x * (threadIdx.y + blockDim.y * threadIdx.z);
+  if (tid >= 32) return;
+  const int64_t rpc = (h + gridDim.x - 1) / gridDim.x;
+  const int64_t r0 = (int64_t)blockIdx.x * rpc, r1 = r0 + rpc < h ? r0 + rpc : h;
+  if (lda * 4 == row_bytes) {  // dense rows: the CTA's rows are one span
+    if (tid == 0 && r0 < r1) prefetch_l2_span(A + r0 * lda, (r1 - r0) * row_bytes);
+  } else {
+    for (int64_t r = r0 + tid; r < r1; r += 32) prefetch_l2_span(A + r * lda, row_bytes);
+  }
+  // x: CTA b takes the b-th 1/gridDim of it.
+  const int64_t xpc = (nx + gridDim.x - 1) / gridDim.x;
+  const int64_t x0 = (int64_t)blockIdx.x * xpc;
+  if (tid == 1 && x0 < nx) prefetch_l2_span(x + x0, 4 * (x0 + xpc < nx ? xpc : nx - x0));
 }
 
 // 256-bit load (sm_100: LDG.E.ENL2.256.CONSTANT), 32-byte aligned: one

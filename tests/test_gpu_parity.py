@@ -779,6 +779,30 @@ def test_chained_calls_without_sync_see_their_predecessors():
     assert_exact(host(red), O.reduce(O.scan(it)), "scan -> reduce chain")
 
 
+def test_narrow_tmv_prefetch_sees_predecessor_writes():
+    # The narrow (C1-shaped) TMV prefetches A and x into L2 BEFORE its
+    # dependency wait.  Each round, the two kernels launched just before it
+    # (no host sync) write NEW values into the very buffers it reads: A by a
+    # scan, x by a reduce.  Every round's output must be that round's product.
+    h = w = 1024
+    Ad = torch.empty(h, w, device="cuda")
+    xd = torch.empty(h, device="cuda")
+    rounds = 6
+    srcA = [synth.items(h, w, "f32_int4", seed=100 + k) for k in range(rounds)]
+    srcx = [synth.items(h, 16, "f32_int4", seed=200 + k) for k in range(rounds)]
+    dA, dx = [dev(a) for a in srcA], [dev(a) for a in srcx]
+    ys = [torch.empty(w, device="cuda") for _ in range(rounds)]
+    torch.cuda.synchronize()
+    for k in range(rounds):
+        S = (64, 128, 32)[k % 3]
+        C.cudanp_batched_loop_scan(dA[k], None, Ad, S=8, map=C.INTRA_WARP)      # writes A
+        C.cudanp_batched_loop_reduce(dx[k], None, xd, S=4, map=C.INTRA_WARP)    # writes x
+        C.cudanp_tmv(Ad, xd, ys[k], S=S, dist=C.BLOCK if k % 2 else C.CYCLIC, map=C.INTER_WARP)
+    for k in range(rounds):
+        ref = O.tmv(O.scan(srcA[k]), O.reduce(srcx[k]))
+        assert_rel(host(ys[k]), ref, h, f"round {k}")
+
+
 # ------------------------------------------------------------------ TMA-staged reduce
 def test_reduce_tma_parity_and_identity_with_ldg():
     # same per-lane order as the LDG intra-warp kernel -> bit-identical even on

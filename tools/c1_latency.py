@@ -89,6 +89,13 @@ def main():
                        for i in range(copies)])
         emit({"impl": "np", "S": S, "dist": "cyclic", "map": "intra", "us": round(us, 3),
               "gbs": round(nb / us / 1e3, 1)})
+    # tuned S = 1 (no nesting): the LDG kernel of each map and the TMA-staged one
+    for m, name in ((C.INTER_WARP, "inter"), (C.INTRA_WARP, "intra"), (C.INTER_WARP_TMA, "inter_tma")):
+        us = graph_us([lambda i=i: C.cudanp_tmv(As[i], x, ys[i], S=1, dist=C.CYCLIC, map=m)
+                       for i in range(copies)])
+        emit({"impl": "s1_tuned", "S": 1, "map": name, "us": round(us, 3), "gbs": round(nb / us / 1e3, 1)})
+    us = graph_us([lambda i=i: C.cudanp_tmv(As[i], x, ys[i]) for i in range(copies)])
+    emit({"impl": "auto", "us": round(us, 3), "gbs": round(nb / us / 1e3, 1)})
     us = graph_us([lambda i=i: C.cudanp_tmv_variant(C.S1_LITERAL, As[i], x, ys[i]) for i in range(copies)])
     emit({"impl": "s1_literal", "us": round(us, 3), "gbs": round(nb / us / 1e3, 1)})
 
