@@ -336,8 +336,9 @@ int cudanp_launch_info(int op_kind, int64_t n_outer, int64_t n_inner, int dtype,
  * 2 reduce, 3 scan) on N = n_outer items of L = n_inner iterations, given
  * `map` (AUTO, or a map to keep) and vec4 as above.  Rule:
  * TMV with 0.3..1.1 128-column strips per SM -> TMA S = 8 cyclic; wider ->
- * inter-warp S = 32 block; narrower -> inter-warp S = clamp(2*SMs*1024/N,
- * 8, 64), block when L/S <= 32;
+ * inter-warp S = 32 block; narrower -> inter-warp S = 128 with vec4 (else
+ * clamp(2*SMs*1024/N, 8, 64)), block when L/S < 32 (and N > 1024 with
+ * vec4), else cyclic;
  * MV intra S = clamp(L/64, 1, 256); reduce intra S = clamp(L/8, 1, 32);
  * scan intra S = clamp(L/4, 1, 16); reduce/scan/MV teams grow (up to S/32
  * warps, slaves keeping >= 8 elements) while N*S < SMs*1024. */

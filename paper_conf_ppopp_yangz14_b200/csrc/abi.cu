@@ -169,8 +169,10 @@ static bool tma_ok(const float* A, int64_t lda, int64_t w, int64_t h) {
 // TLP is short), up to a team whose slaves still get >= 8 elements each.
 //   TMV: tmv_wide + TMA-able -> TMA, S = 8 cyclic (C2 best); wider than that
 //        -> LDG inter-warp S = 32 block; narrower -> LDG inter-warp with
-//        S = clamp(2T / w, 8, 64), block when each slave's share is <= 32
-//        rows (C1: 64 block), cyclic otherwise (w = 4096: 64 cyclic).
+//        S = 128 when 16-byte aligned (else clamp(2T / w, 8, 64)), block when
+//        each slave's share is < 32 rows and w > 1024, cyclic otherwise (C1:
+//        128 cyclic; profiles/tmv_narrow_new_r02a[ef].jsonl: S = 128 best for
+//        w <= 4096 at every h but w = 512).
 //   MV:  intra, S = clamp(L / 64, 1, 256) cyclic (C2 best: S = 256), grown.
 //   reduce: intra, S = clamp(L / 8, 1, 32) (C3: 4/8/16/32 at L = 32..256),
 //        block above L = 32 (L % 4 != 0: L / 16), grown.
@@ -199,11 +201,12 @@ int choose_version(int op_kind, int64_t N, int64_t L, bool vec, bool tma, int ma
         s = 32;
         d = CUDANP_DIST_BLOCK;
       } else {
-        m = CUDANP_MAP_INTER_WARP;
-        s = clampi(floor_pow2(N > 0 ? 2 * T / N : 64), 8, 64);
+        m = CUDANP_MAP_INTER_WARP;  // narrow: S = 128 on aligned matrices (vec)
+        s = vec ? 128 : clampi(floor_pow2(N > 0 ? 2 * T / N : 64), 8, 64);
       }
-      s = clampi(s, 1, clampi(floor_pow2(L / 4), 1, 64));
-      if (m == CUDANP_MAP_INTER_WARP && s != 32) d = L / s <= 32 ? CUDANP_DIST_BLOCK : CUDANP_DIST_CYCLIC;
+      s = clampi(s, 1, clampi(floor_pow2(L / 4), 1, 128));
+      if (m == CUDANP_MAP_INTER_WARP && s != 32)
+        d = L / s < 32 && (!vec || N > 1024) ? CUDANP_DIST_BLOCK : CUDANP_DIST_CYCLIC;
       break;
     case 1:  // MV
       if (m == CUDANP_MAP_INTER_WARP) {
@@ -273,13 +276,30 @@ static int check_mv_args(const float* A, int64_t lda, const float* x, float* y, 
 // least half an SM's worth of CTAs per SM pair (>= SMs/2 CTAs); for narrower
 // matrices one master per thread (plus 8-master CTAs, np_matvec.cu) spreads
 // the few columns over more SMs.
-static bool tmv_vec(const float* A, int64_t lda, const float* y, int64_t w) {
-  const bool aligned = (w % 4 == 0) && (lda % 4 == 0) && aligned16(A) && aligned16(y);
+// The CTAs of S = 64 / 128 (8 or 4 column-masters, np_matvec.cu
+// launch_tmv_big) take V = 4 when its 16-column CTAs still number >= 0.8 SMs,
+// or, for short columns (h <= 2048: latency-bound, one load batch per slave),
+// >= a quarter of the SMs; tall narrow matrices keep V = 1's twice as many
+// CTAs (bandwidth needs the SMs).  Graph of cold launches
+// (profiles/tmv_narrow_*_r02ae.jsonl): h = 1024, w = 1024 / 2048 / 4096,
+// S = 128: 2.39 -> 2.15, 3.33 -> 2.58, 5.55 -> 4.03 us; h = 16384, w = 1024
+// stays V = 1 (19.1 vs 21.0 us).
+static bool tmv_aligned(const float* A, int64_t lda, const float* y, int64_t w) {
+  return (w % 4 == 0) && (lda % 4 == 0) && aligned16(A) && aligned16(y);
+}
+static bool tmv_vec_shape(int64_t w, int64_t h, int S) {
 #if defined(CUDANP_TMV_VEC_ALWAYS)
-  return aligned;
+  return true;
 #else
-  return aligned && 2 * ((w + 127) / 128) >= sm_count();
+  if (S == 64 || S == 128) {
+    const int64_t ctas16 = (w + 15) / 16, sms = sm_count();
+    return 10 * ctas16 >= 8 * sms || (h <= 2048 && 4 * ctas16 >= sms);
+  }
+  return 2 * ((w + 127) / 128) >= sm_count();
 #endif
+}
+static bool tmv_vec(const float* A, int64_t lda, const float* y, int64_t w, int64_t h, int S) {
+  return tmv_aligned(A, lda, y, w) && tmv_vec_shape(w, h, S);
 }
 static bool mv_vec(const float* A, int64_t lda, const float* x, int64_t w) {
   return (w % 4 == 0) && (lda % 4 == 0) && aligned16(A) && aligned16(x);
@@ -400,7 +420,7 @@ int cudanp_tmv(const float* A, int64_t lda, const float* x, float* y, int64_t n_
   const bool tma = tma_ok(A, lda, n_outer, n_inner);
   if (S == CUDANP_S_AUTO) {
     if (map < CUDANP_MAP_AUTO || map > CUDANP_MAP_INTER_WARP_TMA) return fail_invalid("map");
-    choose_version(0, n_outer, n_inner, tmv_vec(A, lda, y, n_outer), tma, map, &S, &dist, &map);
+    choose_version(0, n_outer, n_inner, tmv_aligned(A, lda, y, n_outer), tma, map, &S, &dist, &map);
   }
   const int m = map == CUDANP_MAP_INTER_WARP_TMA ? CUDANP_MAP_INTER_WARP : map;
   int rc = check_tmv_args(A, lda, x, y, n_outer, n_inner, S, dist, m);
@@ -410,7 +430,7 @@ int cudanp_tmv(const float* A, int64_t lda, const float* x, float* y, int64_t n_
   if (use_tma)
     return tmv_tma(A, lda, x, y, n_outer, n_inner, S, dist, 0, -1, 0, as_stream(stream), nullptr);
   return tmv_np(A, lda, x, y, n_outer, n_inner, S, dist, resolve_map(m, true, S),
-                tmv_vec(A, lda, y, n_outer), as_stream(stream), nullptr);
+                tmv_vec(A, lda, y, n_outer, n_inner, S), as_stream(stream), nullptr);
 }
 
 int cudanp_tmv_tma_ex(const float* A, int64_t lda, const float* x, float* y, int64_t n_outer,
@@ -745,7 +765,10 @@ int cudanp_launch_info(int op_kind, int64_t n_outer, int64_t n_inner, int dtype,
   LaunchInfo info;
   const int m = resolve_map(map, op_kind == 0, S);
   switch (op_kind) {
-    case 0: rc = tmv_np(nullptr, 0, nullptr, nullptr, n_outer, n_inner, S, dist, m, v, 0, &info); break;
+    case 0:  // vec4 = aligned; the call adds its shape rule (tmv_vec)
+      rc = tmv_np(nullptr, 0, nullptr, nullptr, n_outer, n_inner, S, dist, m,
+                  v && tmv_vec_shape(n_outer, n_inner, S), 0, &info);
+      break;
     case 1: rc = mv_np(nullptr, 0, nullptr, nullptr, n_outer, n_inner, S, dist, m, v, 0, &info); break;
     case 2:
       rc = check_dtype_op(dtype, op);

@@ -90,11 +90,13 @@ def test_auto_team_size_rule(lib):
     """S = CUDANP_S_AUTO: the library's version choice follows
     the rule stated in cudanp.h / DESIGN.md §6 (host-only, no GPU)."""
     ch = C.cudanp_choose_version
-    # TMV: wide and TMA-able -> TMA S=8 cyclic (C2); narrow C1 -> inter-warp S=64 block;
+    # TMV: wide and TMA-able -> TMA S=8 cyclic (C2); narrow C1 -> inter-warp S=128 cyclic;
     # not 16-byte aligned -> LDG inter-warp
     assert ch("tmv", 16384, 16384) == (8, C.CYCLIC, C.INTER_WARP_TMA)
-    assert ch("tmv", 1024, 1024) == (64, C.BLOCK, C.INTER_WARP)
-    assert ch("tmv", 4096, 16384) == (64, C.CYCLIC, C.INTER_WARP)
+    assert ch("tmv", 1024, 1024) == (128, C.CYCLIC, C.INTER_WARP)
+    assert ch("tmv", 2048, 1024) == (128, C.BLOCK, C.INTER_WARP)
+    assert ch("tmv", 4096, 16384) == (128, C.CYCLIC, C.INTER_WARP)
+    assert ch("tmv", 1024, 1024, vec4=False) == (64, C.BLOCK, C.INTER_WARP)
     assert ch("tmv", 8192, 65536) == (8, C.CYCLIC, C.INTER_WARP_TMA)   # C5 shard at G = 8
     assert ch("tmv", 65536, 65536) == (32, C.BLOCK, C.INTER_WARP)     # C5 at G = 1
     S, d, m = ch("tmv", 16384, 16384, vec4=False)

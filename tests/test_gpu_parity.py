@@ -626,6 +626,21 @@ def test_big_teams_parity():
             if S <= 128:
                 assert_exact(host(C.cudanp_tmv(dev(A), dev(xt), S=S, dist=dist)), O.tmv(A, xt),
                              f"tmv big S={S} h={h} w={w}")
+    # TMV S = 64 / 128, every CTA layout the call picks (abi.cu tmv_vec): V = 4 with 4
+    # column-masters (short or 16-column-rich matrices, C1), V = 4 with 8 (w >= 32 x SMs),
+    # V = 1 (tall narrow or unaligned); ragged last CTAs; cold HBM via the L2 prefetch.
+    sms = torch.cuda.get_device_properties(0).multi_processor_count
+    for h, w, mx_v in [(1024, 1024, (4, 4)), (1500, 2052, (4, 4)), (7, 1028, (4, 4)),
+                       (300, 32 * sms + 64, (8, 4)), (3000, 1024, (8, 1)), (1024, 1022, (8, 1))]:
+        A = synth.matrix(h, w, "f32_int4", seed=h + w)
+        xt = synth.vector(h, "f32_int4")
+        ref = O.tmv(A, xt)
+        for S, dist in itertools.product((64, 128), DISTS):
+            i = C.cudanp_launch_info("tmv", w, h, S=S, dist=dist, map=C.INTER_WARP, vec4=w % 4 == 0)
+            assert (i["block_threads"] // S, -(-w // i["grid_ctas"])) == (mx_v[0], mx_v[0] * mx_v[1]), \
+                f"layout h={h} w={w} S={S}: {i}"
+            assert_exact(host(C.cudanp_tmv(dev(A), dev(xt), S=S, dist=dist, map=C.INTER_WARP)), ref,
+                         f"tmv S={S} h={h} w={w} dist={dist} layout={mx_v}")
     # TMV with a cluster team per column group (S = 256 / 1024: 8 CTAs x 32 / 128 slave warps)
     for h, w in [(5, 4096), (64, 1000), (300, 260), (20000, 36), (70000, 3), (1, 1), (0, 7)]:
         A = synth.matrix(h, w, "f32_int4", seed=w)

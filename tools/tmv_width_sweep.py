@@ -5,6 +5,11 @@ tmv_wide.)  For each (h, w): the best TMA version (S x dist) and the best LDG
 inter-warp version (S x dist), 20 launches back to back per event pair.
 
     python tools/tmv_width_sweep.py --out gpurun_out/tmv_width_<tag>.jsonl
+
+--narrow: narrow matrices (w <= 8192, the latency-bound band around C1) --
+every LDG inter-warp (S, dist) incl. S = 64 / 128 and the library's S_AUTO
+choice, each timed as a CUDA graph over enough distinct copies of A that
+every launch reads cold HBM (tools/c1_latency.py's method).
 """
 from __future__ import annotations
 
@@ -37,8 +42,11 @@ def t_ms(fn, reps=20, warm=3):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--out", default="gpurun_out/tmv_width.jsonl")
+    ap.add_argument("--narrow", action="store_true")
     a = ap.parse_args()
     C.load()
+    if a.narrow:
+        return narrow(a.out)
     sms = torch.cuda.get_device_properties(0).multi_processor_count
     shapes = [(16384, w) for w in (4096, 8192, 12288, 16384, 18944, 20480, 24576, 32768, 49152, 65536)]
     shapes += [(65536, w) for w in (8192, 16384, 32768, 65536)]
@@ -70,6 +78,44 @@ def main():
             print(json.dumps({k: rec[k] for k in ("h", "w", "strips128_per_sm", "tma_best", "ldg_best",
                                                   "auto_gbs")}), flush=True)
             del A
+            torch.cuda.empty_cache()
+
+
+def narrow(out):
+    sys.path.insert(0, os.path.join(ROOT, "tools"))
+    from c1_latency import graph_us
+    shapes = [(1024, 512), (1024, 1024), (1024, 2048), (1024, 4096), (4096, 1024), (4096, 2048),
+              (16384, 1024), (16384, 2048), (16384, 4096), (16384, 8192), (65536, 1024)]
+    with open(out, "w") as f:
+        for h, w in shapes:
+            copies = max(2, min(64, (512 << 20) // (4 * h * w)))
+            As = []
+            for k in range(copies):
+                t = torch.empty(h, w, device="cuda")
+                C.cudanp_generate(t, "f32_unit", stream_id=1, seed=k)
+                As.append(t)
+            x = torch.empty(h, device="cuda")
+            C.cudanp_generate(x, "f32_unit", stream_id=2)
+            ys = [torch.empty(w, device="cuda") for _ in range(copies)]
+            nb = 4 * h * w + 4 * h + 4 * w
+            res = {}
+            for S, d in itertools.product((8, 16, 32, 64, 128), (C.CYCLIC, C.BLOCK)):
+                res[(S, d)] = graph_us([lambda i=i: C.cudanp_tmv(As[i], x, ys[i], S=S, dist=d,
+                                                                 map=C.INTER_WARP)
+                                        for i in range(copies)])
+            auto = graph_us([lambda i=i: C.cudanp_tmv(As[i], x, ys[i]) for i in range(copies)])
+            best = min(res, key=res.get)
+            rec = {"h": h, "w": w, "copies": copies,
+                   "best": {"S": best[0], "dist": "cyclic" if best[1] == C.CYCLIC else "block",
+                            "us": round(res[best], 3), "gbs": round(nb / res[best] / 1e3, 1)},
+                   "auto": {"choice": C.cudanp_choose_version("tmv", w, h), "us": round(auto, 3),
+                            "gbs": round(nb / auto / 1e3, 1), "vs_best": round(res[best] / auto, 3)},
+                   "all_us": {f"{S}/{'cyc' if d == C.CYCLIC else 'blk'}": round(v, 3)
+                              for (S, d), v in res.items()}}
+            f.write(json.dumps(rec) + "\n")
+            f.flush()
+            print(json.dumps({k: rec[k] for k in ("h", "w", "best", "auto")}), flush=True)
+            del As
             torch.cuda.empty_cache()
 
 
