@@ -77,6 +77,13 @@ def main():
             C.cudanp_batched_loop_scan(Xc, None, S=S, dist=d)
             C.cudanp_batched_loop_scan(Xcf, None, S=S, dist=d)
         C.cudanp_mv(A, xm, S=S, dist=C.CYCLIC)
+    # narrow TMV S = 64 / 128 in each CTA layout (V = 4 with 4 / 8 masters, V = 1), ragged
+    # last CTA, with the L2 bulk prefetch before the dependency wait
+    for h, w in ((1024, 1028), (300, 4800), (3000, 1024), (64, 1022)):
+        An, xn = dev(synth.matrix(h, w, "f32_unit")), dev(synth.vector(h))
+        for S in (64, 128):
+            for d in (C.CYCLIC, C.BLOCK):
+                C.cudanp_tmv(An, xn, S=S, dist=d, map=C.INTER_WARP)
     for S in (256, 1024):  # TMV cluster teams
         for d in (C.CYCLIC, C.BLOCK):
             C.cudanp_tmv(A, xt, S=S, dist=d, map=C.INTER_WARP, n_outer=70)
