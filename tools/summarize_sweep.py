@@ -75,6 +75,12 @@ def main(path, out=None):
         lines += [f"| {r['config']} | {r['op']}{(' ' + r['opname']) if r.get('opname') else ''} | {r['dtype']} | "
                   f"{r['L']} | {r['S']} | {r['dist']} | {r['gbs']:.0f} | {r['S_padded']} | {r['gbs_padded']:.0f} | "
                   f"{r['speedup_vs_padded']:.2f}x |" for r in f12]
+    rv = [r for r in recs if r["config"] == "R1" and str(r["impl"]).startswith(("adaptive", "streamed"))]
+    if rv:
+        lines += ["", "R1 — ragged versions beside the swept NP kernels (GB/s; x = time of the best NP / its time)", "",
+                  "| L | impl | GB/s | % HBM | vs best NP |", "|---|---|---|---|---|"]
+        lines += [f"| {r['L']} | {r['impl']} | {r['gbs']:.0f} | {100 * r['gbs'] / PEAK:.1f} | "
+                  f"{1 / r['speedup_of_best_np']:.2f}x |" for r in rv]
     f3 = [r for r in special if r["config"] == "F3"]
     if f3:
         lines += ["", "F3 — Fig 1 memcopy (64M floats): impl, m parents x n children, GB/s", "",
