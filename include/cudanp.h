@@ -208,19 +208,6 @@ int cudanp_ragged_loop_reduce(const void* in, const int64_t* offsets, const void
 int cudanp_ragged_loop_reduce_adaptive(const void* in, const int64_t* offsets, const void* init,
                                        void* out, int64_t n_outer, int dtype, int op,
                                        int64_t threshold, void* stream);
-/* Ragged reduce for many short segments (the regime where nesting does not
- * pay): each lane is still the master of one segment and reads
- * its bounds, but the warp streams its 32 segments' contiguous span
- * with 128-bit loads (512 contiguous bytes per warp instruction) and takes
- * every segment's total from one segmented inclusive scan over the span
- * (P:209's scan primitive over head flags); each master stores its own
- * (P:327).  A tile of 32 segments whose span exceeds 1024 elements, or whose
- * bounds are not monotone, runs the adaptive path with `threshold` instead.
- * Same result contract as cudanp_ragged_loop_reduce (fp32 sums in another
- * association order); threshold >= 1, else CUDANP_ERR_INVALID. */
-int cudanp_ragged_loop_reduce_streamed(const void* in, const int64_t* offsets, const void* init,
-                                       void* out, int64_t n_outer, int dtype, int op,
-                                       int64_t threshold, void* stream);
 /* Comparison: one thread per segment, serial loop (Fig 2 style). */
 int cudanp_ragged_loop_reduce_literal(const void* in, const int64_t* offsets, const void* init,
                                       void* out, int64_t n_outer, int dtype, int op, void* stream);

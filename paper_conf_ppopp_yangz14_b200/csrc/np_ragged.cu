@@ -289,86 +289,6 @@ static int launch_ragged_multi(const T* in, const int64_t* off, const T* init, T
 // turns (ballot of the long ones, bounds broadcast by shfl from their
 // master), with a butterfly team reduction; the master stores
 // (P:327).  Every segment is still reduced by exactly one team.
-// One warp step over K tiles of 32 segments whose bounds each lane's master
-// has read (b, len): part[k] = the fold of lane's segment of tile k.
-template <class T, class Op, int K>
-__device__ __forceinline__ void adaptive_tiles(const T* __restrict__ in, const int64_t (&b)[K],
-                                               const int64_t (&len)[K], int64_t thresh, int lane,
-                                               T (&part)[K]) {
-  const T id = Op::template identity<T>();
-  // short segments: each master alone (a team of one); all K items' loads in flight
-  {
-    const T* p[K];
-    int cnt[K];
-    int64_t stp[K];
-    int trips = 0;
-#pragma unroll
-    for (int k = 0; k < K; ++k) {
-      const int64_t ls = len[k] >= thresh ? 0 : len[k];
-      const SegShare<T, 1, DIST_CYCLIC> sh(in, b[k], ls, 0);
-      p[k] = sh.body; cnt[k] = sh.cnt; stp[k] = sh.step;
-      trips = max(trips, sh.cnt);
-      T hv[3], tv[3];
-      const T* tl = in + b[k] + sh.head + 4 * ((ls - sh.head) >> 2);
-#pragma unroll
-      for (int j = 0; j < 3; ++j) {
-        hv[j] = j < sh.head ? ldg1(in + b[k] + j) : id;
-        tv[j] = j < sh.tail ? ldg1(tl + j) : id;
-      }
-      part[k] = Op::apply(Op::apply(Op::apply(hv[0], hv[1]), hv[2]), Op::apply(Op::apply(tv[0], tv[1]), tv[2]));
-    }
-    V4<T> acc[K];
-#pragma unroll
-    for (int k = 0; k < K; ++k) acc[k] = {id, id, id, id};
-#pragma unroll 2
-    for (int j = 0; j < trips; ++j) {
-      V4<T> v[K];
-#pragma unroll
-      for (int k = 0; k < K; ++k) {
-        v[k] = j < cnt[k] ? ldg4(p[k]) : V4<T>{id, id, id, id};
-        p[k] += stp[k];
-      }
-#pragma unroll
-      for (int k = 0; k < K; ++k) acc[k] = op4r<T, Op>(acc[k], v[k]);
-    }
-#pragma unroll
-    for (int k = 0; k < K; ++k)
-      part[k] = Op::apply(part[k], Op::apply(Op::apply(acc[k].x, acc[k].y), Op::apply(acc[k].z, acc[k].w)));
-  }
-  // long segments: the whole warp as one team, masters taking turns
-#pragma unroll
-  for (int k = 0; k < K; ++k) {
-    unsigned m = __ballot_sync(kFull, len[k] >= thresh);
-    while (m) {
-      const int src = __ffs(m) - 1;
-      m &= m - 1;
-      const int64_t bb = __shfl_sync(kFull, b[k], src);   // read_from_master
-      const int64_t ll = __shfl_sync(kFull, len[k], src);
-      const SegShare<T, 32, DIST_CYCLIC> sh(in, bb, ll, lane);
-      T pv = id;
-      if (lane < sh.head) pv = Op::apply(pv, ldg1(in + bb + lane));
-      const T* tl = in + bb + sh.head + 4 * ((ll - sh.head) >> 2);
-      if (lane < sh.tail) pv = Op::apply(pv, ldg1(tl + lane));
-      V4<T> acc[4] = {{id, id, id, id}, {id, id, id, id}, {id, id, id, id}, {id, id, id, id}};
-      const T* p = sh.body;
-      int c = 0;
-      for (; c + 3 < sh.cnt; c += 4, p += 4 * sh.step) {
-        V4<T> v[4];
-#pragma unroll
-        for (int j = 0; j < 4; ++j) v[j] = ldg4(p + j * sh.step);
-#pragma unroll
-        for (int j = 0; j < 4; ++j) acc[j] = op4r<T, Op>(acc[j], v[j]);
-      }
-      for (; c < sh.cnt; ++c, p += sh.step) acc[0] = op4r<T, Op>(acc[0], ldg4(p));
-      const V4<T> a4 = op4r<T, Op>(op4r<T, Op>(acc[0], acc[1]), op4r<T, Op>(acc[2], acc[3]));
-      pv = Op::apply(pv, Op::apply(Op::apply(a4.x, a4.y), Op::apply(a4.z, a4.w)));
-#pragma unroll
-      for (int o = 16; o > 0; o >>= 1) pv = Op::apply(pv, __shfl_xor_sync(kFull, pv, o));
-      if (lane == src) part[k] = pv;
-    }
-  }
-}
-
 template <class T, class Op>
 __global__ void __launch_bounds__(kRaggedBlock)
 ragged_adaptive_kernel(const T* __restrict__ in, const int64_t* __restrict__ off,
@@ -379,6 +299,7 @@ ragged_adaptive_kernel(const T* __restrict__ in, const int64_t* __restrict__ off
   const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
   const int64_t ntiles = (N + 31) / 32;
+  const T id = Op::template identity<T>();
   for (int64_t t0 = warp * K; t0 < ntiles; t0 += nwarps * K) {
     int64_t item[K], b[K], len[K];
 #pragma unroll
@@ -392,10 +313,78 @@ ragged_adaptive_kernel(const T* __restrict__ in, const int64_t* __restrict__ off
       }
     }
     T part[K];
-    adaptive_tiles<T, Op, K>(in, b, len, thresh, lane, part);
+    // short segments: each master alone (a team of one); all K items' loads in flight
+    {
+      const T* p[K];
+      int cnt[K];
+      int64_t stp[K];
+      int trips = 0;
 #pragma unroll
-    for (int k = 0; k < K; ++k)
+      for (int k = 0; k < K; ++k) {
+        const int64_t ls = len[k] >= thresh ? 0 : len[k];
+        const SegShare<T, 1, DIST_CYCLIC> sh(in, b[k], ls, 0);
+        p[k] = sh.body; cnt[k] = sh.cnt; stp[k] = sh.step;
+        trips = max(trips, sh.cnt);
+        T hv[3], tv[3];
+        const T* tl = in + b[k] + sh.head + 4 * ((ls - sh.head) >> 2);
+#pragma unroll
+        for (int j = 0; j < 3; ++j) {
+          hv[j] = j < sh.head ? ldg1(in + b[k] + j) : id;
+          tv[j] = j < sh.tail ? ldg1(tl + j) : id;
+        }
+        part[k] = Op::apply(Op::apply(Op::apply(hv[0], hv[1]), hv[2]), Op::apply(Op::apply(tv[0], tv[1]), tv[2]));
+      }
+      V4<T> acc[K];
+#pragma unroll
+      for (int k = 0; k < K; ++k) acc[k] = {id, id, id, id};
+#pragma unroll 2
+      for (int j = 0; j < trips; ++j) {
+        V4<T> v[K];
+#pragma unroll
+        for (int k = 0; k < K; ++k) {
+          v[k] = j < cnt[k] ? ldg4(p[k]) : V4<T>{id, id, id, id};
+          p[k] += stp[k];
+        }
+#pragma unroll
+        for (int k = 0; k < K; ++k) acc[k] = op4r<T, Op>(acc[k], v[k]);
+      }
+#pragma unroll
+      for (int k = 0; k < K; ++k)
+        part[k] = Op::apply(part[k], Op::apply(Op::apply(acc[k].x, acc[k].y), Op::apply(acc[k].z, acc[k].w)));
+    }
+    // long segments: the whole warp as one team, masters taking turns
+#pragma unroll
+    for (int k = 0; k < K; ++k) {
+      unsigned m = __ballot_sync(kFull, len[k] >= thresh);
+      while (m) {
+        const int src = __ffs(m) - 1;
+        m &= m - 1;
+        const int64_t bb = __shfl_sync(kFull, b[k], src);   // read_from_master
+        const int64_t ll = __shfl_sync(kFull, len[k], src);
+        const SegShare<T, 32, DIST_CYCLIC> sh(in, bb, ll, lane);
+        T pv = id;
+        if (lane < sh.head) pv = Op::apply(pv, ldg1(in + bb + lane));
+        const T* tl = in + bb + sh.head + 4 * ((ll - sh.head) >> 2);
+        if (lane < sh.tail) pv = Op::apply(pv, ldg1(tl + lane));
+        V4<T> acc[4] = {{id, id, id, id}, {id, id, id, id}, {id, id, id, id}, {id, id, id, id}};
+        const T* p = sh.body;
+        int c = 0;
+        for (; c + 3 < sh.cnt; c += 4, p += 4 * sh.step) {
+          V4<T> v[4];
+#pragma unroll
+          for (int j = 0; j < 4; ++j) v[j] = ldg4(p + j * sh.step);
+#pragma unroll
+          for (int j = 0; j < 4; ++j) acc[j] = op4r<T, Op>(acc[j], v[j]);
+        }
+        for (; c < sh.cnt; ++c, p += sh.step) acc[0] = op4r<T, Op>(acc[0], ldg4(p));
+        const V4<T> a4 = op4r<T, Op>(op4r<T, Op>(acc[0], acc[1]), op4r<T, Op>(acc[2], acc[3]));
+        pv = Op::apply(pv, Op::apply(Op::apply(a4.x, a4.y), Op::apply(a4.z, a4.w)));
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) pv = Op::apply(pv, __shfl_xor_sync(kFull, pv, o));
+        if (lane == src) part[k] = pv;
+      }
       if (item[k] < N) out[item[k]] = init ? Op::apply(init[item[k]], part[k]) : part[k];
+    }
   }
 }
 
@@ -418,149 +407,6 @@ int ragged_adaptive(const void* in, const int64_t* off, const void* init, void* 
   return op == CUDANP_SUM
              ? launch_ragged_adaptive<int32_t, OpSum>((const int32_t*)in, off, (const int32_t*)init, (int32_t*)out, N, thresh, st)
              : launch_ragged_adaptive<int32_t, OpMax>((const int32_t*)in, off, (const int32_t*)init, (int32_t*)out, N, thresh, st);
-}
-
-// ---------------------------------------------------------------- warp-streamed short segments
-// Millions of short segments are the regime where nesting does not pay
-// (P:84): a master's loop is a handful of iterations, and a lane that
-// walks its own segment touches a different 128-byte line on every load (32
-// lines per warp instruction).  Here the 32 masters of a warp keep their
-// sequential sections -- each reads its two bounds -- but stream the
-// tile's CSR span [off[t*32], off[t*32+32]) together: lane l holds elements
-// 8l..8l+7 of each 256-element row (two 128-bit loads, a warp instruction
-// covers 512 contiguous bytes), every row's loads in flight at once.  The
-// segment totals come out of one segmented inclusive scan (P:209's scan
-// primitive, restated over heads): an 8-element scan in registers, a shfl
-// scan of the lanes' aggregates over head flags, the carry between rows; each
-// lane writes the scan value at the tails inside its 8 elements to shared
-// memory, and each master reads its own segment's total at its tail and
-// stores.  Head and tail flags are bitmaps built by the masters from
-// their bounds.  A tile whose span exceeds kStreamCap elements (long
-// segments), or whose bounds are not monotone, runs the adaptive path above.
-constexpr int kStreamCap = 1024;
-template <class T, class Op>
-__global__ void __launch_bounds__(kRaggedBlock, 3)
-ragged_streamed_kernel(const T* __restrict__ in, const int64_t* __restrict__ off,
-                       const T* __restrict__ init, T* __restrict__ out, int64_t N, int64_t thresh) {
-  pdl_entry();
-  constexpr int NW = kRaggedBlock / 32, WORDS = kStreamCap / 32, ROWS = kStreamCap / 256;
-  static_assert(WORDS == 32, "one flag word per lane");
-  __shared__ uint32_t hflag[NW][WORDS], tflag[NW][WORDS];
-  __shared__ T tot[NW][kStreamCap];
-  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-  uint32_t* hf = hflag[wid];
-  uint32_t* tf = tflag[wid];
-  T* tt = tot[wid];
-  const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
-  const int64_t ntiles = (N + 31) / 32;
-  const T id = Op::template identity<T>();
-  for (int64_t t = warp; t < ntiles; t += nwarps) {
-    const int64_t item = t * 32 + lane;
-    int64_t b = 0, e = 0;
-    if (item < N) {  // the master's sequential section: its loop bounds
-      b = off[item];
-      e = off[item + 1];
-    }
-    const int last = (int)(N - 1 - t * 32 < 31 ? N - 1 - t * 32 : 31);
-    const int64_t B = __shfl_sync(kFull, b, 0), E = __shfl_sync(kFull, e, last);
-    const bool mono = __all_sync(kFull, item >= N || e >= b);
-    const int mis = (int)((reinterpret_cast<uintptr_t>(in + B) >> 2) & 3);
-    const int64_t B0 = B - mis;  // 16-byte aligned element; [B0, B) is not read
-    T part = id;
-    if (mono && E - B0 <= kStreamCap) {
-      const int span = (int)(E - B0), nrows = (span + 255) >> 8;
-      hf[lane] = 0u;
-      tf[lane] = 0u;
-      V4<T> v[ROWS][2];
-#pragma unroll
-      for (int r = 0; r < ROWS; ++r) {
-#pragma unroll
-        for (int h = 0; h < 2; ++h) {
-          const int p = 256 * r + 8 * lane + 4 * h;
-          if (r < nrows && p >= mis && p + 4 <= span) {
-            v[r][h] = ldg4(in + B0 + p);
-          } else {
-            T u[4];
-#pragma unroll
-            for (int j = 0; j < 4; ++j)
-              u[j] = (r < nrows && p + j >= mis && p + j < span) ? ldg1(in + B0 + p + j) : id;
-            v[r][h] = {u[0], u[1], u[2], u[3]};
-          }
-        }
-      }
-      __syncwarp();
-      if (e > b) {  // lanes past N have b = e = 0
-        const int hp = (int)(b - B0), tp = (int)(e - 1 - B0);
-        atomicOr(&hf[hp >> 5], 1u << (hp & 31));
-        atomicOr(&tf[tp >> 5], 1u << (tp & 31));
-      }
-      __syncwarp();
-      T carry = id;
-#pragma unroll
-      for (int r = 0; r < ROWS; ++r) {
-        if (r < nrows) {
-          const int sh = 8 * (lane & 3);
-          const uint32_t hb = (hf[8 * r + (lane >> 2)] >> sh) & 0xffu;
-          const uint32_t tb = (tf[8 * r + (lane >> 2)] >> sh) & 0xffu;
-          T x[8] = {v[r][0].x, v[r][0].y, v[r][0].z, v[r][0].w, v[r][1].x, v[r][1].y, v[r][1].z, v[r][1].w};
-#pragma unroll
-          for (int j = 1; j < 8; ++j)  // segmented inclusive scan of the lane's 8 elements
-            if (!((hb >> j) & 1u)) x[j] = Op::apply(x[j - 1], x[j]);
-          T a = x[7];
-          if (lane == 0 && hb == 0u) a = Op::apply(carry, a);
-          uint32_t f = hb != 0u;
-#pragma unroll
-          for (int o = 1; o < 32; o <<= 1) {  // segmented scan of the lanes' aggregates
-            const T au = __shfl_up_sync(kFull, a, o);
-            const uint32_t fu = __shfl_up_sync(kFull, f, o);
-            if (lane >= o) {
-              if (!f) a = Op::apply(au, a);
-              f |= fu;
-            }
-          }
-          T xp = __shfl_up_sync(kFull, a, 1);  // what flows into this lane's first elements
-          if (lane == 0) xp = carry;
-#pragma unroll
-          for (int j = 0; j < 8; ++j)  // elements before the lane's first head take it
-            if (!(hb & ((2u << j) - 1u))) x[j] = Op::apply(xp, x[j]);
-#pragma unroll
-          for (int j = 0; j < 8; ++j)
-            if ((tb >> j) & 1u) tt[256 * r + 8 * lane + j] = x[j];
-          carry = __shfl_sync(kFull, x[7], 31);
-        }
-      }
-      __syncwarp();
-      if (e > b) part = tt[e - 1 - B0];  // the master reads its segment's total
-    } else {
-      int64_t bb[1] = {b}, ll[1] = {e > b ? e - b : 0};
-      T pp[1];
-      adaptive_tiles<T, Op, 1>(in, bb, ll, thresh, lane, pp);
-      part = pp[0];
-    }
-    if (item < N) out[item] = init ? Op::apply(init[item], part) : part;
-  }
-}
-
-template <class T, class Op>
-static int launch_ragged_streamed(const T* in, const int64_t* off, const T* init, T* out, int64_t N,
-                                  int64_t thresh, cudaStream_t st) {
-  if (N == 0) return CUDANP_OK;
-  auto kern = ragged_streamed_kernel<T, Op>;
-  const int64_t grid = persistent_grid(kern, kRaggedBlock, 0, (N + kRaggedBlock - 1) / kRaggedBlock);
-  launch_pdl(kern, dim3((unsigned)grid), dim3(kRaggedBlock), 0, st, in, off, init, out, N, thresh);
-  return check_launch("ragged_loop_reduce (warp-streamed) launch");
-}
-
-int ragged_streamed(const void* in, const int64_t* off, const void* init, void* out, int64_t N,
-                    int dtype, int op, int64_t thresh, cudaStream_t st) {
-  if (dtype == CUDANP_F32)
-    return op == CUDANP_SUM
-               ? launch_ragged_streamed<float, OpSum>((const float*)in, off, (const float*)init, (float*)out, N, thresh, st)
-               : launch_ragged_streamed<float, OpMax>((const float*)in, off, (const float*)init, (float*)out, N, thresh, st);
-  return op == CUDANP_SUM
-             ? launch_ragged_streamed<int32_t, OpSum>((const int32_t*)in, off, (const int32_t*)init, (int32_t*)out, N, thresh, st)
-             : launch_ragged_streamed<int32_t, OpMax>((const int32_t*)in, off, (const int32_t*)init, (int32_t*)out, N, thresh, st);
 }
 
 // ---------------------------------------------------------------- S=1 literal

@@ -54,7 +54,6 @@ _SIGS = {
     "cudanp_ragged_loop_reduce": [_vp, _vp, _vp, _vp, _i64, _int, _int, _int, _int, _int, _vp],
     "cudanp_ragged_loop_reduce_literal": [_vp, _vp, _vp, _vp, _i64, _int, _int, _vp],
     "cudanp_ragged_loop_reduce_adaptive": [_vp, _vp, _vp, _vp, _i64, _int, _int, _i64, _vp],
-    "cudanp_ragged_loop_reduce_streamed": [_vp, _vp, _vp, _vp, _i64, _int, _int, _i64, _vp],
     "cudanp_le_gicov": [_vp, _vp, _vp, _vp, _vp, _i64, _i64, ctypes.c_float, _int, _int, _int,
                         _int, _vp],
     "cudanp_le_gicov_placement": [_vp, _vp, _vp, _vp, _vp, _i64, _i64, ctypes.c_float, _int, _int,
@@ -382,21 +381,6 @@ def cudanp_ragged_loop_reduce_adaptive(x, offsets, init=None, out=None, *, op=SU
     _check(load().cudanp_ragged_loop_reduce_adaptive(_ptr(x), _ptr(offsets), _ptr(init), _ptr(out), N,
                                                      _dtype_code(x), op, threshold, _stream(stream)),
            "cudanp_ragged_loop_reduce_adaptive")
-    return out
-
-
-def cudanp_ragged_loop_reduce_streamed(x, offsets, init=None, out=None, *, op=SUM, threshold=128,
-                                       stream=None):
-    """Ragged reduce for many short segments: the warp streams its 32
-    segments' span and takes every total from one segmented scan (tiles with
-    a span over 1024 elements run the adaptive path with `threshold`)."""
-    import torch
-    N = _ragged_args(x, offsets, init, out, "cudanp_ragged_loop_reduce_streamed")
-    if out is None:
-        out = torch.empty(N, dtype=x.dtype, device=x.device)
-    _check(load().cudanp_ragged_loop_reduce_streamed(_ptr(x), _ptr(offsets), _ptr(init), _ptr(out), N,
-                                                     _dtype_code(x), op, threshold, _stream(stream)),
-           "cudanp_ragged_loop_reduce_streamed")
     return out
 
 

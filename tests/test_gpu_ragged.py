@@ -125,57 +125,3 @@ def test_ragged_adaptive_parity(kind, op, exact):
     with pytest.raises(C.CudanpError):
         C.cudanp_ragged_loop_reduce_adaptive(dev(synth.gen(1, "i32_full", 0, 8)),
                                              dev(synth.offsets_from_lengths(np.array([3, 5]))), threshold=0)
-
-
-@pytest.mark.parametrize("kind,op,exact", [("i32_full", C.SUM, True), ("i32_full", C.MAX, True),
-                                           ("f32_signed", C.MAX, True), ("f32_int4", C.SUM, True),
-                                           ("f32_unit", C.SUM, False)])
-def test_ragged_streamed_parity(kind, op, exact):
-    """Warp-streamed short segments: the tile's span through 128-bit loads and a
-    segmented scan; spans over 1024 elements (long segments) and decreasing
-    bounds take the adaptive path.  Every alignment, base pointers off 16
-    bytes, empty segments, partial last tiles, multi-row spans."""
-    for N, mean, dist in CASES + [(3000, 90, "exp"), (40, 5000, "exp"), (5003, 16, "exp"),
-                                  (4096, 16, "uniform"), (2000, 1, "exp"), (999, 30, "uniform")]:
-        lens = synth.lengths(N, mean, dist, seed=N + mean + 1)
-        off = synth.offsets_from_lengths(lens)
-        for shift, base in ((0, 0), (1, 0), (3, 0), (0, 1), (2, 3)):
-            x = synth.gen(1, kind, 0, int(off[-1]) + 8)
-            offs = off + shift
-            ini = synth.init(N, kind)
-            ref_i = O.ragged_reduce(x[base:], offs, op=op, init=ini)
-            ref = O.ragged_reduce(x[base:], offs, op=op)
-            xd, od, inid = dev(x)[base:], dev(offs), dev(ini)
-            for th in (1, 64, 1 << 40):
-                what = f"streamed {kind} op={op} N={N} mean={mean} shift={shift} base={base} th={th}"
-                got_i = host(C.cudanp_ragged_loop_reduce_streamed(xd, od, inid, op=op, threshold=th))
-                got = host(C.cudanp_ragged_loop_reduce_streamed(xd, od, op=op, threshold=th))
-                if exact:
-                    assert_exact(got_i, ref_i, what)
-                    assert_exact(got, ref, what + " no init")
-                else:
-                    Lmax = int(lens.max()) if N else 1
-                    assert_rel(got_i, ref_i, Lmax, what)
-                    nz = lens > 0
-                    assert_rel(got[nz], ref[nz], Lmax, what + " no init")
-    x = dev(np.arange(8, dtype=np.int32))
-    off = dev(np.array([0, 5, 3, 8], np.int64))
-    assert host(C.cudanp_ragged_loop_reduce_streamed(x, off)).tolist() == [10, 0, 25]
-    with pytest.raises(C.CudanpError):
-        C.cudanp_ragged_loop_reduce_streamed(x, off, threshold=0)
-
-
-def test_ragged_streamed_full_size_sampled():
-    # the R1 sweep's shape: 2^22 segments of mean length 16 (exp), int32 -> bit-exact
-    N = 1 << 22
-    lens = synth.lengths(N, 16, "exp")
-    off = synth.offsets_from_lengths(lens)
-    x = torch.empty(int(off[-1]), dtype=torch.int32, device="cuda")
-    C.cudanp_generate(x, "i32_full", stream_id=1)
-    rng = np.random.default_rng(7)
-    items = np.unique(np.concatenate([rng.integers(0, N, 4096), [0, N - 1]]))
-    xs = O.gen_i32(1, "i32_full", 0, int(off[-1]))
-    got = host(C.cudanp_ragged_loop_reduce_streamed(x, dev(off)))
-    ref = np.array([O.ragged_reduce(xs[off[n]:off[n + 1]], np.array([0, lens[n]], np.int64))[0]
-                    for n in items], dtype=np.int32)
-    assert_exact(got[items], ref, "streamed full size")

@@ -20,7 +20,7 @@ def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--op", required=True, choices=["tmv", "mv", "reduce", "scan", "tmv_literal",
                                                     "mv_literal", "reduce_literal", "scan_literal",
-                                                    "ragged", "ragged_streamed", "ragged_adaptive", "le", "le_literal", "tmv_tma",
+                                                    "ragged", "le", "le_literal", "tmv_tma",
                                                     "mv_tiled", "tmv_tiled", "scan_tiled", "reduce_tiled"])
     ap.add_argument("--lens", default="uniform", help="ragged: length distribution")
     ap.add_argument("--layout", type=int, default=0, help="le: 0 item-major, 1 point-major")
@@ -37,15 +37,13 @@ def main():
     m = {"auto": C.AUTO, "intra": C.INTRA_WARP, "inter": C.INTER_WARP, "inter_tma": C.INTER_WARP_TMA,
          "intra_tma": C.INTRA_WARP_TMA}[a.map]
     C.load()
-    if a.op.startswith("ragged"):
+    if a.op == "ragged":
         import synth
         off = torch.from_numpy(synth.offsets_from_lengths(synth.lengths(a.N, a.L, a.lens))).cuda()
         X = torch.empty(int(off[-1].item()), device="cuda")
         C.cudanp_generate(X, "f32_unit")
         o1 = torch.empty(a.N, device="cuda")
-        fns = {"ragged": lambda: C.cudanp_ragged_loop_reduce(X, off, None, o1, S=a.S, dist=d, map=m),
-               "ragged_streamed": lambda: C.cudanp_ragged_loop_reduce_streamed(X, off, None, o1, threshold=64),
-               "ragged_adaptive": lambda: C.cudanp_ragged_loop_reduce_adaptive(X, off, None, o1, threshold=128)}
+        fns = {"ragged": lambda: C.cudanp_ragged_loop_reduce(X, off, None, o1, S=a.S, dist=d, map=m)}
     elif a.op in ("le", "le_literal"):
         X = torch.empty(*((a.N, a.L) if a.layout == 0 else (a.L, a.N)), device="cuda")
         C.cudanp_generate(X, "f32_unit")

@@ -58,14 +58,6 @@ def main():
             C.cudanp_batched_loop_reduce_backend(Xi4, inii, S=S, backend=be)
     for th in (1, 4, 16):  # ragged reduce with the team size chosen per segment
         C.cudanp_ragged_loop_reduce_adaptive(xr, off, threshold=th)
-    # warp-streamed spans + segmented scan: short tiles, multi-row spans, long tiles (adaptive
-    # fallback), a base pointer off 16 bytes and more tiles than one persistent wave
-    for lens_mean, dist, N in ((16, "exp", 150000), (30, "uniform", 300), (900, "exp", 70)):
-        offs = dev(synth.offsets_from_lengths(synth.lengths(N, lens_mean, dist)))
-        xs = dev(synth.gen(1, "f32_unit", 0, int(offs[-1].item()) + 4))
-        for base in (0, 1):
-            C.cudanp_ragged_loop_reduce_streamed(xs[base:], offs, threshold=64)
-            C.cudanp_ragged_loop_reduce_streamed(xs[base:], offs, op=C.MAX, threshold=64)
     for S in (64, 256, 1024):  # multi-warp teams
         for d in (C.CYCLIC, C.BLOCK):
             for X, ini in ((Xf, inif), (Xi, inii)):

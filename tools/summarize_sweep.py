@@ -75,7 +75,7 @@ def main(path, out=None):
         lines += [f"| {r['config']} | {r['op']}{(' ' + r['opname']) if r.get('opname') else ''} | {r['dtype']} | "
                   f"{r['L']} | {r['S']} | {r['dist']} | {r['gbs']:.0f} | {r['S_padded']} | {r['gbs_padded']:.0f} | "
                   f"{r['speedup_vs_padded']:.2f}x |" for r in f12]
-    rv = [r for r in recs if r["config"] == "R1" and str(r["impl"]).startswith(("adaptive", "streamed"))]
+    rv = [r for r in recs if r["config"] == "R1" and str(r["impl"]).startswith("adaptive")]
     if rv:
         lines += ["", "R1 — ragged versions beside the swept NP kernels (GB/s; x = time of the best NP / its time)", "",
                   "| L | impl | GB/s | % HBM | vs best NP |", "|---|---|---|---|---|"]

@@ -396,9 +396,6 @@ def r1(means=(16, 64, 256, 1024)):
             for th in (64, 128, 256, 512):  # adaptive team size per segment
                 comps.append((f"adaptive_t{th}", time_ms(
                     lambda: C.cudanp_ragged_loop_reduce_adaptive(x, off, None, out, threshold=th))[0]))
-            for th in (64, 256):  # warp-streamed spans + segmented scan (long tiles: adaptive)
-                comps.append((f"streamed_t{th}", time_ms(
-                    lambda: C.cudanp_ragged_loop_reduce_streamed(x, off, None, out, threshold=th))[0]))
             sweep_np("R1", "ragged_reduce", nb,
                      lambda S, d, m: time_ms(lambda: C.cudanp_ragged_loop_reduce(x, off, None, out, S=S, dist=d, map=m)),
                      {"dtype": "f32", "N": N, "L": f"{dist}{mean}"}, literal=lit, comps=comps,
