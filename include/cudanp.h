@@ -335,7 +335,8 @@ int cudanp_launch_info(int op_kind, int64_t n_outer, int64_t n_inner, int dtype,
 /* The (S, dist, map) that S = CUDANP_S_AUTO selects for op_kind (0 tmv, 1 mv,
  * 2 reduce, 3 scan) on N = n_outer items of L = n_inner iterations, given
  * `map` (AUTO, or a map to keep) and vec4 as above.  Rule:
- * TMV with 0.3..1.1 128-column strips per SM -> TMA S = 8 cyclic; wider ->
+ * TMV with 0.3..1.1 128-column strips per SM -> TMA S = 8 cyclic (with vec4
+ * only from 0.75 strips per SM, below that the S = 128 inter rule); wider ->
  * inter-warp S = 32 block; narrower -> inter-warp S = 128 with vec4 (else
  * clamp(2*SMs*1024/N, 8, 64)), block when L/S < 32 (and N > 1024 with
  * vec4), else cyclic;

@@ -167,8 +167,9 @@ static bool tma_ok(const float* A, int64_t lda, int64_t w, int64_t h) {
 // anything.  T = SMs x 1024 threads is "enough threads to fill the GPU":
 // when N x S falls short, the team grows (NP pays when outer
 // TLP is short), up to a team whose slaves still get >= 8 elements each.
-//   TMV: tmv_wide + TMA-able -> TMA, S = 8 cyclic (C2 best); wider than that
-//        -> LDG inter-warp S = 32 block; narrower -> LDG inter-warp with
+//   TMV: tmv_wide + TMA-able -> TMA, S = 8 cyclic (C2 best), except below
+//        0.75 strips per SM on aligned matrices (-> the S = 128 rule below);
+//        wider than that -> LDG inter-warp S = 32 block; narrower -> LDG inter-warp with
 //        S = 128 when 16-byte aligned (else clamp(2T / w, 8, 64)), block when
 //        each slave's share is < 32 rows and w > 1024, cyclic otherwise (C1:
 //        128 cyclic; profiles/tmv_narrow_new_r02a[ef].jsonl: S = 128 best for
@@ -188,8 +189,13 @@ int choose_version(int op_kind, int64_t N, int64_t L, bool vec, bool tma, int ma
   const int cap_l8 = clampi(floor_pow2(L / 8), 1, 1024);
   int s = 1, d = CUDANP_DIST_CYCLIC, m = map_in;
   switch (op_kind) {
-    case 0:  // TMV: N = w columns, L = h rows
-      if ((map_in == CUDANP_MAP_AUTO || map_in == CUDANP_MAP_INTER_WARP_TMA) && tma && tmv_wide(N)) {
+    case 0: {  // TMV: N = w columns, L = h rows
+      // the lower part of the TMA band goes to the 128-bit S = 128 LDG team
+      // when the matrix is aligned (width sweep r02ak: w = 8192 / 12288
+      // 6987 / 6790 vs 6272 / 6617 GB/s for the best TMA version)
+      const bool lower = vec && 4 * ((N + 127) / 128) < 3 * (int64_t)sm_count();
+      if (tma && tmv_wide(N) &&
+          (map_in == CUDANP_MAP_INTER_WARP_TMA || (map_in == CUDANP_MAP_AUTO && !lower))) {
         s = 8; d = CUDANP_DIST_CYCLIC; m = CUDANP_MAP_INTER_WARP_TMA;
         break;
       }
@@ -208,6 +214,7 @@ int choose_version(int op_kind, int64_t N, int64_t L, bool vec, bool tma, int ma
       if (m == CUDANP_MAP_INTER_WARP && s != 32)
         d = L / s < 32 && (!vec || N > 1024) ? CUDANP_DIST_BLOCK : CUDANP_DIST_CYCLIC;
       break;
+    }
     case 1:  // MV
       if (m == CUDANP_MAP_INTER_WARP) {
         s = clampi(floor_pow2(L / 128), 1, 32);

@@ -97,7 +97,10 @@ def test_auto_team_size_rule(lib):
     assert ch("tmv", 2048, 1024) == (128, C.BLOCK, C.INTER_WARP)
     assert ch("tmv", 4096, 16384) == (128, C.CYCLIC, C.INTER_WARP)
     assert ch("tmv", 1024, 1024, vec4=False) == (64, C.BLOCK, C.INTER_WARP)
-    assert ch("tmv", 8192, 65536) == (8, C.CYCLIC, C.INTER_WARP_TMA)   # C5 shard at G = 8
+    assert ch("tmv", 8192, 65536) == (128, C.CYCLIC, C.INTER_WARP)    # C5 shard at G = 8
+    assert ch("tmv", 8192, 65536, map=C.INTER_WARP_TMA) == (8, C.CYCLIC, C.INTER_WARP_TMA)
+    assert ch("tmv", 12288, 16384) == (128, C.CYCLIC, C.INTER_WARP)
+    assert ch("tmv", 14336, 16384) == (8, C.CYCLIC, C.INTER_WARP_TMA)
     assert ch("tmv", 65536, 65536) == (32, C.BLOCK, C.INTER_WARP)     # C5 at G = 1
     S, d, m = ch("tmv", 16384, 16384, vec4=False)
     assert m == C.INTER_WARP and 8 <= S <= 64

@@ -314,7 +314,7 @@ def test_inter_warp_non_power_of_two_S(S):
 def test_auto_version_parity():
     """S = CUDANP_S_AUTO runs the (S, dist, map) cudanp_choose_version names,
     on every op, with results equal to the oracle's."""
-    for h, w in ((1, 1), (300, 260), (129, 512), (1024, 1024), (2048, 4096)):
+    for h, w in ((1, 1), (300, 260), (129, 512), (1024, 1024), (2048, 4096), (300, 8192), (65, 12288)):
         A = synth.matrix(h, w, "f32_int4")
         xt, xm = synth.vector(h, "f32_int4"), synth.vector(w, "f32_int4")
         assert_exact(host(C.cudanp_tmv(dev(A), dev(xt))), O.tmv(A, xt), f"tmv auto {h}x{w}")

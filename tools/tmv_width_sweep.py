@@ -61,7 +61,7 @@ def main():
             res = {}
             for S, d in itertools.product((4, 8, 16, 32), (C.CYCLIC, C.BLOCK)):
                 res[("tma", S, d)] = t_ms(lambda: C.cudanp_tmv(A, x, y, S=S, dist=d, map=C.INTER_WARP_TMA))
-            for S, d in itertools.product((8, 16, 32, 64), (C.CYCLIC, C.BLOCK)):
+            for S, d in itertools.product((8, 16, 32, 64, 128), (C.CYCLIC, C.BLOCK)):
                 res[("ldg", S, d)] = t_ms(lambda: C.cudanp_tmv(A, x, y, S=S, dist=d, map=C.INTER_WARP))
             res[("auto", 0, 0)] = t_ms(lambda: C.cudanp_tmv(A, x, y))
             bt = min((k for k in res if k[0] == "tma"), key=res.get)
