@@ -15,7 +15,9 @@
 //  cyclic: one box of R rows per stage (TmaShape); slave s owns the box rows
 //          k*S + s, i.e. global rows i = s (mod S) exactly as P:166.
 //  block : S boxes of R/S rows per stage, one from each slave's contiguous
-//          chunk [s*c, (s+1)*c) (c = ceil(h/S)).
+//          chunk [s*c, (s+1)*c) (c = ceil(h/S)).  When S divides h the
+//          tensor map views A as [S chunks][c rows][w columns] and the S
+//          boxes are one 3-D box, one copy instruction per stage (box3d).
 // Rows past h come back zero-filled by TMA and are masked before x is read.
 // A block stage's box may run past the slave's chunk into the next slave's
 // rows (RK need not divide c); those rows are skipped (no FMA), so a
@@ -57,7 +59,7 @@ template <int S> struct TmaMinBlocks {
 template <int S, int DIST, int COLS, int RK>
 __global__ void __launch_bounds__(TmaThreads<S>::value, TmaMinBlocks<S>::value)
 tmv_tma_kernel(const __grid_constant__ CUtensorMap mapA, const float* __restrict__ x,
-               float* __restrict__ y, int64_t w, int64_t h, int stages) {
+               float* __restrict__ y, int64_t w, int64_t h, int stages, int box3d) {
   pdl_entry();
   constexpr bool PW = TmaPW<S>::value;
   constexpr int V = COLS / 32;
@@ -91,6 +93,8 @@ tmv_tma_kernel(const __grid_constant__ CUtensorMap mapA, const float* __restrict
     mbar_expect_tx(&full[st], stage_bytes);
     if (DIST == DIST_CYCLIC) {
       tma_load_2d(dst, &mapA, col0, t * R, &full[st]);
+    } else if (box3d) {
+      tma_load_3d(dst, &mapA, col0, t * RK, 0, &full[st]);
     } else {
       for (int k = 0; k < S; ++k)
         tma_load_2d(dst + k * RK * COLS, &mapA, col0, (int)(k * c + (int64_t)t * RK), &full[st]);
@@ -113,45 +117,68 @@ tmv_tma_kernel(const __grid_constant__ CUtensorMap mapA, const float* __restrict
     for (int t = 0; t < ntiles; ++t) {
       const int st = t % stages;
       // x does not depend on the TMA: issue its loads before waiting on the
-      // stage so their latency hides behind the tile's arrival.
-      float xs[RK];
+      // stage so their latency hides behind the tile's arrival.  Tall block
+      // shares (RK > 16) take x 16 rows at a time, the next chunk's loads in
+      // flight during this chunk's FMAs, so the x registers never outgrow
+      // the budget (RK = 32-128 block spilled 200-424 bytes).
+      constexpr int XC = DIST == DIST_BLOCK && RK > 16 ? 16 : RK;
       // block: is every row of this tile inside the slave's chunk and below h?
       const bool whole = DIST == DIST_CYCLIC ||
                          ((int64_t)(t + 1) * RK <= c && s * c + (int64_t)(t + 1) * RK <= h);
-#pragma unroll
-      for (int kk = 0; kk < RK; ++kk) {
-        int64_t row;
-        bool ok;
-        if (DIST == DIST_CYCLIC) {
-          row = (int64_t)t * R + kk * S + s;   // i = slave_id + k*slave_size
-          ok = row < h;
-        } else {
-          const int64_t k = (int64_t)t * RK + kk;
-          row = s * c + k;                    // R5: slave s owns [s*c, (s+1)*c)
-          ok = k < c && row < h;
-        }
-        xs[kk] = ok ? __ldg(x + row) : 0.f;
-      }
-      mbar_wait(&full[st], (t / stages) & 1);
       const float* tile = tiles + st * R * COLS;
+      auto load_x = [&](float (&xs)[XC], int k0) {
 #pragma unroll
-      for (int kk = 0; kk < RK; ++kk) {
-        const int lr = DIST == DIST_CYCLIC ? kk * S + s : s * RK + kk;
-        const float xv = xs[kk];
-        if (DIST == DIST_BLOCK && !whole) {  // ragged last tile: skip rows outside the chunk
-          const int64_t k = (int64_t)t * RK + kk;
-          if (!(k < c && s * c + k < h)) continue;
+        for (int j = 0; j < XC; ++j) {
+          const int kk = k0 + j;
+          int64_t row;
+          bool ok;
+          if (DIST == DIST_CYCLIC) {
+            row = (int64_t)t * R + kk * S + s;   // i = slave_id + k*slave_size
+            ok = row < h;
+          } else {
+            const int64_t k = (int64_t)t * RK + kk;
+            row = s * c + k;                    // R5: slave s owns [s*c, (s+1)*c)
+            ok = k < c && row < h;
+          }
+          xs[j] = ok ? __ldg(x + row) : 0.f;
         }
-        const float* ap = tile + lr * COLS + lane * V;
-        if constexpr (V == 4) {
-          const float4 a = *reinterpret_cast<const float4*>(ap);
-          acc.x = fmaf(a.x, xv, acc.x); acc.y = fmaf(a.y, xv, acc.y);
-          acc.z = fmaf(a.z, xv, acc.z); acc.w = fmaf(a.w, xv, acc.w);
-        } else if constexpr (V == 2) {
-          const float2 a = *reinterpret_cast<const float2*>(ap);
-          acc.x = fmaf(a.x, xv, acc.x); acc.y = fmaf(a.y, xv, acc.y);
-        } else {
-          acc.x = fmaf(*ap, xv, acc.x);
+      };
+      auto fma_rows = [&](const float (&xs)[XC], int k0) {
+#pragma unroll
+        for (int j = 0; j < XC; ++j) {
+          const int kk = k0 + j;
+          const int lr = DIST == DIST_CYCLIC ? kk * S + s : s * RK + kk;
+          const float xv = xs[j];
+          if (DIST == DIST_BLOCK && !whole) {  // ragged last tile: skip rows outside the chunk
+            const int64_t k = (int64_t)t * RK + kk;
+            if (!(k < c && s * c + k < h)) continue;
+          }
+          const float* ap = tile + lr * COLS + lane * V;
+          if constexpr (V == 4) {
+            const float4 a = *reinterpret_cast<const float4*>(ap);
+            acc.x = fmaf(a.x, xv, acc.x); acc.y = fmaf(a.y, xv, acc.y);
+            acc.z = fmaf(a.z, xv, acc.z); acc.w = fmaf(a.w, xv, acc.w);
+          } else if constexpr (V == 2) {
+            const float2 a = *reinterpret_cast<const float2*>(ap);
+            acc.x = fmaf(a.x, xv, acc.x); acc.y = fmaf(a.y, xv, acc.y);
+          } else {
+            acc.x = fmaf(*ap, xv, acc.x);
+          }
+        }
+      };
+      float xa[XC];
+      load_x(xa, 0);
+      mbar_wait(&full[st], (t / stages) & 1);
+      if constexpr (XC == RK) {
+        fma_rows(xa, 0);
+      } else {
+#pragma unroll
+        for (int k0 = 0; k0 < RK; k0 += XC) {
+          float xb[XC];
+          if (k0 + XC < RK) load_x(xb, k0 + XC);
+          fma_rows(xa, k0);
+#pragma unroll
+          for (int j = 0; j < XC; ++j) xa[j] = xb[j];
         }
       }
       __syncwarp();
@@ -231,12 +258,17 @@ static int launch_tmv_tma_s(const float* A, int64_t lda, const float* x, float* 
     return CUDANP_ERR_CUDA;
   }
   CUtensorMap map;
-  const cuuint64_t dims[2] = {(cuuint64_t)w, (cuuint64_t)h};
-  const cuuint64_t strides[1] = {(cuuint64_t)lda * 4};
-  const cuuint32_t box[2] = {(cuuint32_t)COLS, DIST == DIST_CYCLIC ? (cuuint32_t)R : (cuuint32_t)RK};
-  const cuuint32_t estr[2] = {1, 1};
-  CUresult r = enc(&map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, (void*)A, dims, strides, box, estr,
-                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+  // block distribution with S | h: A as [S][h/S][w], one 3-D box of RK rows
+  // from every chunk per stage
+  const int box3d = DIST == DIST_BLOCK && S > 1 && h % S == 0 ? 1 : 0;
+  const cuuint64_t c = (cuuint64_t)(h / S);
+  const cuuint64_t dims[3] = {(cuuint64_t)w, box3d ? c : (cuuint64_t)h, (cuuint64_t)S};
+  const cuuint64_t strides[2] = {(cuuint64_t)lda * 4, c * (cuuint64_t)lda * 4};
+  const cuuint32_t box[3] = {(cuuint32_t)COLS, DIST == DIST_CYCLIC ? (cuuint32_t)R : (cuuint32_t)RK,
+                             (cuuint32_t)S};
+  const cuuint32_t estr[3] = {1, 1, 1};
+  CUresult r = enc(&map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, box3d ? 3 : 2, (void*)A, dims, strides, box,
+                   estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
                    CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) {
     set_error("cuTensorMapEncodeTiled failed (%d)", (int)r);
@@ -244,7 +276,7 @@ static int launch_tmv_tma_s(const float* A, int64_t lda, const float* x, float* 
   }
   if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess)
     return check_launch("tmv_tma smem attribute");
-  launch_pdl(kern, dim3(grid), dim3(TmaThreads<S>::value), smem, st, map, x, y, w, h, stages);
+  launch_pdl(kern, dim3(grid), dim3(TmaThreads<S>::value), smem, st, map, x, y, w, h, stages, box3d);
   return check_launch("tmv_tma launch");
 }
 
