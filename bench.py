@@ -428,9 +428,23 @@ def run_cudanp(args):
         e2e_ms = max_over_ranks(f0.elapsed_time(f1) / args.e2e_steps, world)
         h2d = A_h.numel() * 4 + (0 if Am_h is A_h else Am_h.numel() * 4) + x_h.numel() * 4
         d2h = (yt_h.numel() + ym_h.numel()) * 4
+        # the PCIe bound of this path: the same pinned H2D copies alone
+        f0.record(st)
+        for _ in range(args.e2e_steps):
+            A_t.copy_(A_h, non_blocking=True)
+            if Am_h is not A_h:
+                A_m.copy_(Am_h, non_blocking=True)
+            x_t.copy_(x_h, non_blocking=True)
+        f1.record(st)
+        torch.cuda.synchronize()
+        copy_ms = max_over_ranks(f0.elapsed_time(f1) / args.e2e_steps, world)
         e2e = {"value": round(total_bytes / (e2e_ms * 1e-3) / 1e9, 3), "unit": "GB/s",
                "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
                "ms_per_step": round(e2e_ms, 4),
+               "h2d_alone_ms": round(copy_ms, 4),
+               "h2d_gbs": round(h2d / (copy_ms * 1e-3) / 1e9, 1),
+               "bound": "PCIe host->device: the step's H2D copies alone take "
+                        f"{100 * copy_ms / e2e_ms:.1f} % of the e2e step",
                "path": "pinned host A,x -> H2D -> cudanp_tmv + cudanp_mv -> D2H y (per rank)"}
         del A_h, Am_h
 
