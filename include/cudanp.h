@@ -306,7 +306,9 @@ int cudanp_dp_memcopy(const float* in, float* out, int64_t total, int64_t m, int
  * under CUDA events on `stream` with the caller's operands (a = A or in,
  * b = x or init, out = y or out; lda for tmv/mv; dtype/op for reduce, dtype
  * for scan), writes the mean ms per launch to ms_table[i] (INFINITY for a
- * combination this shape does not support; ms_table may be NULL) and the
+ * combination this shape does not support, and for a team larger than both
+ * a warp and the loop -- S > 32 and S > n_inner: slaves without a single
+ * iteration, not timed; ms_table may be NULL) and the
  * fastest candidate's index to *best_index.  Synchronizes `stream`.  `out` is
  * overwritten by every candidate (the last run's result is valid). */
 int cudanp_autotune_count(int op_kind);

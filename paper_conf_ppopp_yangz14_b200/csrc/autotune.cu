@@ -92,6 +92,14 @@ int cudanp_autotune(int op_kind, const void* a, const void* b, void* out, int64_
   int rc = CUDANP_OK;
   for (size_t i = 0; i < c.size(); ++i) {
     float ms = INFINITY;
+    if (c[i].S > 32 && c[i].S > n_inner) {
+      // a team larger than both a warp and the loop: slaves without a single
+      // iteration (P:426's idle slaves taken to the extreme) -- not a version
+      // worth timing (C5's 64-element items under 8192-thread cluster teams
+      // took ~6 s per launch)
+      if (ms_table) ms_table[i] = ms;
+      continue;
+    }
     // warm-up launch doubles as the validity check (unsupported combos are skipped)
     int r = run_one(op_kind, c[i], a, b, out, lda, n_outer, n_inner, dtype, op, stream);
     if (r == CUDANP_OK) {

@@ -760,6 +760,9 @@ def test_autotune_picks_a_valid_fastest_version():
     best, table = C.cudanp_autotune("reduce", X, None, out, n_outer=4096, n_inner=96, dtype=C.I32, reps=2)
     assert_exact(host(out), O.reduce(host(X)), "autotune reduce: last run result")
     assert table[(64, C.CYCLIC, C.INTRA_WARP)] != float("inf")  # multi-warp reduce team
+    # teams larger than both a warp and the 96-iteration loop are not timed
+    assert table[(128, C.CYCLIC, C.INTRA_WARP)] == float("inf")
+    assert table[(8192, C.CYCLIC, C.INTRA_WARP)] == float("inf")
     # TMV's candidate list only holds the built combinations (inter-warp for S > 32)
     assert (64, C.CYCLIC, C.INTRA_WARP) not in tables["tmv"]
     assert tables["tmv"][(64, C.CYCLIC, C.INTER_WARP)] != float("inf")
