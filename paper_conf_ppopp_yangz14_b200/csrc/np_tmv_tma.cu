@@ -174,11 +174,14 @@ tmv_tma_kernel(const __grid_constant__ CUtensorMap mapA, const float* __restrict
       } else {
 #pragma unroll
         for (int k0 = 0; k0 < RK; k0 += XC) {
+          const bool more = k0 + XC < RK;
           float xb[XC];
-          if (k0 + XC < RK) load_x(xb, k0 + XC);
+          if (more) load_x(xb, k0 + XC);
           fma_rows(xa, k0);
+          if (more) {
 #pragma unroll
-          for (int j = 0; j < XC; ++j) xa[j] = xb[j];
+            for (int j = 0; j < XC; ++j) xa[j] = xb[j];
+          }
         }
       }
       __syncwarp();
