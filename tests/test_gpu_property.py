@@ -141,3 +141,18 @@ def test_big_and_cluster_teams_random(N, L, S, dist, shift, use_init, seed):
         A = synth.matrix(h, w, "f32_int4", seed=seed)
         xm = synth.vector(w, "f32_int4", seed=seed)
         assert_exact(host(C.cudanp_mv(dev(A), dev(xm), S=S, dist=dist)), O.mv(A, xm), "mv " + what)
+
+
+@settings(max_examples=60, deadline=None, suppress_health_check=list(HealthCheck))
+@given(h=st.integers(0, 3000), w=st.integers(1, 6000), pad=st.integers(0, 5), S=st.sampled_from([64, 128]),
+       dist=D_, seed=st.integers(0, 10**6))
+def test_narrow_tmv_big_teams_random(h, w, pad, S, dist, seed):
+    """TMV S = 64 / 128: every CTA layout the call picks (V = 4 with 4 or 8
+    column-masters, V = 1), the L2 prefetch before the dependency wait, any
+    alignment of the row pitch."""
+    lda = w + pad
+    A = synth.matrix(h, lda, "f32_int4", seed=seed)
+    x = synth.vector(h, "f32_int4", seed=seed)
+    ref = O.tmv(A, x, w) if h else np.zeros(w, np.float32)
+    got = host(C.cudanp_tmv(dev(A), dev(x), S=S, dist=dist, map=C.INTER_WARP, n_outer=w))
+    assert_exact(got, ref, f"narrow TMV h={h} w={w} lda={lda} S={S} dist={dist}")
