@@ -552,6 +552,12 @@ def run_cudanp(args):
         "gpu_launches": 2 * args.steps,
         "clocks": clk,
         "e2e": e2e,
+        # the paper's own speedups (other hardware): context, not a target
+        "paper_context": {"speedup_over_optimized_baseline": {"max": 6.69, "geomean": 2.18,
+                                                              "range_min": 1.36},
+                          "tmv_vs_cublas": 4.9, "tmv_dp_slowdown": 7.61,
+                          "hardware": "GTX 680 (DP: Tesla K20c)",
+                          "source": "PAPER.md P:23, P:41, P:417, P:451, P:482"},
     }
     if c5 is not None:
         line["c5"] = c5
