@@ -16,7 +16,7 @@ from sweep import time_ms  # noqa: E402
 
 C.load()
 N = 1 << 22
-for mean in (16, 64):
+for mean in (16, 64, 256):
     for dist in ("uniform", "exp"):
         off = torch.from_numpy(synth.offsets_from_lengths(synth.lengths(N, mean, dist))).cuda()
         total = int(off[-1].item())
@@ -25,8 +25,9 @@ for mean in (16, 64):
         out = torch.empty(N, device="cuda")
         nb = 4 * total + 8 * (N + 1) + 4 * N
         res = {}
-        for th in (4, 8, 16, 24, 32, 48, 64, 128):
+        for th in (64, 128):
             res[f"adaptive_t{th}"] = time_ms(lambda: C.cudanp_ragged_loop_reduce_adaptive(x, off, None, out, threshold=th))[0]
+        res["balanced"] = time_ms(lambda: C.cudanp_ragged_loop_reduce_balanced(x, off, None, out))[0]
         for S, d, m in ((1, C.CYCLIC, C.INTRA_WARP), (1, C.BLOCK, C.INTER_WARP), (4, C.BLOCK, C.INTRA_WARP)):
             res[f"np_S{S}_{'cyc' if d == C.CYCLIC else 'blk'}_{'intra' if m == C.INTRA_WARP else 'inter'}"] = \
                 time_ms(lambda: C.cudanp_ragged_loop_reduce(x, off, None, out, S=S, dist=d, map=m))[0]
