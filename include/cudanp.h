@@ -208,16 +208,6 @@ int cudanp_ragged_loop_reduce(const void* in, const int64_t* offsets, const void
 int cudanp_ragged_loop_reduce_adaptive(const void* in, const int64_t* offsets, const void* init,
                                        void* out, int64_t n_outer, int dtype, int op,
                                        int64_t threshold, void* stream);
-/* Ragged reduce balanced over the lanes (skewed length mixes): each
- * lane is the master of one segment of the warp's 32 and reads its bounds
- * (P:193), but the tile's elements and segment ends are split evenly over the
- * lanes along the merge path (a binary search over the ends); a lane folds its
- * share and emits a total at each end it meets, the pieces of a segment that
- * spans lanes joined in index order through a segmented scan of the lanes'
- * open partials.  Same result contract as cudanp_ragged_loop_reduce
- * (fp32 sums in another association order). */
-int cudanp_ragged_loop_reduce_balanced(const void* in, const int64_t* offsets, const void* init,
-                                       void* out, int64_t n_outer, int dtype, int op, void* stream);
 /* Comparison: one thread per segment, serial loop (Fig 2 style). */
 int cudanp_ragged_loop_reduce_literal(const void* in, const int64_t* offsets, const void* init,
                                       void* out, int64_t n_outer, int dtype, int op, void* stream);

@@ -41,7 +41,6 @@ int ragged_np(const void*, const int64_t*, const void*, void*, int64_t, int, int
 int ragged_literal(const void*, const int64_t*, const void*, void*, int64_t, int, int, cudaStream_t);
 int ragged_adaptive(const void*, const int64_t*, const void*, void*, int64_t, int, int, int64_t,
                     cudaStream_t);
-int ragged_balanced(const void*, const int64_t*, const void*, void*, int64_t, int, int, cudaStream_t);
 int le_np(const float*, float*, float*, float*, float*, int64_t, int64_t, float, int, int, int, int,
           bool, cudaStream_t);
 int le_tma(const float*, float*, float*, float*, float*, int64_t, int64_t, float, int, int,
@@ -579,13 +578,6 @@ int cudanp_ragged_loop_reduce_adaptive(const void* in, const int64_t* offsets, c
   if (rc) return rc;
   if (threshold < 1) return fail_invalid("threshold must be >= 1");
   return ragged_adaptive(in, offsets, init, out, n_outer, dtype, op, threshold, as_stream(stream));
-}
-
-int cudanp_ragged_loop_reduce_balanced(const void* in, const int64_t* offsets, const void* init,
-                                       void* out, int64_t n_outer, int dtype, int op, void* stream) {
-  int rc = check_ragged(in, offsets, out, n_outer, 1, 0, 0, dtype, op);
-  if (rc) return rc;
-  return ragged_balanced(in, offsets, init, out, n_outer, dtype, op, as_stream(stream));
 }
 
 int cudanp_ragged_loop_reduce_literal(const void* in, const int64_t* offsets, const void* init,

@@ -398,129 +398,6 @@ static int launch_ragged_adaptive(const T* in, const int64_t* off, const T* init
   return check_launch("ragged_loop_reduce (adaptive teams) launch");
 }
 
-// ---------------------------------------------------------------- balanced (merge path)
-// Skewed length mixes (the exponential R1 mixes, P:340's imbalance): with one
-// master per segment a warp runs as long as its longest segment.  Here the
-// 32 masters of a tile still read their bounds, but the tile's work
-// -- its span's elements and its 32 segment ends, in merge order -- is split
-// evenly over the lanes (each lane finds its start on the merge path by a
-// binary search over the ends).  A lane folds the elements of its share and
-// emits a segment's total at each end it meets; the part of a segment that
-// began in an earlier lane arrives as a carry from a segmented scan of the
-// lanes' open partials (P:209's scan over "has emitted" heads), so every
-// total is folded in index order of its pieces and stored once.
-template <class T, class Op>
-__global__ void __launch_bounds__(kRaggedBlock)
-ragged_balanced_kernel(const T* __restrict__ in, const int64_t* __restrict__ off,
-                       const T* __restrict__ init, T* __restrict__ out, int64_t N) {
-  pdl_entry();
-  constexpr int NW = kRaggedBlock / 32;
-  __shared__ int64_t ends[NW][33];
-  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-  int64_t* es = ends[wid];
-  const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
-  const int64_t ntiles = (N + 31) / 32;
-  const T id = Op::template identity<T>();
-  for (int64_t t = warp; t < ntiles; t += nwarps) {
-    const int64_t n0 = t * 32, item = n0 + lane;
-    const int cnt = (int)(N - n0 < 32 ? N - n0 : 32);
-    int64_t b = 0, e = 0;
-    if (item < N) {  // the master's sequential section: its loop bounds
-      b = off[item];
-      e = off[item + 1];
-    }
-    const int64_t B = __shfl_sync(kFull, b, 0);
-    const bool mono = __all_sync(kFull, item >= N || e >= b);
-    T res = id;
-    if (!mono) {  // decreasing bounds (empty loops by contract): each master alone
-      for (int64_t i = b; i < e; ++i) res = Op::apply(res, ldg1(in + i));
-    } else {
-      const int64_t E = __shfl_sync(kFull, e, cnt - 1) - B;  // the tile's span
-      __syncwarp();
-      es[lane] = (lane < cnt ? e : B + E) - B;              // relative ends
-      __syncwarp();
-      const int64_t W = E + cnt;                            // merge-path length
-      const int64_t per = (W + 31) / 32;
-      // merge-path search: the split (k, p = d - k) of diagonal d takes end k
-      // before element p iff ends[k] <= p
-      auto split = [&](int64_t d) {
-        int64_t lo = d - E > 0 ? d - E : 0, hi = d < cnt ? d : cnt;
-        while (lo < hi) {
-          const int64_t mid = (lo + hi) >> 1;
-          if (es[mid] > d - mid - 1) hi = mid; else lo = mid + 1;
-        }
-        return lo;
-      };
-      const int64_t d0 = (int64_t)lane * per < W ? (int64_t)lane * per : W;
-      const int64_t d1 = d0 + per < W ? d0 + per : W;
-      int64_t k = split(d0);
-      const int64_t k1 = split(d1);
-      int64_t p = d0 - k;
-      const int64_t p1 = d1 - k1;
-      T acc = id, first_acc = id;
-      int64_t first_k = -1;
-      int64_t next_end = k < k1 ? es[k] : INT64_MAX;
-      auto emit = [&]() {
-        if (first_k < 0) { first_k = k; first_acc = acc; }
-        else out[n0 + k] = init ? Op::apply(init[n0 + k], acc) : acc;
-        acc = id;
-        ++k;
-        next_end = k < k1 ? es[k] : INT64_MAX;
-      };
-      // elements in 16-byte units where the span is aligned to them
-      const T* base = in + B;
-      for (; p < p1; ++p) {
-        while (next_end <= p) emit();
-        acc = Op::apply(acc, ldg1(base + p));
-      }
-      while (k < k1) emit();
-      // carries: a segmented inclusive scan of the lanes' open partials,
-      // restarting at every lane that emitted
-      T c = acc;
-      bool f = first_k >= 0;
-#pragma unroll
-      for (int o = 1; o < 32; o <<= 1) {
-        const T cu = __shfl_up_sync(kFull, c, o);
-        const bool fu = __shfl_up_sync(kFull, (int)f, o);
-        if (lane >= o) {
-          if (!f) c = Op::apply(cu, c);
-          f = f || fu;
-        }
-      }
-      T cin = __shfl_up_sync(kFull, c, 1);
-      if (lane == 0) cin = id;
-      if (first_k >= 0) {
-        const T v = Op::apply(cin, first_acc);
-        out[n0 + first_k] = init ? Op::apply(init[n0 + first_k], v) : v;
-      }
-      continue;
-    }
-    if (item < N) out[item] = init ? Op::apply(init[item], res) : res;
-  }
-}
-
-template <class T, class Op>
-static int launch_ragged_balanced(const T* in, const int64_t* off, const T* init, T* out, int64_t N,
-                                  cudaStream_t st) {
-  if (N == 0) return CUDANP_OK;
-  auto kern = ragged_balanced_kernel<T, Op>;
-  const int64_t grid = persistent_grid(kern, kRaggedBlock, 0, (N + kRaggedBlock - 1) / kRaggedBlock);
-  launch_pdl(kern, dim3((unsigned)grid), dim3(kRaggedBlock), 0, st, in, off, init, out, N);
-  return check_launch("ragged_loop_reduce (balanced) launch");
-}
-
-int ragged_balanced(const void* in, const int64_t* off, const void* init, void* out, int64_t N,
-                    int dtype, int op, cudaStream_t st) {
-  if (dtype == CUDANP_F32)
-    return op == CUDANP_SUM
-               ? launch_ragged_balanced<float, OpSum>((const float*)in, off, (const float*)init, (float*)out, N, st)
-               : launch_ragged_balanced<float, OpMax>((const float*)in, off, (const float*)init, (float*)out, N, st);
-  return op == CUDANP_SUM
-             ? launch_ragged_balanced<int32_t, OpSum>((const int32_t*)in, off, (const int32_t*)init, (int32_t*)out, N, st)
-             : launch_ragged_balanced<int32_t, OpMax>((const int32_t*)in, off, (const int32_t*)init, (int32_t*)out, N, st);
-}
-
 int ragged_adaptive(const void* in, const int64_t* off, const void* init, void* out, int64_t N,
                     int dtype, int op, int64_t thresh, cudaStream_t st) {
   if (dtype == CUDANP_F32)

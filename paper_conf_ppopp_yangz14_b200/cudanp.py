@@ -54,7 +54,6 @@ _SIGS = {
     "cudanp_ragged_loop_reduce": [_vp, _vp, _vp, _vp, _i64, _int, _int, _int, _int, _int, _vp],
     "cudanp_ragged_loop_reduce_literal": [_vp, _vp, _vp, _vp, _i64, _int, _int, _vp],
     "cudanp_ragged_loop_reduce_adaptive": [_vp, _vp, _vp, _vp, _i64, _int, _int, _i64, _vp],
-    "cudanp_ragged_loop_reduce_balanced": [_vp, _vp, _vp, _vp, _i64, _int, _int, _vp],
     "cudanp_le_gicov": [_vp, _vp, _vp, _vp, _vp, _i64, _i64, ctypes.c_float, _int, _int, _int,
                         _int, _vp],
     "cudanp_le_gicov_placement": [_vp, _vp, _vp, _vp, _vp, _i64, _i64, ctypes.c_float, _int, _int,
@@ -382,18 +381,6 @@ def cudanp_ragged_loop_reduce_adaptive(x, offsets, init=None, out=None, *, op=SU
     _check(load().cudanp_ragged_loop_reduce_adaptive(_ptr(x), _ptr(offsets), _ptr(init), _ptr(out), N,
                                                      _dtype_code(x), op, threshold, _stream(stream)),
            "cudanp_ragged_loop_reduce_adaptive")
-    return out
-
-
-def cudanp_ragged_loop_reduce_balanced(x, offsets, init=None, out=None, *, op=SUM, stream=None):
-    """Ragged reduce with the tile's work split evenly over the lanes (merge path)."""
-    import torch
-    N = _ragged_args(x, offsets, init, out, "cudanp_ragged_loop_reduce_balanced")
-    if out is None:
-        out = torch.empty(N, dtype=x.dtype, device=x.device)
-    _check(load().cudanp_ragged_loop_reduce_balanced(_ptr(x), _ptr(offsets), _ptr(init), _ptr(out), N,
-                                                     _dtype_code(x), op, _stream(stream)),
-           "cudanp_ragged_loop_reduce_balanced")
     return out
 
 

@@ -125,37 +125,3 @@ def test_ragged_adaptive_parity(kind, op, exact):
     with pytest.raises(C.CudanpError):
         C.cudanp_ragged_loop_reduce_adaptive(dev(synth.gen(1, "i32_full", 0, 8)),
                                              dev(synth.offsets_from_lengths(np.array([3, 5]))), threshold=0)
-
-
-@pytest.mark.parametrize("kind,op,exact", [("i32_full", C.SUM, True), ("i32_full", C.MAX, True),
-                                           ("f32_signed", C.MAX, True), ("f32_int4", C.SUM, True),
-                                           ("f32_unit", C.SUM, False)])
-def test_ragged_balanced_parity(kind, op, exact):
-    """Merge-path split of each tile's work over the lanes: segments spanning
-    several lanes, empty segments, partial last tiles, every alignment,
-    base pointers off 16 bytes, long and skewed mixes, decreasing bounds."""
-    for N, mean, dist in CASES + [(3000, 90, "exp"), (40, 5000, "exp"), (5003, 16, "exp"),
-                                  (4096, 16, "uniform"), (2000, 1, "exp"), (999, 30, "uniform")]:
-        lens = synth.lengths(N, mean, dist, seed=N + mean + 2)
-        off = synth.offsets_from_lengths(lens)
-        for shift, base in ((0, 0), (1, 0), (3, 0), (0, 1), (2, 3)):
-            x = synth.gen(1, kind, 0, int(off[-1]) + 8)
-            offs = off + shift
-            ini = synth.init(N, kind)
-            ref_i = O.ragged_reduce(x[base:], offs, op=op, init=ini)
-            ref = O.ragged_reduce(x[base:], offs, op=op)
-            xd, od, inid = dev(x)[base:], dev(offs), dev(ini)
-            what = f"balanced {kind} op={op} N={N} mean={mean} shift={shift} base={base}"
-            got_i = host(C.cudanp_ragged_loop_reduce_balanced(xd, od, inid, op=op))
-            got = host(C.cudanp_ragged_loop_reduce_balanced(xd, od, op=op))
-            if exact:
-                assert_exact(got_i, ref_i, what)
-                assert_exact(got, ref, what + " no init")
-            else:
-                Lmax = int(lens.max()) if N else 1
-                assert_rel(got_i, ref_i, Lmax, what)
-                nz = lens > 0
-                assert_rel(got[nz], ref[nz], Lmax, what + " no init")
-    x = dev(np.arange(8, dtype=np.int32))
-    off = dev(np.array([0, 5, 3, 8], np.int64))
-    assert host(C.cudanp_ragged_loop_reduce_balanced(x, off)).tolist() == [10, 0, 25]

@@ -27,7 +27,6 @@ for mean in (16, 64, 256):
         res = {}
         for th in (64, 128):
             res[f"adaptive_t{th}"] = time_ms(lambda: C.cudanp_ragged_loop_reduce_adaptive(x, off, None, out, threshold=th))[0]
-        res["balanced"] = time_ms(lambda: C.cudanp_ragged_loop_reduce_balanced(x, off, None, out))[0]
         for S, d, m in ((1, C.CYCLIC, C.INTRA_WARP), (1, C.BLOCK, C.INTER_WARP), (4, C.BLOCK, C.INTRA_WARP)):
             res[f"np_S{S}_{'cyc' if d == C.CYCLIC else 'blk'}_{'intra' if m == C.INTRA_WARP else 'inter'}"] = \
                 time_ms(lambda: C.cudanp_ragged_loop_reduce(x, off, None, out, S=S, dist=d, map=m))[0]
