@@ -42,6 +42,7 @@ CASES = [
     ("C1 TMV 1024²", "S=1 TMA (no NP)", "--op tmv --n 1024 --S 1 --dist cyclic --map inter_tma", "tmv_"),
     ("C1 TMV 1024²", "NP S=32 cyclic inter", "--op tmv --n 1024 --S 32 --dist cyclic --map inter", "tmv_"),
     ("C1 TMV 1024²", "NP S=64 block inter", "--op tmv --n 1024 --S 64 --dist block --map inter", "tmv_"),
+    ("C1 TMV 1024²", "NP S=128 cyclic inter (V=4, 4 masters)", "--op tmv --n 1024 --S 128 --dist cyclic --map inter", "tmv_"),
     ("C2 MV 16384²", "S=1 inter (no NP)", "--op mv --S 1 --dist cyclic --map inter", "mv_"),
     ("C2 MV 16384²", "literal", "--op mv_literal", "mv_"),
     ("C2 MV 16384²", "S=1 TMA-tiled (no NP; SMM-style)", "--op mv_tiled", "mv_"),
